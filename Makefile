@@ -1,0 +1,41 @@
+# Builds every native artefact in-tree (the .so files travel to the GPU box
+# with the gpurun snapshot).  `__graft_entry__.build()` runs `make`.
+#
+#   oracle/liboracle.so   CPU oracle (test infrastructure only)
+#   synth/libsynth.so     seeded synthetic frames (tests + bench)
+#   paper_conf_icpp_fanjzac15_b200/libsharp.so   the product: sm_100a kernels + C ABI
+
+NVCC     ?= /usr/local/cuda/bin/nvcc
+CUDA_HOME ?= /usr/local/cuda
+HOSTCC   := /usr/bin/gcc
+PKG      := paper_conf_icpp_fanjzac15_b200
+ARCH     := -gencode arch=compute_100a,code=sm_100a
+
+ORACLE_CFLAGS := -std=c11 -O2 -ffp-contract=off -fno-fast-math -fopenmp -fPIC -shared -Wall -Wextra
+SYNTH_CFLAGS  := -std=c11 -O2 -fopenmp -fPIC -shared -Wall -Wextra
+
+# --fmad=false: no implicit FMA contraction; every fused multiply-add in the
+# kernels is an explicit __fmaf_rn / fma.rn (bit-exact parity, R15).
+NVCC_FLAGS := $(ARCH) -O3 -lineinfo -std=c++17 --fmad=false -Xptxas -v \
+              -Xcompiler -fPIC,-O2,-Wall -I include -I $(PKG)/csrc
+
+SHARP_SRCS := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
+SHARP_HDRS := $(wildcard $(PKG)/csrc/*.cuh) $(wildcard $(PKG)/csrc/*.h) include/sharp.h
+
+all: oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so
+
+oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
+	$(HOSTCC) $(ORACLE_CFLAGS) -o $@ oracle/oracle.c -lm
+
+synth/libsynth.so: synth/synth.c
+	$(HOSTCC) $(SYNTH_CFLAGS) -o $@ synth/synth.c
+
+$(PKG)/libsharp.so: $(SHARP_SRCS) $(SHARP_HDRS)
+	$(NVCC) $(NVCC_FLAGS) -shared -o $@ $(SHARP_SRCS) 2> build/ptxas.log || (cat build/ptxas.log; false)
+
+$(shell mkdir -p build)
+
+clean:
+	rm -f oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so
+
+.PHONY: all clean

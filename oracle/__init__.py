@@ -1,0 +1,163 @@
+"""ctypes wrapper of the CPU oracle (oracle.c).
+
+TEST INFRASTRUCTURE ONLY: imported by tests/, __graft_entry__.smoke() and the
+cpu_baseline / --impl reference legs of bench.py -- never by the product
+package paper_conf_icpp_fanjzac15_b200/.
+"""
+import ctypes
+import os
+
+import numpy as np
+
+_here = os.path.dirname(os.path.abspath(__file__))
+_lib = None
+
+_P = ctypes.c_void_p
+_I = ctypes.c_int
+_F = ctypes.c_float
+_D = ctypes.c_double
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        path = os.path.join(_here, "liboracle.so")
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} missing: run `make` (or __graft_entry__.build())")
+        lib = ctypes.CDLL(path)
+        sigs = {
+            "oracle_check_geometry": ([_I, _I], _I),
+            "oracle_downscale": ([_P, _I, _I, _P], None),
+            "oracle_upscale": ([_P, _I, _I, _P], None),
+            "oracle_upscale_steps": ([_P, _I, _I, _P, _I], None),
+            "oracle_perror": ([_P, _P, _I, _P], None),
+            "oracle_sobel": ([_P, _I, _I, _P], None),
+            "oracle_reduce": ([_P, _I, _I, _P, _P], None),
+            "oracle_strength": ([_P, _I, _D, _F, _F, _P], None),
+            "oracle_preliminary": ([_P, _P, _P, _I, _P], None),
+            "oracle_overshoot": ([_P, _P, _P, _I, _I, _D, _F, _F, _P], None),
+            "oracle_output": ([_P, _I, _P], None),
+            "oracle_sharpen": ([_P, _I, _I, _F, _F, _F, _F, _P, _P, _P], _I),
+            "oracle_sharpen_batch": ([_P, _I, _I, _I, _F, _F, _F, _F, _P, _P, _I], _I),
+        }
+        for name, (args, res) in sigs.items():
+            fn = getattr(lib, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = lib
+    return _lib
+
+
+DEFAULTS = dict(amount=1.0, gamma=0.5, osc_gain=0.5, osc_scale=2.0)  # DESIGN.md R16
+
+
+def _c(a, dtype):
+    a = np.ascontiguousarray(a, dtype=dtype)
+    return a, a.ctypes.data
+
+
+def downscale(O):
+    O, p = _c(O, np.uint8)
+    H, W = O.shape
+    D = np.empty((H // 4, W // 4), np.float32)
+    _load().oracle_downscale(p, W, H, D.ctypes.data)
+    return D
+
+
+def upscale(D, W, H):
+    D, p = _c(D, np.float32)
+    U = np.empty((H, W), np.float32)
+    _load().oracle_upscale(p, W, H, U.ctypes.data)
+    return U
+
+
+def upscale_steps(D, W, H, last_step):
+    D, p = _c(D, np.float32)
+    U = np.empty((H, W), np.float32)
+    _load().oracle_upscale_steps(p, W, H, U.ctypes.data, last_step)
+    return U
+
+
+def perror(O, U):
+    O, po = _c(O, np.uint8)
+    U, pu = _c(U, np.float32)
+    E = np.empty(O.shape, np.float32)
+    _load().oracle_perror(po, pu, O.size, E.ctypes.data)
+    return E
+
+
+def sobel(O):
+    O, p = _c(O, np.uint8)
+    H, W = O.shape
+    pE = np.empty((H, W), np.int32)
+    _load().oracle_sobel(p, W, H, pE.ctypes.data)
+    return pE
+
+
+def reduce(pE):
+    pE, p = _c(pE, np.int32)
+    H, W = pE.shape
+    S = ctypes.c_uint64()
+    mean = ctypes.c_double()
+    _load().oracle_reduce(p, W, H, ctypes.byref(S), ctypes.byref(mean))
+    return S.value, mean.value
+
+
+def strength(pE, mean, amount, gamma):
+    pE, p = _c(pE, np.int32)
+    adj = np.empty(pE.shape, np.float32)
+    _load().oracle_strength(p, pE.size, mean, amount, gamma, adj.ctypes.data)
+    return adj
+
+
+def preliminary(adj, E, U):
+    adj, pa = _c(adj, np.float32)
+    E, pe = _c(E, np.float32)
+    U, pu = _c(U, np.float32)
+    P = np.empty(adj.shape, np.float32)
+    _load().oracle_preliminary(pa, pe, pu, adj.size, P.ctypes.data)
+    return P
+
+
+def overshoot(O, P, pE, mean, osc_gain, osc_scale):
+    O, po = _c(O, np.uint8)
+    P, pp = _c(P, np.float32)
+    pE, pq = _c(pE, np.int32)
+    H, W = O.shape
+    F = np.empty((H, W), np.float32)
+    _load().oracle_overshoot(po, pp, pq, W, H, mean, osc_gain, osc_scale, F.ctypes.data)
+    return F
+
+
+def output(F):
+    F, p = _c(F, np.float32)
+    out = np.empty(F.shape, np.uint8)
+    _load().oracle_output(p, F.size, out.ctypes.data)
+    return out
+
+
+def sharpen(O, amount=1.0, gamma=0.5, osc_gain=0.5, osc_scale=2.0):
+    """Whole pipeline -> (out uint8 [H,W], S, mean).  Raises on invalid input."""
+    O, p = _c(O, np.uint8)
+    H, W = O.shape
+    out = np.empty((H, W), np.uint8)
+    S = ctypes.c_uint64()
+    mean = ctypes.c_double()
+    rc = _load().oracle_sharpen(p, W, H, amount, gamma, osc_gain, osc_scale, out.ctypes.data,
+                                ctypes.byref(S), ctypes.byref(mean))
+    if rc != 0:
+        raise ValueError("oracle_sharpen: invalid geometry or parameters")
+    return out, S.value, mean.value
+
+
+def sharpen_batch(imgs, amount=1.0, gamma=0.5, osc_gain=0.5, osc_scale=2.0, threads=0):
+    """[n,H,W] -> (outs [n,H,W], sums [n] uint64).  Frames split over threads."""
+    imgs, p = _c(imgs, np.uint8)
+    n, H, W = imgs.shape
+    outs = np.empty_like(imgs)
+    sums = np.empty(n, np.uint64)
+    rc = _load().oracle_sharpen_batch(p, n, W, H, amount, gamma, osc_gain, osc_scale,
+                                      outs.ctypes.data, sums.ctypes.data, threads)
+    if rc != 0:
+        raise ValueError("oracle_sharpen_batch: invalid geometry or parameters")
+    return outs, sums
