@@ -1,0 +1,300 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 sharpness pipeline (one JSON line on rank 0).
+
+Workload (BASELINE.json configs[4], frame = configs[1]): a batch of 1024
+synthetic 1920x1080 8-bit frames split across the N GPUs (one process per
+GPU).  A step = the whole hot path (pass 1: Sobel + reduction + LUTs; pass 2:
+fused downscale/upscale/pError/Sobel/min-max/strength/preliminary/overshoot)
+over the whole batch.
+
+  value  : Mpix/s, device-resident (inputs already in HBM), CUDA events on the
+           launch stream, max over ranks.  The 2.1 GB batch is larger than the
+           126 MB L2, so no L2 flush is needed between steps.
+  e2e    : same metric through the public API with HOST (pinned) buffers:
+           sharp_run_batch does H2D || compute || D2H itself.
+  roofline: the dominant kernel (pass 2) -- algorithmic bytes 2 B/px (read
+           the frame, write the result) / its average launch duration.
+  cpu_baseline: the CPU oracle timed on a bounded sample (rank 0, N=1).
+
+`--impl reference` times the CPU oracle (the reference arm of this tier).
+"""
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "megapixels/sec end-to-end sharpen (device-timed) and % of HBM roofline, 1/2/4/8 B200"
+UNIT = "Mpix/s"
+PARAMS = (1.0, 0.5, 0.5, 2.0)  # DESIGN.md R16 defaults
+ALG_BYTES_PER_PX = 2.0         # compulsory: 1 B in + 1 B out
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+class ClockSampler:
+    """Samples SM clock and clock-event reasons with NVML while running."""
+    BITS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+            0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks"}
+
+    def __init__(self, index, period=0.02):
+        self.index, self.period = index, period
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self.ok = True
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.ok = False
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for b, name in self.BITS.items():
+                    if r & b:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"]}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def split(n, world, rank):
+    base, rem = divmod(n, world)
+    start = rank * base + min(rank, rem)
+    return start, base + (1 if rank < rem else 0)
+
+
+def cpu_oracle_rate(frames, threads):
+    """Oracle Mpix/s on `frames` ([k,H,W]) with `threads` OpenMP threads."""
+    import oracle
+    t0 = time.perf_counter()
+    oracle.sharpen_batch(frames, *PARAMS, threads=threads)
+    dt = time.perf_counter() - t0
+    return frames.size / dt / 1e6, dt
+
+
+def run_reference(args, world, rank):
+    """Reference arm of this tier: the CPU oracle, as it stands, on host cores."""
+    if rank != 0:
+        return
+    import synth
+    cores = len(os.sched_getaffinity(0))
+    sample = args.ref_sample
+    idx = list(range(0, args.frames, max(1, args.frames // sample)))[:sample]
+    frames = np.stack([synth.image(args.width, args.height, "natural", seed=synth.BASE_SEED + 5 + i) for i in idx])
+    for _ in range(args.warmup):
+        cpu_oracle_rate(frames[:1], cores)
+    rates, times = [], []
+    for _ in range(args.steps):
+        r, dt = cpu_oracle_rate(frames, cores)
+        rates.append(r)
+        times.append(dt)
+    value = float(np.median(rates))
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(np.median(times) * 1e3),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic", "config": workload_config(args, world),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"{len(idx)} of {args.frames} frames per step (every "
+                                   f"{max(1, args.frames // sample)}th), OpenMP over frames"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(args, world):
+    return {"workload": f"{args.frames} x {args.width}x{args.height} u8 frames (BASELINE configs[4]; "
+                        f"frame = configs[1])",
+            "frames": args.frames, "width": args.width, "height": args.height,
+            "params": dict(zip(["amount", "gamma", "osc_gain", "osc_scale"], PARAMS)),
+            "parallelism": f"frames split over {world} GPU(s), no collective on the data path",
+            "l2": "batch (2.1 GB in + out) > 126 MB L2: no flush needed between steps"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--frames", type=int, default=1024)
+    ap.add_argument("--width", type=int, default=1920)
+    ap.add_argument("--height", type=int, default=1080)
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--cpu-sample", type=int, default=32)
+    ap.add_argument("--ref-sample", type=int, default=16)
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    world, rank, local = dist_setup()
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_icpp_fanjzac15_b200 import Sharpener
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    W, H = args.width, args.height
+    start, n = split(args.frames, world, rank)
+    fb = W * H
+    # Inputs: pinned host (for e2e) and a device copy (device-resident value).
+    h_in = torch.empty((n, H, W), dtype=torch.uint8).pin_memory()
+    synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 5 + start, out=h_in.numpy())
+    h_out = torch.empty_like(h_in).pin_memory()
+    d_in = h_in.to(f"cuda:{local}")
+    d_out = torch.empty_like(d_in)
+    stream = torch.cuda.current_stream()
+    sh = Sharpener(device=local)
+    sh.set_stream(stream)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=f"cuda:{local}")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---- device-resident timed region
+    for _ in range(args.warmup):
+        sh.enqueue_batch(d_in, d_out, PARAMS)
+    torch.cuda.synchronize()
+    launches_per_step = sh.stats().kernels
+    sh.set_profiling(True)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            sh.enqueue_batch(d_in, d_out, PARAMS)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    barrier()
+    ms_step = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
+    kt = sh.kernel_times()
+    sh.set_profiling(False)
+    total_px = args.frames * fb
+    value = total_px / (ms_step * 1e-3) / 1e6
+
+    # dominant kernel: pass 2 (sharpen); pass-1 share reported beside it
+    px_per_launch = kt.pixels / max(1, kt.pass1_launches)
+    p2_avg_ms = kt.pass2_ms / max(1, kt.pass2_launches)
+    p1_avg_ms = kt.pass1_ms / max(1, kt.pass1_launches)
+    pk, pk_src = peaks()
+    peak = float(pk["hbm_gbs"])
+    achieved = ALG_BYTES_PER_PX * px_per_launch / (p2_avg_ms * 1e-3) / 1e9
+    step_achieved = ALG_BYTES_PER_PX * total_px / world / (ms_step * 1e-3) / 1e9
+
+    # ---- parity spot check of this run's outputs (two frames, vs the oracle)
+    parity = None
+    if rank == 0 and not args.no_cpu:
+        import oracle
+        chk = [0, n - 1]
+        ref, _ = oracle.sharpen_batch(h_in.numpy()[chk], *PARAMS)
+        got = d_out[chk].cpu().numpy()
+        parity = {"frames_checked": len(chk), "mismatched_pixels": int((got != ref).sum())}
+
+    # ---- e2e through the public API with host (pinned) buffers
+    sh.set_stream(None)
+    sh.run_batch(h_in, PARAMS, h_out)  # warm the staging buffers
+    barrier()
+    t_e2e = []
+    for _ in range(args.e2e_steps):
+        barrier()
+        t0 = time.perf_counter()
+        sh.run_batch(h_in, PARAMS, h_out)
+        t_e2e.append(time.perf_counter() - t0)
+    e2e_ms = max_over_ranks(float(np.median(t_e2e)) * 1e3)
+    e2e_value = total_px / (e2e_ms * 1e-3) / 1e6
+
+    # ---- CPU oracle baseline (rank 0, N=1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cores = len(os.sched_getaffinity(0))
+        idx = list(range(0, n, max(1, n // args.cpu_sample)))[:args.cpu_sample]
+        rate, dt = cpu_oracle_rate(h_in.numpy()[idx], cores)
+        cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{len(idx)} of {n} frames (every {max(1, n // args.cpu_sample)}th), "
+                         f"{dt:.1f} s wall on {cores} threads"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": workload_config(args, world),
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": None,
+                         "kernel": "sharpen_kernel (pass 2)", "peak_source": pk_src,
+                         "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px_per_launch,
+                         "pass2_avg_ms": p2_avg_ms, "pass1_avg_ms": p1_avg_ms,
+                         "pass2_share": kt.pass2_ms / max(1e-9, kt.pass1_ms + kt.pass2_ms),
+                         "step_frac": step_achieved / peak},
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": total_px // world,
+                    "d2h_bytes_per_step": total_px // world, "ms_per_step": e2e_ms,
+                    "api": "sharp_run_batch(pinned host in, pinned host out)"},
+            "gpu_launches": launches_per_step * args.steps,
+            "clocks": clk.summary(),
+            "cpu_baseline": cpu,
+            "parity": parity,
+        }
+        print(json.dumps(line), flush=True)
+    sh.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,147 @@
+/*
+ * include/sharp.h -- C ABI of the B200-native sharpness pipeline
+ * (libsharp.so, built from paper_conf_icpp_fanjzac15_b200/csrc/).
+ *
+ * Method: M. Fan et al., "Optimizing Image Sharpening Algorithm on GPU",
+ * ICPP 2015, section III: downscale (L130) -> upscale
+ * border + body (L140-L146) -> pError (L148) -> Sobel pEdge (L158-L172) ->
+ * global mean of pEdge (L174, the one global reduction) -> brightness
+ * strength / adjusted pEdge (L178) -> preliminary sharpened image (L178) ->
+ * overshoot control (L180-L212, Fig. 8) -> 8-bit image.  The readings of the
+ * places where the paper is silent (R1..R16) are listed in DESIGN.md sec. 3;
+ * the results are bit-identical to the CPU oracle in oracle/ (tests/).
+ *
+ * Conventions (all entry points):
+ *  - Images are 8-bit single-channel, dense row-major, pitch == width
+ *    ("4096 x 4096 bytes").  A batch is dense [n][h][w].
+ *  - Width and height must be multiples of 4 and >= 8 (R1: the downscaled
+ *    matrix is width/4 x height/4, L130); otherwise SHARP_EINVAL.
+ *  - Pointers may be device pointers (on the context's device), pinned host
+ *    or pageable host memory; the library classifies them
+ *    (cudaPointerGetAttributes).  Host pointers go through pinned staging with
+ *    H2D / compute / D2H overlapped across streams (sec. V-A).
+ *  - Input and output must not overlap (in-place is rejected: the stencils
+ *    read halos), else SHARP_EINVAL.  On any error `out` is left untouched
+ *    unless the error is SHARP_ECUDA (device state unknown).
+ *  - Ownership: the caller owns every image buffer; the library never retains
+ *    them past return and never frees them.  The context owns all device
+ *    scratch, streams, events and pinned staging; sharp_destroy releases them.
+ *  - Synchrony: sharp_run / sharp_run_batch / sharp_run_bands return after the
+ *    output is complete.  sharp_enqueue_batch is asynchronous on the
+ *    context's stream (device pointers only).
+ *  - Threads: a context is used by one thread at a time.
+ *  - After a sticky CUDA error the context is poisoned: every later call
+ *    returns SHARP_ESTATE until sharp_destroy.
+ */
+#ifndef SHARP_H
+#define SHARP_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct sharp_ctx sharp_ctx; /* opaque */
+
+/* "User-defined parameters" of the strength (L178) and of the overshoot
+ * tuning (L210).  Readings R9 / R11:
+ *   adjusted pEdge  adj(p) = amount * (p / m)^gamma,  m = max(mean(pEdge), 1)
+ *   oscStrength     osc(p) = clamp(osc_gain * exp(-p / (osc_scale * m)), 0, 1)
+ * All must be finite and inside the ranges below, else SHARP_EINVAL. */
+typedef struct {
+  float amount;    /* A in [0, 16]       default 1.0 */
+  float gamma;     /* gamma in [0, 4]    default 0.5 */
+  float osc_gain;  /* G in [0, 1]        default 0.5 */
+  float osc_scale; /* K in (0, 1e6]      default 2.0 */
+} sharp_params;
+
+typedef struct {
+  int device;             /* CUDA device ordinal; -1 -> current device          */
+  int max_width;          /* scratch pre-sizing hints; 0 -> grow on demand       */
+  int max_height;
+  int max_frames;
+  int streams;            /* transfer pipeline depth for host buffers; 0 -> 3    */
+  int chunk_frames;       /* frames per pass-1/pass-2 chunk; 0 -> automatic      */
+} sharp_config;
+
+typedef struct {
+  uint64_t edge_sum;  /* S = sum of pEdge over the image (frame 0 of a batch)    */
+  double edge_mean;   /* S / (w*h)                                               */
+  float device_ms;    /* device time of the last call (CUDA events)              */
+  float total_ms;     /* host wall time of the last call                         */
+  int frames;         /* frames processed by the last call                       */
+  int kernels;        /* kernel launches issued by the last call                 */
+} sharp_stats;
+
+enum {
+  SHARP_OK = 0,
+  SHARP_EINVAL = -1,      /* bad argument (geometry, NULL, params, overlap)     */
+  SHARP_ENOMEM = -2,      /* device or pinned allocation failed                 */
+  SHARP_ECUDA = -3,       /* CUDA runtime / launch error                        */
+  SHARP_ENCCL = -4,       /* multi-GPU communication error                      */
+  SHARP_EUNSUPPORTED = -5,/* valid request this build cannot serve              */
+  SHARP_ESTATE = -6       /* context poisoned by an earlier sticky error        */
+};
+
+/* Creates a context on cfg->device (NULL cfg -> defaults).  *ctx is set to
+ * NULL on failure.  Returns SHARP_OK / SHARP_EINVAL / SHARP_ENOMEM / SHARP_ECUDA. */
+int sharp_create(sharp_ctx **ctx, const sharp_config *cfg);
+
+/* Releases everything the context owns.  NULL-safe. */
+void sharp_destroy(sharp_ctx *ctx);
+
+/* Fills *p with the defaults above (R16). */
+void sharp_default_params(sharp_params *p);
+
+/* Kernels are launched on `stream` (a cudaStream_t of the context's device,
+ * e.g. torch.cuda.current_stream().cuda_stream); NULL restores the
+ * context's own stream. */
+int sharp_set_stream(sharp_ctx *ctx, void *stream);
+
+/* One image: img, out are w*h bytes.  params NULL -> defaults. */
+int sharp_run(sharp_ctx *ctx, const uint8_t *img, int w, int h, const sharp_params *params,
+              uint8_t *out);
+
+/* n images, dense [n][h][w] in and out.  Frames are independent: each has its
+ * own pEdge mean.  Host buffers are pipelined through pinned staging. */
+int sharp_run_batch(sharp_ctx *ctx, const uint8_t *imgs, int n, int w, int h,
+                    const sharp_params *params, uint8_t *outs);
+
+/* Asynchronous variant for DEVICE pointers only: enqueues the whole batch on
+ * the context's stream and returns (no host synchronisation; stats.device_ms
+ * is not updated).  Used for graph capture / device-resident benchmarking. */
+int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int h,
+                        const sharp_params *params, uint8_t *d_outs);
+
+/* Statistics of the last completed call. */
+int sharp_get_stats(const sharp_ctx *ctx, sharp_stats *s);
+
+/* Per-frame pEdge sums S of the last run / enqueued batch (waits for the
+ * context's stream).  n must not exceed the number of frames of that call. */
+int sharp_get_batch_sums(sharp_ctx *ctx, uint64_t *sums, int n);
+
+/* Per-kernel device time accounting (CUDA events around every launch, on
+ * the launch stream).  enable != 0 starts (and resets) accounting. */
+typedef struct {
+  float pass1_ms;      /* summed duration of edge_sum launches (Sobel+reduction+LUT) */
+  float pass2_ms;      /* summed duration of sharpen launches (fused per-pixel pass)  */
+  int pass1_launches;
+  int pass2_launches;
+  double pixels;       /* pixels processed by the accounted launches               */
+} sharp_kernel_times;
+int sharp_set_profiling(sharp_ctx *ctx, int enable);
+/* Waits for the launch stream, then returns the accumulated times. */
+int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
+
+/* Static strings. */
+const char *sharp_strerror(int code);
+const char *sharp_last_error(const sharp_ctx *ctx);
+
+/* Library build / kernel information (e.g. "sm_100a ..."). */
+const char *sharp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SHARP_H */

@@ -1,0 +1,278 @@
+"""ctypes binding of include/sharp.h -- same names as the C ABI.
+
+Marshalling only (pointers, sizes, parameter structs).  The library is loaded
+from this package directory (built in-tree by `make`); a missing library is an
+error, never a fallback.
+"""
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+library_path = os.path.join(_HERE, "libsharp.so")
+
+SHARP_OK = 0
+SHARP_EINVAL = -1
+SHARP_ENOMEM = -2
+SHARP_ECUDA = -3
+SHARP_ENCCL = -4
+SHARP_EUNSUPPORTED = -5
+SHARP_ESTATE = -6
+LUT_SIZE = 1536
+
+
+class SharpParams(ctypes.Structure):
+    _fields_ = [("amount", ctypes.c_float), ("gamma", ctypes.c_float),
+                ("osc_gain", ctypes.c_float), ("osc_scale", ctypes.c_float)]
+
+
+class SharpConfig(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("max_width", ctypes.c_int), ("max_height", ctypes.c_int),
+                ("max_frames", ctypes.c_int), ("streams", ctypes.c_int), ("chunk_frames", ctypes.c_int)]
+
+
+class SharpStats(ctypes.Structure):
+    _fields_ = [("edge_sum", ctypes.c_uint64), ("edge_mean", ctypes.c_double),
+                ("device_ms", ctypes.c_float), ("total_ms", ctypes.c_float),
+                ("frames", ctypes.c_int), ("kernels", ctypes.c_int)]
+
+
+class SharpKernelTimes(ctypes.Structure):
+    _fields_ = [("pass1_ms", ctypes.c_float), ("pass2_ms", ctypes.c_float),
+                ("pass1_launches", ctypes.c_int), ("pass2_launches", ctypes.c_int),
+                ("pixels", ctypes.c_double)]
+
+
+_P = ctypes.c_void_p
+_I = ctypes.c_int
+_SIGS = {
+    "sharp_create": ([ctypes.POINTER(_P), ctypes.POINTER(SharpConfig)], _I),
+    "sharp_destroy": ([_P], None),
+    "sharp_default_params": ([ctypes.POINTER(SharpParams)], None),
+    "sharp_set_stream": ([_P, _P], _I),
+    "sharp_run": ([_P, _P, _I, _I, ctypes.POINTER(SharpParams), _P], _I),
+    "sharp_run_batch": ([_P, _P, _I, _I, _I, ctypes.POINTER(SharpParams), _P], _I),
+    "sharp_enqueue_batch": ([_P, _P, _I, _I, _I, ctypes.POINTER(SharpParams), _P], _I),
+    "sharp_get_stats": ([_P, ctypes.POINTER(SharpStats)], _I),
+    "sharp_get_batch_sums": ([_P, _P, _I], _I),
+    "sharp_set_profiling": ([_P, _I], _I),
+    "sharp_get_kernel_times": ([_P, ctypes.POINTER(SharpKernelTimes)], _I),
+    "sharp_strerror": ([_I], ctypes.c_char_p),
+    "sharp_last_error": ([_P], ctypes.c_char_p),
+    "sharp_version": ([], ctypes.c_char_p),
+}
+
+_lib = None
+
+
+def lib():
+    """The loaded libsharp.so (raises if it was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(library_path):
+            raise RuntimeError(f"{library_path} is missing: build it with `make` / __graft_entry__.build(); "
+                               "there is no CPU fallback")
+        L = ctypes.CDLL(library_path)
+        for name, (args, res) in _SIGS.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+class SharpError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"{msg} ({code})")
+        self.code = code
+
+
+def _addr(buf):
+    """Raw address of a torch tensor / numpy array / int (no copies)."""
+    if buf is None:
+        return None
+    if isinstance(buf, int):
+        return buf
+    if hasattr(buf, "data_ptr"):  # torch.Tensor
+        if not buf.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        return buf.data_ptr()
+    if hasattr(buf, "ctypes"):  # numpy
+        if not buf.flags["C_CONTIGUOUS"]:
+            raise ValueError("array must be C-contiguous")
+        return buf.ctypes.data
+    raise TypeError(f"unsupported buffer type {type(buf)}")
+
+
+def _params(p):
+    if p is None:
+        return None
+    if isinstance(p, SharpParams):
+        return p
+    if isinstance(p, dict):
+        d = sharp_default_params()
+        for k, v in p.items():
+            setattr(d, k, float(v))
+        return d
+    return SharpParams(*[float(x) for x in p])
+
+
+def _check(rc, ctx=None):
+    if rc != SHARP_OK:
+        detail = sharp_last_error(ctx) if ctx else ""
+        raise SharpError(rc, f"{sharp_strerror(rc)}: {detail}")
+    return rc
+
+
+# ---------------------------------------------------------------- C-ABI names
+def sharp_create(cfg=None):
+    """-> opaque context handle (int).  cfg: SharpConfig or dict or None."""
+    if isinstance(cfg, dict):
+        c = SharpConfig(device=-1)
+        for k, v in cfg.items():
+            setattr(c, k, int(v))
+        cfg = c
+    h = _P()
+    rc = lib().sharp_create(ctypes.byref(h), ctypes.byref(cfg) if cfg is not None else None)
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_create: {sharp_strerror(rc)}")
+    return h.value
+
+
+def sharp_destroy(ctx):
+    lib().sharp_destroy(ctx)
+
+
+def sharp_default_params():
+    p = SharpParams()
+    lib().sharp_default_params(ctypes.byref(p))
+    return p
+
+
+def sharp_set_stream(ctx, stream):
+    """stream: torch.cuda.Stream, raw cudaStream_t int, or None (context's own)."""
+    s = getattr(stream, "cuda_stream", stream)
+    return _check(lib().sharp_set_stream(ctx, s), ctx)
+
+
+def _pp(params):
+    p = _params(params)
+    return ctypes.byref(p) if p is not None else None
+
+
+def sharp_run(ctx, img, w, h, params, out):
+    return _check(lib().sharp_run(ctx, _addr(img), w, h, _pp(params), _addr(out)), ctx)
+
+
+def sharp_run_batch(ctx, imgs, n, w, h, params, outs):
+    return _check(lib().sharp_run_batch(ctx, _addr(imgs), n, w, h, _pp(params), _addr(outs)), ctx)
+
+
+def sharp_enqueue_batch(ctx, d_imgs, n, w, h, params, d_outs):
+    return _check(lib().sharp_enqueue_batch(ctx, _addr(d_imgs), n, w, h, _pp(params), _addr(d_outs)), ctx)
+
+
+def sharp_get_stats(ctx):
+    s = SharpStats()
+    _check(lib().sharp_get_stats(ctx, ctypes.byref(s)), ctx)
+    return s
+
+
+def sharp_get_batch_sums(ctx, n):
+    arr = (ctypes.c_uint64 * n)()
+    _check(lib().sharp_get_batch_sums(ctx, ctypes.cast(arr, _P), n), ctx)
+    return list(arr)
+
+
+def sharp_set_profiling(ctx, enable):
+    return _check(lib().sharp_set_profiling(ctx, int(bool(enable))), ctx)
+
+
+def sharp_get_kernel_times(ctx):
+    t = SharpKernelTimes()
+    _check(lib().sharp_get_kernel_times(ctx, ctypes.byref(t)), ctx)
+    return t
+
+
+def sharp_strerror(code):
+    return lib().sharp_strerror(code).decode()
+
+
+def sharp_last_error(ctx):
+    return lib().sharp_last_error(ctx).decode()
+
+
+def sharp_version():
+    return lib().sharp_version().decode()
+
+
+# ---------------------------------------------------------------- convenience
+class Sharpener:
+    """Owns one sharp_ctx.  Images: uint8 [H, W] (run) or [N, H, W] (run_batch)."""
+
+    def __init__(self, device=-1, streams=0, chunk_frames=0, max_width=0, max_height=0, max_frames=0):
+        self.ctx = sharp_create(dict(device=device, streams=streams, chunk_frames=chunk_frames,
+                                     max_width=max_width, max_height=max_height, max_frames=max_frames))
+
+    def close(self):
+        if self.ctx:
+            sharp_destroy(self.ctx)
+            self.ctx = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @staticmethod
+    def _shape(x):
+        return tuple(x.shape)
+
+    def _like(self, x):
+        try:
+            import torch
+            if isinstance(x, torch.Tensor):
+                return torch.empty_like(x)
+        except ImportError:
+            pass
+        import numpy as np
+        return np.empty_like(x)
+
+    def set_stream(self, stream):
+        sharp_set_stream(self.ctx, stream)
+
+    def run(self, img, params=None, out=None):
+        H, W = self._shape(img)
+        if out is None:
+            out = self._like(img)
+        sharp_run(self.ctx, img, W, H, params, out)
+        return out
+
+    def run_batch(self, imgs, params=None, out=None):
+        N, H, W = self._shape(imgs)
+        if out is None:
+            out = self._like(imgs)
+        sharp_run_batch(self.ctx, imgs, N, W, H, params, out)
+        return out
+
+    def enqueue_batch(self, d_imgs, d_outs, params=None):
+        N, H, W = self._shape(d_imgs)
+        sharp_enqueue_batch(self.ctx, d_imgs, N, W, H, params, d_outs)
+
+    def stats(self):
+        return sharp_get_stats(self.ctx)
+
+    def batch_sums(self, n):
+        return sharp_get_batch_sums(self.ctx, n)
+
+    def set_profiling(self, enable=True):
+        sharp_set_profiling(self.ctx, enable)
+
+    def kernel_times(self):
+        return sharp_get_kernel_times(self.ctx)

@@ -1,0 +1,460 @@
+// sm_100a kernels of the sharpness pipeline (sec. III).
+//
+// Two passes per chunk of frames (the pEdge mean, L174, is a global
+// dependency of every output pixel):
+//   pass 1  edge_sum_kernel : Sobel (L158-L172) + reduction (L174, sec. V-C)
+//           -> per-CTA u32 partial via warp reductions -> u64 atomic -> the
+//           last CTA of a frame computes the mean and both per-frame lookup
+//           tables (strength L178 / oscStrength L184), "last-block-done".
+//   pass 2  sharpen_kernel  : downscale (L130) + upscale body/border
+//           (L140-L146) + pError (L148) + Sobel + 3x3 max/min (L182) +
+//           strength lookup + preliminary (L178) + overshoot (L180-L212)
+//           -> u8, all in registers (the paper's "sharpness" fusion, L280,
+//           extended to every stage).
+// Chunks are sized so a chunk's input stays in L2 between the passes, so HBM
+// sees ~1 B/px in + 1 B/px out.
+//
+// Work decomposition: a warp owns a 256-column x 32-row tile; each lane owns
+// 8 adjacent columns (two 32-bit words per row) and walks down the rows with a
+// 3-row sliding window in registers.  Pixels are held as f16x2 pairs (even /
+// odd columns of each word) so the Sobel / max / min arithmetic runs two
+// pixels per instruction; all of it is exact (integers < 2048).  Halo
+// columns come from the neighbouring lanes by shuffle.
+//
+// Arithmetic (R15): D, U and pError are exact (dyadic rationals);
+// P = fma(adj, E, U) and the overshoot fma are single-rounding f32, exactly
+// as the oracle; the lookup tables are evaluated in f64 and rounded once.
+#include <cuda_fp16.h>
+#include <stdint.h>
+
+#include "kernels.h"
+
+namespace sharp {
+namespace {
+
+constexpr int kPx = 8;                 // pixels per lane per row
+constexpr int kWarpCols = 32 * kPx;    // 256 columns per warp tile
+constexpr int kTileRows = 32;          // rows per warp tile (multiple of 4)
+constexpr int kWarps = 4;              // warps per CTA
+constexpr int kThreads = kWarps * 32;
+
+// ---------------------------------------------------------------- helpers
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t s) {
+  return __byte_perm(a, b, s);
+}
+__device__ __forceinline__ __half2 H(uint32_t u) {
+  __half2 h;
+  *reinterpret_cast<uint32_t *>(&h) = u;
+  return h;
+}
+__device__ __forceinline__ uint32_t U32(__half2 h) { return *reinterpret_cast<uint32_t *>(&h); }
+__device__ __forceinline__ uint32_t hadd(uint32_t a, uint32_t b) { return U32(__hadd2(H(a), H(b))); }
+__device__ __forceinline__ uint32_t hsub(uint32_t a, uint32_t b) { return U32(__hsub2(H(a), H(b))); }
+__device__ __forceinline__ uint32_t hfma(uint32_t a, uint32_t b, uint32_t c) {
+  return U32(__hfma2(H(a), H(b), H(c)));
+}
+__device__ __forceinline__ uint32_t habsadd(uint32_t a, uint32_t b) {
+  return U32(__hadd2(__habs2(H(a)), __habs2(H(b))));
+}
+// f32 + f16 (sm_100 mixed-precision add, one FHADD): exact here.
+__device__ __forceinline__ float add_f32_f16(uint16_t a, float c) {
+  float d;
+  asm("add.f32.f16 %0, %1, %2;" : "=f"(d) : "h"(a), "f"(c));
+  return d;
+}
+__device__ __forceinline__ uint16_t lo16(uint32_t u) { return (uint16_t)(u & 0xffffu); }
+__device__ __forceinline__ uint16_t hi16(uint32_t u) { return (uint16_t)(u >> 16); }
+__device__ __forceinline__ uint32_t cvt_u8(float a) {  // round-half-even, saturate to [0,255] (R14)
+  uint32_t r;
+  asm("cvt.rni.sat.u8.f32 %0, %1;" : "=r"(r) : "f"(a));
+  return r;
+}
+__device__ __forceinline__ float2 lds_v2(uint32_t addr) {
+  float2 v;
+  asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(addr));
+  return v;
+}
+
+constexpr uint32_t kF16Bias = 0x64646464u;    // byte 0x64 -> f16 exponent of 1024
+constexpr uint32_t kMinus1024 = 0xE400E400u;  // (-1024, -1024) as f16x2
+constexpr uint32_t kTwo = 0x40004000u;        // (2, 2)
+constexpr uint32_t kF16_255 = 0x5BF8u;        // 255.0 as f16
+
+// A row of the lane's 8 pixels plus one halo column each side, as words:
+// pw = columns c0-4..c0-1, w0 = c0..c0+3, w1 = c0+4..c0+7, nw = c0+8..c0+11.
+struct Words {
+  uint32_t pw, w0, w1, nw;
+};
+
+__device__ __forceinline__ uint32_t ldw(const uint8_t *__restrict__ img, int W, int H, int r, int c) {
+  if (r < 0 || r >= H || c < 0 || c >= W) return 0u;  // outside the image: 0
+  return __ldg(reinterpret_cast<const uint32_t *>(img + (size_t)r * W + c));
+}
+
+// All 32 lanes must call this (shuffles).
+__device__ __forceinline__ Words load_row(const uint8_t *__restrict__ img, int W, int H, int r, int c0,
+                                          int lane) {
+  Words x;
+  x.w0 = ldw(img, W, H, r, c0);
+  x.w1 = ldw(img, W, H, r, c0 + 4);
+  x.pw = __shfl_up_sync(0xffffffffu, x.w1, 1);
+  x.nw = __shfl_down_sync(0xffffffffu, x.w0, 1);
+  if (lane == 0) x.pw = ldw(img, W, H, r, c0 - 4);
+  if (lane == 31) x.nw = ldw(img, W, H, r, c0 + 8);
+  return x;
+}
+
+// Pair layout (f16x2, low half first):
+//   p[0] = (c0,   c0+2)   p[1] = (c0+1, c0+3)   p[2] = (c0+4, c0+6)   p[3] = (c0+5, c0+7)
+// Pixel x (0..7) lives in pair kPair[x], half kHalf[x].
+__device__ __forceinline__ int pair_of(int x) { return (x & 1) + ((x >> 2) << 1); }
+__device__ __forceinline__ int half_of(int x) { return (x >> 1) & 1; }
+
+// Per image row: what the 3-row window needs.
+struct RowD {
+  uint32_t h[4];   // right - left neighbour (for Gx)
+  uint32_t s[4];   // left + 2 centre + right (for Gy)
+  uint32_t mx[4];  // max of left/centre/right (u16 order of non-negative f16 == value order)
+  uint32_t mn[4];
+  uint32_t c[4];   // centre value
+};
+
+template <bool kMinMax>
+__device__ __forceinline__ RowD derive(const Words &x) {
+  const uint32_t E0 = hadd(prmt(x.w0, kF16Bias, 0x4240), kMinus1024);  // (c0, c0+2)
+  const uint32_t O0 = hadd(prmt(x.w0, kF16Bias, 0x4341), kMinus1024);  // (c0+1, c0+3)
+  const uint32_t E1 = hadd(prmt(x.w1, kF16Bias, 0x4240), kMinus1024);  // (c0+4, c0+6)
+  const uint32_t O1 = hadd(prmt(x.w1, kF16Bias, 0x4341), kMinus1024);  // (c0+5, c0+7)
+  const uint32_t PO = hadd(prmt(x.pw, kF16Bias, 0x4341), kMinus1024);  // (c0-3, c0-1)
+  const uint32_t NE = hadd(prmt(x.nw, kF16Bias, 0x4240), kMinus1024);  // (c0+8, c0+10)
+  const uint32_t p[4] = {E0, O0, E1, O1};
+  const uint32_t l[4] = {prmt(PO, O0, 0x5432), E0, prmt(O0, O1, 0x5432), E1};
+  const uint32_t r[4] = {O0, prmt(E0, E1, 0x5432), O1, prmt(E1, NE, 0x5432)};
+  RowD d;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    d.c[i] = p[i];
+    d.h[i] = hsub(r[i], l[i]);
+    d.s[i] = hadd(hfma(kTwo, p[i], l[i]), r[i]);
+    if (kMinMax) {
+      d.mx[i] = __vimax3_u16x2(l[i], p[i], r[i]);
+      d.mn[i] = __vimin3_u16x2(l[i], p[i], r[i]);
+    }
+  }
+  return d;
+}
+
+// pEdge of the middle row b (L166: |Gx| + |Gy|, standard Sobel pair, R7).
+__device__ __forceinline__ void sobel(const RowD &a, const RowD &b, const RowD &c, uint32_t pe[4]) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t gx = hadd(hfma(kTwo, b.h[i], a.h[i]), c.h[i]);
+    const uint32_t gy = hsub(c.s[i], a.s[i]);
+    pe[i] = habsadd(gx, gy);
+  }
+}
+
+// Zero the pEdge lane of pixel x (frame column).
+__device__ __forceinline__ void zero_px(uint32_t v[4], int x, uint32_t fill) {
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+    if (i == x) {
+      const int p = pair_of(i);
+      v[p] = half_of(i) ? ((v[p] & 0xffffu) | (fill << 16)) : ((v[p] & 0xffff0000u) | fill);
+    }
+}
+
+// Sum of the 4x4 block of bytes in words a..d (one column of D, times 16).
+__device__ __forceinline__ uint32_t blk(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  uint32_t s = __dp4a(a, 0x01010101u, 0u);
+  s = __dp4a(b, 0x01010101u, s);
+  s = __dp4a(c, 0x01010101u, s);
+  return __dp4a(d, 0x01010101u, s);
+}
+
+struct Block {  // 4 rows of words + the four D sums (16*D) of columns j0-1..j0+2
+  Words r[4];
+  float S[4];
+};
+
+__device__ __forceinline__ void load_block(Block &B, const uint8_t *__restrict__ img, int W, int H, int k,
+                                           int c0, int lane) {
+#pragma unroll
+  for (int a = 0; a < 4; ++a) B.r[a] = load_row(img, W, H, 4 * k + a, c0, lane);
+  B.S[0] = (float)blk(B.r[0].pw, B.r[1].pw, B.r[2].pw, B.r[3].pw);
+  B.S[1] = (float)blk(B.r[0].w0, B.r[1].w0, B.r[2].w0, B.r[3].w0);
+  B.S[2] = (float)blk(B.r[0].w1, B.r[1].w1, B.r[2].w1, B.r[3].w1);
+  B.S[3] = (float)blk(B.r[0].nw, B.r[1].nw, B.r[2].nw, B.r[3].nw);
+}
+
+// ------------------------------------------------------- upscale border (R4, R5)
+// line(v, n)[c] of L140, given the 16*D values x = v[c>>2], y = v[(c>>2)+1]:
+// k = c & 3;  k == 0 -> x, else ((4-k) x + k y) / 4;  as U: divide by 16.
+__device__ __forceinline__ float line_val(float x16, float y16, int k) {
+  return __fmul_rn(__fadd_rn(__fmul_rn((float)(4 - k), x16), __fmul_rn((float)k, y16)), 1.0f / 64.0f);
+}
+
+// Final value of U at a pixel of the 2-pixel ring (last writer of steps
+// i..vii of L140-L142).  Sc = 16*D of the current D row block (row k) for
+// columns j0-1..j0+2, Sn = the next D row (k+1); j0 = c0/4; r = 4k + a'.
+__device__ float ring_u(int r, int c, int W, int H, int j0, const float Sc[4], const float Sn[4]) {
+  const int w = W >> 2, h = H >> 2;
+  auto col = [&](int j) { return j - j0 + 1; };  // index into Sc/Sn
+  if (r >= H - 2 && c >= W - 2) {                 // (vii): third last of last column = D[h-1][w-1]
+    return __fmul_rn(Sc[col(w - 1)], 1.0f / 16.0f);
+  }
+  if ((c <= 1 || c >= W - 2) && r <= H - 3) {     // (vi)/(ii)/(iv): column lines
+    const int j = (c <= 1) ? 0 : w - 1;
+    if (c <= 1 && r <= 1) return __fmul_rn(Sc[col(0)], 1.0f / 16.0f);  // (v) then (vi): D[0][0]
+    const int rr = (r == H - 3) ? H - 4 : r;   // third last <- fourth last
+    const int k = rr & 3;                      // rr>>2 == current D row (rr in the block of r)
+    return line_val(Sc[col(j)], Sn[col(j)], k);
+  }
+  // rows 0/1 (line of D row 0) or H-2/H-1 (line of D row h-1); Sc is that D row.
+  const int cc = (c == W - 3) ? W - 4 : c;
+  const int jj = cc >> 2, k = cc & 3;
+  const float x = Sc[col(jj)];
+  const float y = (k == 0) ? x : Sc[col(jj + 1)];
+  (void)h;
+  return line_val(x, y, k);
+}
+
+// =========================================================================
+// Pass 1: Sobel + reduction + last-block-done LUT construction.
+// =========================================================================
+__global__ void __launch_bounds__(kThreads) edge_sum_kernel(const uint8_t *__restrict__ imgs, int W, int H,
+                                                            int tiles_x, int tiles_y, Params prm,
+                                                            unsigned long long *__restrict__ sums,
+                                                            unsigned int *__restrict__ counters,
+                                                            float2 *__restrict__ luts,
+                                                            double *__restrict__ means) {
+  __shared__ uint32_t warp_sum[kWarps];
+  __shared__ int am_last;
+  const int f = blockIdx.y;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int tile = blockIdx.x * kWarps + warp;
+  const uint8_t *img = imgs + (size_t)f * W * H;
+  float acc = 0.0f;  // exact: < 8 px * 32 rows * 1530 < 2^24
+  if (tile < tiles_x * tiles_y) {
+    const int tx = tile % tiles_x, ty = tile / tiles_x;
+    const int c0 = tx * kWarpCols + lane * kPx;
+    const int R0 = ty * kTileRows;
+    const int R1 = min(R0 + kTileRows, H);
+    RowD a = derive<false>(load_row(img, W, H, R0 - 1, c0, lane));
+    RowD b = derive<false>(load_row(img, W, H, R0, c0, lane));
+    for (int r = R0; r < R1; ++r) {
+      const RowD c = derive<false>(load_row(img, W, H, r + 1, c0, lane));
+      uint32_t pe[4];
+      sobel(a, b, c, pe);
+      if (r == 0 || r == H - 1) {  // Sobel border rows are 0 (L160)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) pe[i] = 0u;
+      }
+      if (c0 == 0) zero_px(pe, 0, 0u);                          // first column
+      if (c0 <= W - 1 && W - 1 < c0 + kPx) zero_px(pe, W - 1 - c0, 0u);  // last column
+      if (c0 + kPx > W) {                                       // pixels beyond the image
+#pragma unroll
+        for (int x = 0; x < kPx; ++x)
+          if (c0 + x >= W) zero_px(pe, x, 0u);
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        acc = add_f32_f16(lo16(pe[i]), acc);
+        acc = add_f32_f16(hi16(pe[i]), acc);
+      }
+      a = b;
+      b = c;
+    }
+  }
+  // Reduction stage 1 (sec. V-C, Fig. 9): warp reduction then CTA partial.
+  const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
+  if (lane == 0) warp_sum[warp] = ws;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long part = 0;
+#pragma unroll
+    for (int i = 0; i < kWarps; ++i) part += warp_sum[i];
+    atomicAdd(&sums[f], part);
+    __threadfence();
+    const unsigned int ticket = atomicAdd(&counters[f], 1u);
+    am_last = (ticket == gridDim.x - 1);
+  }
+  __syncthreads();
+  if (!am_last) return;
+  // Stage 2 (last-block-done): mean and the per-frame lookup tables.
+  __threadfence();
+  const unsigned long long S = atomicAdd(&sums[f], 0ull);
+  const double mean = (double)S / ((double)W * (double)H);
+  const double m = mean > 1.0 ? mean : 1.0;
+  for (int p = threadIdx.x; p < kLutSize; p += kThreads) {
+    float adj = 0.0f, osc = 0.0f;
+    if (p <= 1530) {
+      adj = (float)((double)prm.amount * pow((double)p / m, (double)prm.gamma));
+      osc = (float)fmin(fmax((double)prm.osc_gain * exp(-(double)p / ((double)prm.osc_scale * m)), 0.0), 1.0);
+    }
+    luts[(size_t)f * kLutSize + p] = make_float2(adj, osc);
+  }
+  if (threadIdx.x == 0) {
+    means[f] = mean;
+    counters[f] = 0u;  // re-arm for the next launch
+  }
+}
+
+// =========================================================================
+// Pass 2: everything else, fused.
+// =========================================================================
+// Upscale weights (R3): P = [[7,1],[5,3],[3,5],[1,7]] / 8.  For the lane's 8
+// columns x = 0..7 (column 4*j0 + x), the horizontal pair of D columns
+// (relative index jl, jl+1 into S[]) and the left weight *8.
+__device__ __forceinline__ int wl_of(int x) { return (x & 3) == 0 ? 3 : (x & 3) == 1 ? 1 : (x & 3) == 2 ? 7 : 5; }
+__device__ __forceinline__ int jl_of(int x) { return x < 2 ? 0 : (x < 6 ? 1 : 2); }
+
+__global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__restrict__ imgs, int W, int H,
+                                                           int tiles_x, int tiles_y,
+                                                           const float2 *__restrict__ luts,
+                                                           uint8_t *__restrict__ outs) {
+  __shared__ float2 lut[kLutSize];
+  const int f = blockIdx.y;
+  for (int i = threadIdx.x; i < kLutSize; i += kThreads) lut[i] = luts[(size_t)f * kLutSize + i];
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int tile = blockIdx.x * kWarps + warp;
+  if (tile >= tiles_x * tiles_y) return;
+  // LDS address of lut[p] from the bits of (2^23 + p) as f32: q*8 + base'.
+  const uint32_t lut_base = (uint32_t)__cvta_generic_to_shared(lut) - (0x4B000000u << 3);
+
+  const int tx = tile % tiles_x, ty = tile / tiles_x;
+  const int c0 = tx * kWarpCols + lane * kPx;
+  const int j0 = c0 >> 2;
+  const int R0 = ty * kTileRows;  // multiple of 4
+  const int R1 = min(R0 + kTileRows, H);
+  const uint8_t *img = imgs + (size_t)f * W * H;
+  uint8_t *out = outs + (size_t)f * W * H;
+  const bool ring_cols = (c0 < 2) || (c0 + kPx > W - 2);
+
+  Block prev, cur, next;
+  load_block(prev, img, W, H, (R0 >> 2) - 1, c0, lane);
+  load_block(cur, img, W, H, R0 >> 2, c0, lane);
+  RowD ra = derive<true>(prev.r[3]);
+  RowD rb = derive<true>(cur.r[0]);
+
+  for (int k = R0 >> 2; 4 * k < R1; ++k) {
+    load_block(next, img, W, H, k + 1, c0, lane);
+#pragma unroll
+    for (int a = 0; a < 4; ++a) {
+      const int r = 4 * k + a;
+      const RowD rc = derive<true>(a < 3 ? cur.r[a + 1] : next.r[0]);
+      if (r < R1) {
+        uint32_t pe[4], MX[4], MN[4];
+        sobel(ra, rb, rc, pe);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          MX[i] = __vimax3_u16x2(ra.mx[i], rb.mx[i], rc.mx[i]);
+          MN[i] = __vimin3_u16x2(ra.mn[i], rb.mn[i], rc.mn[i]);
+        }
+        // Frame of the image: Sobel 0 (L160) and no overshoot window (L208,
+        // R13: the frame is the clamped preliminary value == window [0,255]).
+        if (r == 0 || r == H - 1) {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            pe[i] = 0u;
+            MX[i] = kF16_255 | (kF16_255 << 16);
+            MN[i] = 0u;
+          }
+        }
+        if (c0 == 0) {
+          zero_px(pe, 0, 0u);
+          zero_px(MX, 0, kF16_255);
+          zero_px(MN, 0, 0u);
+        }
+        if (c0 <= W - 1 && W - 1 < c0 + kPx) {
+          zero_px(pe, W - 1 - c0, 0u);
+          zero_px(MX, W - 1 - c0, kF16_255);
+          zero_px(MN, W - 1 - c0, 0u);
+        }
+        // Vertical interpolation of the three D-column sums (16*D):
+        //   a' = 0,1: U block row k-1, weights (3,5),(1,7) on D rows (k-1,k)
+        //   a' = 2,3: U block row k,   weights (7,1),(5,3) on D rows (k,k+1)
+        const float wt = (float)(a == 0 ? 3 : a == 1 ? 1 : a == 2 ? 7 : 5);
+        const float wb = 8.0f - wt;
+        float V[4];  // 128 * D interpolated vertically (exact)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const float top = a < 2 ? prev.S[j] : cur.S[j];
+          const float bot = a < 2 ? cur.S[j] : next.S[j];
+          V[j] = __fmaf_rn(wb, bot, __fmul_rn(wt, top));
+        }
+        float NU[8];  // -U, exact
+#pragma unroll
+        for (int x = 0; x < 8; ++x) {
+          const int jl = jl_of(x);
+          const float wl = (float)wl_of(x);
+          NU[x] = __fmaf_rn(-(8.0f - wl) * (1.0f / 1024.0f), V[jl + 1], __fmul_rn(-wl * (1.0f / 1024.0f), V[jl]));
+        }
+        if (r < 2 || r >= H - 2 || ring_cols) {  // the 2-pixel upscale border ring
+          const float *Sc = cur.S;  // D row k: row 0 for rows 0,1; row h-1 for rows H-2,H-1
+          const float *Sn = next.S;
+#pragma unroll
+          for (int x = 0; x < 8; ++x) {
+            const int c = c0 + x;
+            if (c < W && (r < 2 || r >= H - 2 || c < 2 || c >= W - 2)) NU[x] = -ring_u(r, c, W, H, j0, Sc, Sn);
+          }
+        }
+        uint32_t o[8];
+#pragma unroll
+        for (int x = 0; x < 8; ++x) {
+          const int p = pair_of(x);
+          const bool hi = half_of(x);
+          const uint16_t pe_h = hi ? hi16(pe[p]) : lo16(pe[p]);
+          const uint16_t c_h = hi ? hi16(rb.c[p]) : lo16(rb.c[p]);
+          const uint16_t mx_h = hi ? hi16(MX[p]) : lo16(MX[p]);
+          const uint16_t mn_h = hi ? hi16(MN[p]) : lo16(MN[p]);
+          const uint32_t q = __float_as_uint(add_f32_f16(pe_h, 8388608.0f));  // 2^23 + pEdge
+          const float2 L = lds_v2(q * 8u + lut_base);                        // {adj, osc}
+          const float E = add_f32_f16(c_h, NU[x]);                           // pError = O - U (L148)
+          const float P = __fmaf_rn(L.x, E, -NU[x]);                         // preliminary (L178)
+          const float mxf = add_f32_f16(mx_h, 0.0f), mnf = add_f32_f16(mn_h, 0.0f);
+          const float t = fminf(fmaxf(P, mnf), mxf);                         // Fig. 8 branch target
+          const float F = __fmaf_rn(L.y, __fsub_rn(P, t), t);                // osc max / osc min / P
+          o[x] = cvt_u8(F);                                                  // clamp [0,255], RNE
+        }
+        const uint32_t o0 = prmt(prmt(o[0], o[1], 0x0040), prmt(o[2], o[3], 0x0040), 0x5410);
+        const uint32_t o1 = prmt(prmt(o[4], o[5], 0x0040), prmt(o[6], o[7], 0x0040), 0x5410);
+        uint8_t *orow = out + (size_t)r * W;
+        if (c0 < W) *reinterpret_cast<uint32_t *>(orow + c0) = o0;
+        if (c0 + 4 < W) *reinterpret_cast<uint32_t *>(orow + c0 + 4) = o1;
+      }
+      ra = rb;
+      rb = rc;
+    }
+    prev = cur;
+    cur = next;
+  }
+}
+
+}  // namespace
+
+static void geometry(int W, int H, int &tiles_x, int &tiles_y, int &ctas) {
+  tiles_x = (W + kWarpCols - 1) / kWarpCols;
+  tiles_y = (H + kTileRows - 1) / kTileRows;
+  ctas = (tiles_x * tiles_y + kWarps - 1) / kWarps;
+}
+
+cudaError_t launch_edge_sum(const uint8_t *imgs, int n, int W, int H, const Params &p,
+                            unsigned long long *sums, unsigned int *counters, float2 *luts,
+                            double *means, cudaStream_t stream) {
+  int tx, ty, ctas;
+  geometry(W, H, tx, ty, ctas);
+  edge_sum_kernel<<<dim3(ctas, n), kThreads, 0, stream>>>(imgs, W, H, tx, ty, p, sums, counters, luts, means);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts, uint8_t *outs,
+                           cudaStream_t stream) {
+  int tx, ty, ctas;
+  geometry(W, H, tx, ty, ctas);
+  sharpen_kernel<<<dim3(ctas, n), kThreads, 0, stream>>>(imgs, W, H, tx, ty, luts, outs);
+  return cudaGetLastError();
+}
+
+}  // namespace sharp

@@ -1,0 +1,32 @@
+// Internal launch interface of the sm_100a kernels (not part of the C ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace sharp {
+
+// Lookup tables built once per frame by the last CTA of pass 1: entry p
+// (p = pEdge value, 0..1530 = 6*255) holds {adj(p), osc(p)} (R9, R11).
+constexpr int kLutSize = 1536;
+
+struct Params {
+  float amount, gamma, osc_gain, osc_scale;
+};
+
+// Pass 1 (Sobel + reduction + LUT): for frames [0, n) of `imgs` (dense
+// [n][H][W]) accumulates S into sums[frame_base + f] (must be zero on entry),
+// and the last CTA of each frame writes means[frame_base + f] and
+// luts[f * kLutSize ..] and re-arms counters[f] (must be zero on entry).
+cudaError_t launch_edge_sum(const uint8_t *imgs, int n, int W, int H, const Params &p,
+                            unsigned long long *sums, unsigned int *counters, float2 *luts,
+                            double *means, cudaStream_t stream);
+
+// Pass 2 (fused downscale/upscale/pError/Sobel/min-max/strength/preliminary/
+// overshoot/output): frames [0, n) with the per-frame LUTs of pass 1.
+cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts,
+                           uint8_t *outs, cudaStream_t stream);
+
+// Kernel launches issued per (pass-1, pass-2) chunk.
+constexpr int kLaunchesPerChunk = 2;
+
+}  // namespace sharp

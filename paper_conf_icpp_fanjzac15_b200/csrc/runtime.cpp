@@ -1,0 +1,505 @@
+// C ABI + runtime of libsharp.so (include/sharp.h).
+//
+// The runtime owns: the device scratch of the two passes (per-frame u64 edge
+// sums, per-frame means, per-chunk-frame counters and lookup tables), the
+// stream it launches on, a pipeline of `streams` slots (stream + device
+// in/out buffers + pinned host staging) used when the caller passes host
+// memory (sec. V-A: bulk read/write transfers, only O up and the
+// final image down, L252-L266, L336), and the error state.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <vector>
+
+#include "kernels.h"
+#include "sharp.h"
+
+namespace {
+
+constexpr size_t kL2ChunkBudget = 24u << 20;  // input bytes per chunk kept L2-resident between passes
+constexpr int kMaxSlots = 8;
+
+struct Slot {
+  cudaStream_t stream = nullptr;
+  cudaEvent_t done = nullptr;
+  uint8_t *d_in = nullptr, *d_out = nullptr;   // device staging (chunk)
+  uint8_t *h_in = nullptr, *h_out = nullptr;   // pinned staging (chunk)
+  unsigned int *counters = nullptr;            // per chunk frame
+  float2 *luts = nullptr;                      // per chunk frame
+};
+
+}  // namespace
+
+struct sharp_ctx {
+  int device = 0;
+  cudaStream_t own_stream = nullptr;
+  cudaStream_t stream = nullptr;  // launch stream (own or caller's)
+  cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
+  int nslots = 3;
+  int chunk_cfg = 0;
+  Slot slots[kMaxSlots];
+  size_t slot_chunk_frames = 0, slot_stage_bytes = 0;  // capacity of the slot buffers
+  unsigned long long *sums = nullptr;
+  double *means = nullptr;
+  size_t frames_cap = 0;
+  int last_frames = 0;
+  sharp_stats stats{};
+  // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2)
+  bool profiling = false;
+  struct Rec { cudaEvent_t a, b; int kind; double px; };
+  std::vector<Rec> recs;
+  std::vector<cudaEvent_t> ev_pool;
+  bool poisoned = false;
+  char err[256] = {0};
+};
+
+namespace {
+
+int set_err(sharp_ctx *c, int code, const char *fmt, const char *what) {
+  if (c) snprintf(c->err, sizeof(c->err), fmt, what);
+  return code;
+}
+
+// Maps a CUDA error to a return code; sticky errors poison the context.
+int cuda_fail(sharp_ctx *c, cudaError_t e, const char *where) {
+  if (e == cudaSuccess) return SHARP_OK;
+  if (c) {
+    snprintf(c->err, sizeof(c->err), "%s: %s", where, cudaGetErrorString(e));
+    if (e == cudaErrorMemoryAllocation) {
+      cudaGetLastError();
+      return SHARP_ENOMEM;
+    }
+    // Probe whether the error is sticky (the context is unusable).
+    cudaError_t probe = cudaDeviceSynchronize();
+    if (probe != cudaSuccess) c->poisoned = true;
+    cudaGetLastError();
+  }
+  return SHARP_ECUDA;
+}
+
+#define CK(expr)                                          \
+  do {                                                    \
+    cudaError_t e__ = (expr);                             \
+    if (e__ != cudaSuccess) return cuda_fail(ctx, e__, #expr); \
+  } while (0)
+
+bool params_ok(const sharp_params &p) {
+  // R16 ranges; NaN fails every comparison.
+  return p.amount >= 0.0f && p.amount <= 16.0f && p.gamma >= 0.0f && p.gamma <= 4.0f &&
+         p.osc_gain >= 0.0f && p.osc_gain <= 1.0f && p.osc_scale > 0.0f && p.osc_scale <= 1.0e6f;
+}
+
+enum Kind { kDevice, kPinned, kPageable };
+
+int classify(sharp_ctx *ctx, const void *p, Kind *k) {
+  cudaPointerAttributes a;
+  cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    *k = kPageable;
+    return SHARP_OK;
+  }
+  switch (a.type) {
+    case cudaMemoryTypeDevice:
+    case cudaMemoryTypeManaged:
+      if (a.device != ctx->device)
+        return set_err(ctx, SHARP_EINVAL, "%s", "device pointer belongs to another device");
+      *k = kDevice;
+      break;
+    case cudaMemoryTypeHost: *k = kPinned; break;
+    default: *k = kPageable;
+  }
+  return SHARP_OK;
+}
+
+int ensure_frames(sharp_ctx *ctx, size_t n) {
+  if (n <= ctx->frames_cap) return SHARP_OK;
+  cudaFree(ctx->sums);
+  cudaFree(ctx->means);
+  ctx->sums = nullptr;
+  ctx->means = nullptr;
+  ctx->frames_cap = 0;
+  CK(cudaMalloc(&ctx->sums, n * sizeof(unsigned long long)));
+  CK(cudaMalloc(&ctx->means, n * sizeof(double)));
+  ctx->frames_cap = n;
+  return SHARP_OK;
+}
+
+void free_slot(Slot &s) {
+  cudaFree(s.d_in);
+  cudaFree(s.d_out);
+  cudaFreeHost(s.h_in);
+  cudaFreeHost(s.h_out);
+  cudaFree(s.counters);
+  cudaFree(s.luts);
+  s.d_in = s.d_out = s.h_in = s.h_out = nullptr;
+  s.counters = nullptr;
+  s.luts = nullptr;
+}
+
+// Every slot gets counters + LUTs for `chunk` frames; device/pinned staging
+// buffers of chunk*frame_bytes only when `staging` (host-memory calls).
+int ensure_slots(sharp_ctx *ctx, size_t chunk, size_t frame_bytes, bool staging) {
+  const size_t need_stage = staging ? chunk * frame_bytes : 0;
+  if (chunk <= ctx->slot_chunk_frames && need_stage <= ctx->slot_stage_bytes) return SHARP_OK;
+  CK(cudaStreamSynchronize(ctx->stream));
+  for (int i = 0; i < ctx->nslots; ++i) CK(cudaStreamSynchronize(ctx->slots[i].stream));
+  const size_t cap = std::max(chunk, ctx->slot_chunk_frames);
+  const size_t stage = std::max(need_stage, ctx->slot_stage_bytes);
+  ctx->slot_chunk_frames = 0;
+  ctx->slot_stage_bytes = 0;
+  for (int i = 0; i < ctx->nslots; ++i) {
+    Slot &s = ctx->slots[i];
+    free_slot(s);
+    CK(cudaMalloc(&s.counters, cap * sizeof(unsigned int)));
+    CK(cudaMemset(s.counters, 0, cap * sizeof(unsigned int)));
+    CK(cudaMalloc(&s.luts, cap * sharp::kLutSize * sizeof(float2)));
+    if (stage) {
+      CK(cudaMalloc(&s.d_in, stage));
+      CK(cudaMalloc(&s.d_out, stage));
+      CK(cudaHostAlloc(&s.h_in, stage, cudaHostAllocDefault));
+      CK(cudaHostAlloc(&s.h_out, stage, cudaHostAllocDefault));
+    }
+  }
+  ctx->slot_chunk_frames = cap;
+  ctx->slot_stage_bytes = stage;
+  return SHARP_OK;
+}
+
+size_t chunk_frames(const sharp_ctx *ctx, size_t frame_bytes, int n) {
+  size_t c = ctx->chunk_cfg > 0 ? (size_t)ctx->chunk_cfg : std::max<size_t>(1, kL2ChunkBudget / frame_bytes);
+  c = std::min<size_t>(c, 65535);
+  return std::min<size_t>(c, (size_t)n);
+}
+
+int validate(sharp_ctx *ctx, const void *in, const void *out, int n, int w, int h, const sharp_params *p) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  if (!in || !out) return set_err(ctx, SHARP_EINVAL, "%s", "NULL image pointer");
+  if (n < 1) return set_err(ctx, SHARP_EINVAL, "%s", "n < 1");
+  if (w < 8 || h < 8 || (w & 3) || (h & 3))
+    return set_err(ctx, SHARP_EINVAL, "%s", "width and height must be multiples of 4 and >= 8 (R1)");
+  if ((long long)w * h >= (1ll << 31) || w > 65536 || h > 65536)
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "image larger than 2^31 pixels");
+  if (p && !params_ok(*p)) return set_err(ctx, SHARP_EINVAL, "%s", "parameter out of range or not finite");
+  const size_t bytes = (size_t)n * w * h;
+  const uintptr_t a = (uintptr_t)in, b = (uintptr_t)out;
+  if (a < b + bytes && b < a + bytes) return set_err(ctx, SHARP_EINVAL, "%s", "input and output overlap");
+  return SHARP_OK;
+}
+
+cudaEvent_t pool_event(sharp_ctx *ctx) {
+  if (!ctx->ev_pool.empty()) {
+    cudaEvent_t e = ctx->ev_pool.back();
+    ctx->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  if (cudaEventCreate(&e) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return e;
+}
+
+// Records an event pair around `launch` when profiling.
+template <typename F>
+cudaError_t timed(sharp_ctx *ctx, cudaStream_t st, int kind, double px, F launch) {
+  if (!ctx->profiling) return launch();
+  cudaEvent_t a = pool_event(ctx), b = pool_event(ctx);
+  if (!a || !b) return launch();
+  cudaEventRecord(a, st);
+  cudaError_t e = launch();
+  cudaEventRecord(b, st);
+  ctx->recs.push_back({a, b, kind, px});
+  return e;
+}
+
+// Device-resident batch: chunks of frames, pass 1 then pass 2 per chunk, on
+// one stream (the chunk's input is still in L2 when pass 2 re-reads it).
+int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, const sharp::Params &prm,
+                   uint8_t *dout, cudaStream_t st, Slot &slot, size_t chunk, size_t frame_base, int *launches) {
+  const size_t fb = (size_t)w * h;
+  for (size_t f0 = 0; f0 < (size_t)n; f0 += chunk) {
+    const int cn = (int)std::min(chunk, (size_t)n - f0);
+    const double px = (double)cn * fb;
+    CK(timed(ctx, st, 1, px, [&] {
+      return sharp::launch_edge_sum(din + f0 * fb, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters,
+                                    slot.luts, ctx->means + frame_base + f0, st);
+    }));
+    CK(timed(ctx, st, 2, px, [&] { return sharp::launch_sharpen(din + f0 * fb, cn, w, h, slot.luts, dout + f0 * fb, st); }));
+    *launches += sharp::kLaunchesPerChunk;
+  }
+  return SHARP_OK;
+}
+
+int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp_params *pp, uint8_t *out,
+             bool async) {
+  int rc = validate(ctx, in, out, n, w, h, pp);
+  if (rc) return rc;
+  sharp_params p;
+  if (pp) p = *pp;
+  else sharp_default_params(&p);
+  const sharp::Params prm{p.amount, p.gamma, p.osc_gain, p.osc_scale};
+  Kind kin, kout;
+  if ((rc = classify(ctx, in, &kin)) || (rc = classify(ctx, out, &kout))) return rc;
+  if (async && (kin != kDevice || kout != kDevice))
+    return set_err(ctx, SHARP_EINVAL, "%s", "sharp_enqueue_batch takes device pointers only");
+  if ((kin == kDevice && ((uintptr_t)in & 3)) || (kout == kDevice && ((uintptr_t)out & 3)))
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "device buffers must be 4-byte aligned");
+  CK(cudaSetDevice(ctx->device));
+  const auto t0 = std::chrono::steady_clock::now();
+  const size_t fb = (size_t)w * h;
+  const size_t chunk = chunk_frames(ctx, fb, n);
+  const bool staged = !(kin == kDevice && kout == kDevice);
+  if ((rc = ensure_frames(ctx, (size_t)n))) return rc;
+  if ((rc = ensure_slots(ctx, chunk, fb, staged))) return rc;
+  int launches = 0;
+  CK(cudaMemsetAsync(ctx->sums, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
+  if (!async) CK(cudaEventRecord(ctx->ev_start, ctx->stream));
+  if (!staged) {
+    if ((rc = enqueue_device(ctx, in, n, w, h, prm, out, ctx->stream, ctx->slots[0], chunk, 0, &launches)))
+      return rc;
+  } else {
+    // Host pipeline (sec. V-A): chunk c on slot c % nslots; H2D || kernels || D2H.
+    const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
+    std::vector<size_t> pending_off(ctx->nslots, (size_t)-1), pending_n(ctx->nslots, 0);
+    for (int i = 0; i < ctx->nslots; ++i) CK(cudaStreamWaitEvent(ctx->slots[i].stream, ctx->ev_start, 0));
+    auto drain = [&](int s) -> int {
+      if (pending_off[s] == (size_t)-1) return SHARP_OK;
+      CK(cudaEventSynchronize(ctx->slots[s].done));
+      if (kout == kPageable) memcpy(out + pending_off[s] * fb, ctx->slots[s].h_out, pending_n[s] * fb);
+      pending_off[s] = (size_t)-1;
+      return SHARP_OK;
+    };
+    for (size_t c = 0; c < nchunks; ++c) {
+      const int s = (int)(c % ctx->nslots);
+      Slot &sl = ctx->slots[s];
+      if ((rc = drain(s))) return rc;
+      const size_t f0 = c * chunk, cn = std::min(chunk, (size_t)n - f0), bytes = cn * fb;
+      const uint8_t *src = in + f0 * fb;
+      const uint8_t *dsrc = src;
+      if (kin != kDevice) {
+        if (kin == kPageable) {
+          memcpy(sl.h_in, src, bytes);
+          src = sl.h_in;
+        }
+        CK(cudaMemcpyAsync(sl.d_in, src, bytes, cudaMemcpyHostToDevice, sl.stream));
+        dsrc = sl.d_in;
+      }
+      uint8_t *ddst = (kout == kDevice) ? out + f0 * fb : sl.d_out;
+      if ((rc = enqueue_device(ctx, dsrc, (int)cn, w, h, prm, ddst, sl.stream, sl, cn, f0, &launches))) return rc;
+      if (kout != kDevice) {
+        uint8_t *hdst = (kout == kPinned) ? out + f0 * fb : sl.h_out;
+        CK(cudaMemcpyAsync(hdst, sl.d_out, bytes, cudaMemcpyDeviceToHost, sl.stream));
+      }
+      CK(cudaEventRecord(sl.done, sl.stream));
+      pending_off[s] = f0;
+      pending_n[s] = cn;
+    }
+    for (int s = 0; s < ctx->nslots; ++s) {
+      if ((rc = drain(s))) return rc;
+      CK(cudaStreamWaitEvent(ctx->stream, ctx->slots[s].done, 0));
+    }
+  }
+  ctx->last_frames = n;
+  ctx->stats.frames = n;
+  ctx->stats.kernels = launches;
+  if (async) return SHARP_OK;
+  CK(cudaEventRecord(ctx->ev_stop, ctx->stream));
+  CK(cudaEventSynchronize(ctx->ev_stop));
+  float ms = 0.0f;
+  CK(cudaEventElapsedTime(&ms, ctx->ev_start, ctx->ev_stop));
+  unsigned long long s0 = 0;
+  double m0 = 0.0;
+  CK(cudaMemcpy(&s0, ctx->sums, sizeof(s0), cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(&m0, ctx->means, sizeof(m0), cudaMemcpyDeviceToHost));
+  ctx->stats.edge_sum = s0;
+  ctx->stats.edge_mean = m0;
+  ctx->stats.device_ms = ms;
+  ctx->stats.total_ms =
+      std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return SHARP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void sharp_default_params(sharp_params *p) {
+  if (!p) return;
+  p->amount = 1.0f;    // R16
+  p->gamma = 0.5f;
+  p->osc_gain = 0.5f;
+  p->osc_scale = 2.0f;
+}
+
+int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
+  if (!out) return SHARP_EINVAL;
+  *out = nullptr;
+  sharp_config c{};
+  c.device = -1;
+  if (cfg) c = *cfg;
+  if (c.streams < 0 || c.streams > kMaxSlots || c.chunk_frames < 0 || c.max_frames < 0) return SHARP_EINVAL;
+  sharp_ctx *ctx = new (std::nothrow) sharp_ctx();
+  if (!ctx) return SHARP_ENOMEM;
+  int dev = c.device;
+  cudaError_t e = cudaSuccess;
+  if (dev < 0) e = cudaGetDevice(&dev);
+  int ndev = 0;
+  if (e == cudaSuccess) e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || dev >= ndev) {
+    cudaGetLastError();
+    delete ctx;
+    return e != cudaSuccess ? SHARP_ECUDA : SHARP_EINVAL;
+  }
+  ctx->device = dev;
+  ctx->nslots = c.streams ? c.streams : 3;
+  ctx->chunk_cfg = c.chunk_frames;
+  int rc = SHARP_OK;
+  do {
+    if ((e = cudaSetDevice(dev)) != cudaSuccess) break;
+    if ((e = cudaStreamCreateWithFlags(&ctx->own_stream, cudaStreamNonBlocking)) != cudaSuccess) break;
+    ctx->stream = ctx->own_stream;
+    if ((e = cudaEventCreate(&ctx->ev_start)) != cudaSuccess) break;
+    if ((e = cudaEventCreate(&ctx->ev_stop)) != cudaSuccess) break;
+    for (int i = 0; i < ctx->nslots && e == cudaSuccess; ++i) {
+      e = cudaStreamCreateWithFlags(&ctx->slots[i].stream, cudaStreamNonBlocking);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->slots[i].done, cudaEventDisableTiming);
+    }
+    if (e != cudaSuccess) break;
+    if (c.max_frames > 0 && (rc = ensure_frames(ctx, (size_t)c.max_frames))) break;
+    if (c.max_width > 0 && c.max_height > 0) {
+      const size_t fb = (size_t)c.max_width * c.max_height;
+      if ((rc = ensure_slots(ctx, chunk_frames(ctx, fb, c.max_frames > 0 ? c.max_frames : 1), fb, false))) break;
+    }
+  } while (0);
+  if (e != cudaSuccess || rc != SHARP_OK) {
+    cudaGetLastError();
+    sharp_destroy(ctx);
+    return rc ? rc : (e == cudaErrorMemoryAllocation ? SHARP_ENOMEM : SHARP_ECUDA);
+  }
+  *out = ctx;
+  return SHARP_OK;
+}
+
+void sharp_destroy(sharp_ctx *ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->device);
+  if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+  for (int i = 0; i < kMaxSlots; ++i) {
+    Slot &s = ctx->slots[i];
+    if (s.stream) cudaStreamSynchronize(s.stream);
+    free_slot(s);
+    if (s.done) cudaEventDestroy(s.done);
+    if (s.stream) cudaStreamDestroy(s.stream);
+  }
+  cudaFree(ctx->sums);
+  cudaFree(ctx->means);
+  for (auto &r : ctx->recs) {
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
+  for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
+  if (ctx->ev_stop) cudaEventDestroy(ctx->ev_stop);
+  if (ctx->own_stream) cudaStreamDestroy(ctx->own_stream);
+  cudaGetLastError();
+  delete ctx;
+}
+
+int sharp_set_stream(sharp_ctx *ctx, void *stream) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  ctx->stream = stream ? (cudaStream_t)stream : ctx->own_stream;
+  return SHARP_OK;
+}
+
+int sharp_run(sharp_ctx *ctx, const uint8_t *img, int w, int h, const sharp_params *params, uint8_t *out) {
+  return run_impl(ctx, img, 1, w, h, params, out, false);
+}
+
+int sharp_run_batch(sharp_ctx *ctx, const uint8_t *imgs, int n, int w, int h, const sharp_params *params,
+                    uint8_t *outs) {
+  return run_impl(ctx, imgs, n, w, h, params, outs, false);
+}
+
+int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int h, const sharp_params *params,
+                        uint8_t *d_outs) {
+  return run_impl(ctx, d_imgs, n, w, h, params, d_outs, true);
+}
+
+int sharp_get_stats(const sharp_ctx *ctx, sharp_stats *s) {
+  if (!ctx || !s) return SHARP_EINVAL;
+  *s = ctx->stats;
+  return SHARP_OK;
+}
+
+int sharp_get_batch_sums(sharp_ctx *ctx, uint64_t *sums, int n) {
+  if (!ctx || !sums || n < 0) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  if (n > ctx->last_frames) return set_err(ctx, SHARP_EINVAL, "%s", "n exceeds the frames of the last call");
+  if (n == 0) return SHARP_OK;
+  CK(cudaStreamSynchronize(ctx->stream));
+  CK(cudaMemcpy(sums, ctx->sums, (size_t)n * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+  return SHARP_OK;
+}
+
+int sharp_set_profiling(sharp_ctx *ctx, int enable) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  CK(cudaStreamSynchronize(ctx->stream));
+  for (auto &r : ctx->recs) {
+    ctx->ev_pool.push_back(r.a);
+    ctx->ev_pool.push_back(r.b);
+  }
+  ctx->recs.clear();
+  ctx->profiling = enable != 0;
+  return SHARP_OK;
+}
+
+int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t) {
+  if (!ctx || !t) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  *t = sharp_kernel_times{};
+  for (auto &r : ctx->recs) {
+    CK(cudaEventSynchronize(r.b));
+    float ms = 0.0f;
+    CK(cudaEventElapsedTime(&ms, r.a, r.b));
+    if (r.kind == 1) {
+      t->pass1_ms += ms;
+      t->pass1_launches++;
+      t->pixels += r.px;
+    } else {
+      t->pass2_ms += ms;
+      t->pass2_launches++;
+    }
+  }
+  return SHARP_OK;
+}
+
+const char *sharp_strerror(int code) {
+  switch (code) {
+    case SHARP_OK: return "ok";
+    case SHARP_EINVAL: return "invalid argument";
+    case SHARP_ENOMEM: return "out of memory";
+    case SHARP_ECUDA: return "CUDA error";
+    case SHARP_ENCCL: return "communication error";
+    case SHARP_EUNSUPPORTED: return "unsupported request";
+    case SHARP_ESTATE: return "context poisoned by an earlier error";
+    default: return "unknown error";
+  }
+}
+
+const char *sharp_last_error(const sharp_ctx *ctx) { return ctx ? ctx->err : "no context"; }
+
+const char *sharp_version(void) {
+  return "libsharp 0.1 (sm_100a; two-pass fused sharpen: edge_sum + sharpen; f16x2 SIMD Sobel)";
+}
+
+}  // extern "C"

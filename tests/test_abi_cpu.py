@@ -1,0 +1,77 @@
+"""CPU-only checks of the boundary: libsharp.so loads and exports every symbol
+that include/sharp.h declares; the binding exposes the same names; the product
+package never imports the oracle (task rule 3).  No compute call needs a GPU
+here."""
+import ast
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+PKG = os.path.join(ROOT, "paper_conf_icpp_fanjzac15_b200")
+
+
+def declared_functions():
+    src = open(os.path.join(ROOT, "include", "sharp.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(sharp_[a-z_]+)\s*\(", src)))
+
+
+def test_header_declares_the_north_star_calls():
+    names = declared_functions()
+    for n in ["sharp_create", "sharp_run", "sharp_run_batch", "sharp_destroy"]:
+        assert n in names
+
+
+def test_library_loads_and_exports_every_declared_symbol():
+    lib = ctypes.CDLL(os.path.join(PKG, "libsharp.so"))
+    for name in declared_functions():
+        assert hasattr(lib, name), name
+
+
+def test_binding_exposes_same_names():
+    import paper_conf_icpp_fanjzac15_b200 as p
+    for name in declared_functions():
+        assert hasattr(p, name), name
+
+
+def test_static_strings_without_gpu():
+    import paper_conf_icpp_fanjzac15_b200 as p
+    assert "sm_100a" in p.sharp_version()
+    assert p.sharp_strerror(p.SHARP_EINVAL) == "invalid argument"
+    d = p.sharp_default_params()
+    assert (d.amount, d.gamma, d.osc_gain, d.osc_scale) == (1.0, 0.5, 0.5, 2.0)
+
+
+def test_library_is_sm100a_code():
+    import subprocess
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", os.path.join(PKG, "libsharp.so")],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_product_package_never_imports_or_loads_the_oracle():
+    for dirpath, _, files in os.walk(PKG):
+        for f in files:
+            path = os.path.join(dirpath, f)
+            if f.endswith(".py"):
+                tree = ast.parse(open(path).read())
+                for node in ast.walk(tree):
+                    if isinstance(node, ast.Import):
+                        assert all(not a.name.startswith("oracle") for a in node.names), path
+                    if isinstance(node, ast.ImportFrom):
+                        assert not (node.module or "").startswith("oracle"), path
+            if f.endswith((".py", ".cu", ".cpp", ".h", ".cuh")):
+                assert "liboracle" not in open(path).read(), path
+                assert "oracle.h" not in open(path).read(), path
+
+
+def test_no_cpu_fallback_create_fails_loudly_without_gpu():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    import paper_conf_icpp_fanjzac15_b200 as p
+    with pytest.raises(p.SharpError):
+        p.sharp_create()

@@ -1,0 +1,185 @@
+"""GPU <-> oracle parity through the C ABI (task rule 3).
+
+Every output pixel must be bit-identical to the oracle (the oracle fixes the
+f32 evaluation order everywhere, R15), the pEdge sum S exact and
+the mean exact.  Inputs: tests/../synth (seeded), the same bytes on both sides.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from paper_conf_icpp_fanjzac15_b200 import SHARP_EINVAL, SharpError, Sharpener
+
+pytestmark = pytest.mark.gpu
+
+DEFAULT = (1.0, 0.5, 0.5, 2.0)
+PARAMS = [
+    DEFAULT,
+    (1.0, 0.0, 0.5, 2.0),     # identity: adj == 1
+    (0.0, 0.5, 0.0, 2.0),     # A = 0, G = 0
+    (2.5, 1.0, 0.25, 1.0),
+    (16.0, 4.0, 1.0, 1e6),    # extremes
+    (0.5, 2.0, 0.0, 0.5),
+    (6.0, 0.3, 0.9, 8.0),
+]
+
+
+@pytest.fixture(scope="module")
+def sh():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    s = Sharpener()
+    yield s
+    s.close()
+
+
+def gpu_run(sh, img, prm=DEFAULT):
+    d = torch.from_numpy(img).cuda()
+    o = torch.empty_like(d)
+    sh.run(d, prm, o)
+    torch.cuda.synchronize()
+    st = sh.stats()
+    return o.cpu().numpy(), st.edge_sum, st.edge_mean
+
+
+def assert_parity(sh, img, prm=DEFAULT):
+    out, S, mean = gpu_run(sh, img, prm)
+    ref, S_ref, mean_ref = oracle.sharpen(img, *prm)
+    bad = np.argwhere(out != ref)
+    assert S == S_ref, f"edge sum {S} != {S_ref}"
+    assert mean == mean_ref
+    assert bad.size == 0, (f"{len(bad)} mismatches of {out.size}, first at {bad[:5].tolist()}: "
+                           f"gpu {out[tuple(bad[0])]} oracle {ref[tuple(bad[0])]}")
+
+
+SIZES = [(8, 8), (12, 8), (8, 12), (16, 16), (20, 12), (64, 48), (100, 36), (252, 20), (260, 36),
+         (300, 68), (516, 44), (1028, 40)]
+
+
+@pytest.mark.parametrize("W,H", SIZES)
+@pytest.mark.parametrize("kind", ["natural", "noise"])
+def test_small_sizes_tiles_and_ragged_tails(W, H, kind, sh):
+    img = synth.image(W, H, kind, seed=W * 1000 + H)
+    assert_parity(sh, img)
+
+
+@pytest.mark.parametrize("kind,param", [("natural", 0), ("noise", 0), ("ramp", 0), ("const", 0),
+                                        ("const", 255), ("const", 131), ("checker", 30),
+                                        ("impulse", 255)])
+@pytest.mark.parametrize("prm", PARAMS)
+def test_kinds_and_params_512(kind, param, prm, sh):
+    img = synth.image(512, 512, kind, seed=synth.BASE_SEED, param=param)
+    assert_parity(sh, img, prm)
+
+
+@pytest.mark.parametrize("W,H,seed", [(1920, 1080, 1), (3840, 2160, 2)])
+def test_full_frames_1080p_4k(W, H, seed, sh):
+    img = synth.image(W, H, "natural", seed=synth.BASE_SEED + seed)
+    assert_parity(sh, img)
+
+
+def test_full_frame_8k(sh):
+    img = synth.image(7680, 4320, "natural", seed=synth.BASE_SEED + 3)
+    assert_parity(sh, img)
+
+
+def test_identity_params_reproduce_input_on_gpu(sh):
+    img = synth.image(1920, 1080, "noise", seed=7)
+    out, _, _ = gpu_run(sh, img, (1.0, 0.0, 0.3, 2.0))
+    np.testing.assert_array_equal(out, img)
+
+
+def test_batch_frames_independent_and_equal_to_oracle(sh):
+    imgs = synth.frames(6, 264, 40, "natural", seed=123)
+    imgs[2] = 77  # a constant frame in the middle: S = 0
+    d = torch.from_numpy(imgs).cuda()
+    o = torch.empty_like(d)
+    sh.run_batch(d, DEFAULT, o)
+    sums = sh.batch_sums(6)
+    out = o.cpu().numpy()
+    ref, ref_sums = oracle.sharpen_batch(imgs, *DEFAULT)
+    np.testing.assert_array_equal(out, ref)
+    assert sums == [int(s) for s in ref_sums]
+
+
+def test_batch_chunking_many_chunks():
+    # chunk_frames=3 forces several pass-1/pass-2 chunk pairs on one stream
+    imgs = synth.frames(10, 128, 64, "natural", seed=9)
+    with Sharpener(chunk_frames=3) as s:
+        d = torch.from_numpy(imgs).cuda()
+        o = torch.empty_like(d)
+        s.run_batch(d, DEFAULT, o)
+        sums = s.batch_sums(10)
+    ref, ref_sums = oracle.sharpen_batch(imgs, *DEFAULT)
+    np.testing.assert_array_equal(o.cpu().numpy(), ref)
+    assert sums == [int(x) for x in ref_sums]
+
+
+@pytest.mark.parametrize("mode", ["pageable", "pinned", "dev_in_host_out", "host_in_dev_out"])
+def test_host_memory_paths(mode):
+    imgs = synth.frames(7, 1920, 1080, "natural", seed=44)
+    ref, ref_sums = oracle.sharpen_batch(imgs, *DEFAULT)
+    with Sharpener(chunk_frames=2, streams=3) as s:
+        if mode == "pageable":
+            out = np.empty_like(imgs)
+            s.run_batch(imgs, DEFAULT, out)
+        elif mode == "pinned":
+            src = torch.from_numpy(imgs).pin_memory()
+            dst = torch.empty_like(src).pin_memory()
+            s.run_batch(src, DEFAULT, dst)
+            out = dst.numpy()
+        elif mode == "dev_in_host_out":
+            src = torch.from_numpy(imgs).cuda()
+            out = np.empty_like(imgs)
+            s.run_batch(src, DEFAULT, out)
+        else:
+            dst = torch.empty(imgs.shape, dtype=torch.uint8, device="cuda")
+            s.run_batch(imgs, DEFAULT, dst)
+            out = dst.cpu().numpy()
+        sums = s.batch_sums(7)
+    np.testing.assert_array_equal(out, ref)
+    assert sums == [int(x) for x in ref_sums]
+
+
+def test_bench_configuration_sampled_frames():
+    """The bench's launch configuration (1024 x 1080p, device-resident,
+    automatic chunking) compared on sampled frames against the oracle."""
+    n, W, H = 1024, 1920, 1080
+    imgs = synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 5)
+    with Sharpener() as s:
+        d = torch.from_numpy(imgs).cuda()
+        o = torch.empty_like(d)
+        s.enqueue_batch(d, o, DEFAULT)
+        torch.cuda.synchronize()
+        sums = s.batch_sums(n)
+    sample = list(range(0, n, 33))[:32]
+    ref, ref_sums = oracle.sharpen_batch(imgs[sample], *DEFAULT)
+    out = o[sample].cpu().numpy()
+    np.testing.assert_array_equal(out, ref)
+    assert [sums[i] for i in sample] == [int(x) for x in ref_sums]
+
+
+@pytest.mark.parametrize("W,H", [(6, 8), (8, 6), (10, 8), (8, 10)])
+def test_invalid_geometry_rejected_out_untouched(W, H, sh):
+    d = torch.zeros((H, W), dtype=torch.uint8, device="cuda")
+    o = torch.full((H, W), 7, dtype=torch.uint8, device="cuda")
+    with pytest.raises(SharpError) as e:
+        sh.run(d, DEFAULT, o)
+    assert e.value.code == SHARP_EINVAL
+    assert bool((o == 7).all())
+
+
+def test_invalid_params_and_overlap_rejected(sh):
+    d = torch.zeros((64, 64), dtype=torch.uint8, device="cuda")
+    o = torch.full((64, 64), 7, dtype=torch.uint8, device="cuda")
+    for bad in [(float("nan"), 0.5, 0.5, 2.0), (1.0, 5.0, 0.5, 2.0), (1.0, 0.5, -0.1, 2.0),
+                (1.0, 0.5, 0.5, 0.0), (17.0, 0.5, 0.5, 2.0)]:
+        with pytest.raises(SharpError) as e:
+            sh.run(d, bad, o)
+        assert e.value.code == SHARP_EINVAL
+    assert bool((o == 7).all())
+    big = torch.zeros((2, 64, 64), dtype=torch.uint8, device="cuda")
+    with pytest.raises(SharpError) as e:
+        sh.run(big[0], DEFAULT, big[0])  # in place
+    assert e.value.code == SHARP_EINVAL
