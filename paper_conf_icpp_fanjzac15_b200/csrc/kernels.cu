@@ -27,6 +27,7 @@
 #include <cuda_fp16.h>
 #include <stdint.h>
 
+#include "device_common.cuh"
 #include "kernels.h"
 
 namespace sharp {
@@ -38,53 +39,7 @@ constexpr int kTileRows = 32;          // rows per warp tile (multiple of 4)
 constexpr int kWarps = 4;              // warps per CTA
 constexpr int kThreads = kWarps * 32;
 
-// ---------------------------------------------------------------- helpers
-__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t s) {
-  return __byte_perm(a, b, s);
-}
-__device__ __forceinline__ __half2 H(uint32_t u) {
-  __half2 h;
-  *reinterpret_cast<uint32_t *>(&h) = u;
-  return h;
-}
-__device__ __forceinline__ uint32_t U32(__half2 h) { return *reinterpret_cast<uint32_t *>(&h); }
-__device__ __forceinline__ uint32_t hadd(uint32_t a, uint32_t b) { return U32(__hadd2(H(a), H(b))); }
-__device__ __forceinline__ uint32_t hsub(uint32_t a, uint32_t b) { return U32(__hsub2(H(a), H(b))); }
-__device__ __forceinline__ uint32_t hfma(uint32_t a, uint32_t b, uint32_t c) {
-  return U32(__hfma2(H(a), H(b), H(c)));
-}
-__device__ __forceinline__ uint32_t habsadd(uint32_t a, uint32_t b) {
-  return U32(__hadd2(__habs2(H(a)), __habs2(H(b))));
-}
-// f32 + f16 (sm_100 mixed-precision add, one FHADD): exact here.
-__device__ __forceinline__ float add_f32_f16(uint16_t a, float c) {
-  float d;
-  asm("add.f32.f16 %0, %1, %2;" : "=f"(d) : "h"(a), "f"(c));
-  return d;
-}
-__device__ __forceinline__ uint16_t lo16(uint32_t u) { return (uint16_t)(u & 0xffffu); }
-__device__ __forceinline__ uint16_t hi16(uint32_t u) { return (uint16_t)(u >> 16); }
-__device__ __forceinline__ uint32_t cvt_u8(float a) {  // round-half-even, saturate to [0,255] (R14)
-  uint32_t r;
-  asm("cvt.rni.sat.u8.f32 %0, %1;" : "=r"(r) : "f"(a));
-  return r;
-}
-__device__ __forceinline__ float2 lds_v2(uint32_t addr) {
-  float2 v;
-  asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(addr));
-  return v;
-}
-
-constexpr uint32_t kF16Bias = 0x64646464u;    // byte 0x64 -> f16 exponent of 1024
-constexpr uint32_t kMinus1024 = 0xE400E400u;  // (-1024, -1024) as f16x2
-constexpr uint32_t kTwo = 0x40004000u;        // (2, 2)
-constexpr uint32_t kF16_255 = 0x5BF8u;        // 255.0 as f16
-
-// A row of the lane's 8 pixels plus one halo column each side, as words:
-// pw = columns c0-4..c0-1, w0 = c0..c0+3, w1 = c0+4..c0+7, nw = c0+8..c0+11.
-struct Words {
-  uint32_t pw, w0, w1, nw;
-};
+using namespace dev;
 
 __device__ __forceinline__ uint32_t ldw(const uint8_t *__restrict__ img, int W, int H, int r, int c) {
   if (r < 0 || r >= H || c < 0 || c >= W) return 0u;  // outside the image: 0
@@ -104,74 +59,6 @@ __device__ __forceinline__ Words load_row(const uint8_t *__restrict__ img, int W
   return x;
 }
 
-// Pair layout (f16x2, low half first):
-//   p[0] = (c0,   c0+2)   p[1] = (c0+1, c0+3)   p[2] = (c0+4, c0+6)   p[3] = (c0+5, c0+7)
-// Pixel x (0..7) lives in pair kPair[x], half kHalf[x].
-__device__ __forceinline__ int pair_of(int x) { return (x & 1) + ((x >> 2) << 1); }
-__device__ __forceinline__ int half_of(int x) { return (x >> 1) & 1; }
-
-// Per image row: what the 3-row window needs.
-struct RowD {
-  uint32_t h[4];   // right - left neighbour (for Gx)
-  uint32_t s[4];   // left + 2 centre + right (for Gy)
-  uint32_t mx[4];  // max of left/centre/right (u16 order of non-negative f16 == value order)
-  uint32_t mn[4];
-  uint32_t c[4];   // centre value
-};
-
-template <bool kMinMax>
-__device__ __forceinline__ RowD derive(const Words &x) {
-  const uint32_t E0 = hadd(prmt(x.w0, kF16Bias, 0x4240), kMinus1024);  // (c0, c0+2)
-  const uint32_t O0 = hadd(prmt(x.w0, kF16Bias, 0x4341), kMinus1024);  // (c0+1, c0+3)
-  const uint32_t E1 = hadd(prmt(x.w1, kF16Bias, 0x4240), kMinus1024);  // (c0+4, c0+6)
-  const uint32_t O1 = hadd(prmt(x.w1, kF16Bias, 0x4341), kMinus1024);  // (c0+5, c0+7)
-  const uint32_t PO = hadd(prmt(x.pw, kF16Bias, 0x4341), kMinus1024);  // (c0-3, c0-1)
-  const uint32_t NE = hadd(prmt(x.nw, kF16Bias, 0x4240), kMinus1024);  // (c0+8, c0+10)
-  const uint32_t p[4] = {E0, O0, E1, O1};
-  const uint32_t l[4] = {prmt(PO, O0, 0x5432), E0, prmt(O0, O1, 0x5432), E1};
-  const uint32_t r[4] = {O0, prmt(E0, E1, 0x5432), O1, prmt(E1, NE, 0x5432)};
-  RowD d;
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    d.c[i] = p[i];
-    d.h[i] = hsub(r[i], l[i]);
-    d.s[i] = hadd(hfma(kTwo, p[i], l[i]), r[i]);
-    if (kMinMax) {
-      d.mx[i] = __vimax3_u16x2(l[i], p[i], r[i]);
-      d.mn[i] = __vimin3_u16x2(l[i], p[i], r[i]);
-    }
-  }
-  return d;
-}
-
-// pEdge of the middle row b (L166: |Gx| + |Gy|, standard Sobel pair, R7).
-__device__ __forceinline__ void sobel(const RowD &a, const RowD &b, const RowD &c, uint32_t pe[4]) {
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const uint32_t gx = hadd(hfma(kTwo, b.h[i], a.h[i]), c.h[i]);
-    const uint32_t gy = hsub(c.s[i], a.s[i]);
-    pe[i] = habsadd(gx, gy);
-  }
-}
-
-// Zero the pEdge lane of pixel x (frame column).
-__device__ __forceinline__ void zero_px(uint32_t v[4], int x, uint32_t fill) {
-#pragma unroll
-  for (int i = 0; i < 8; ++i)
-    if (i == x) {
-      const int p = pair_of(i);
-      v[p] = half_of(i) ? ((v[p] & 0xffffu) | (fill << 16)) : ((v[p] & 0xffff0000u) | fill);
-    }
-}
-
-// Sum of the 4x4 block of bytes in words a..d (one column of D, times 16).
-__device__ __forceinline__ uint32_t blk(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
-  uint32_t s = __dp4a(a, 0x01010101u, 0u);
-  s = __dp4a(b, 0x01010101u, s);
-  s = __dp4a(c, 0x01010101u, s);
-  return __dp4a(d, 0x01010101u, s);
-}
-
 struct Block {  // 4 rows of words + the four D sums (16*D) of columns j0-1..j0+2
   Words r[4];
   float S[4];
@@ -181,23 +68,17 @@ __device__ __forceinline__ void load_block(Block &B, const uint8_t *__restrict__
                                            int c0, int lane) {
 #pragma unroll
   for (int a = 0; a < 4; ++a) B.r[a] = load_row(img, W, H, 4 * k + a, c0, lane);
-  B.S[0] = (float)blk(B.r[0].pw, B.r[1].pw, B.r[2].pw, B.r[3].pw);
-  B.S[1] = (float)blk(B.r[0].w0, B.r[1].w0, B.r[2].w0, B.r[3].w0);
-  B.S[2] = (float)blk(B.r[0].w1, B.r[1].w1, B.r[2].w1, B.r[3].w1);
-  B.S[3] = (float)blk(B.r[0].nw, B.r[1].nw, B.r[2].nw, B.r[3].nw);
+  B.S[0] = (float)blk4(B.r[0].pw, B.r[1].pw, B.r[2].pw, B.r[3].pw);
+  B.S[1] = (float)blk4(B.r[0].w0, B.r[1].w0, B.r[2].w0, B.r[3].w0);
+  B.S[2] = (float)blk4(B.r[0].w1, B.r[1].w1, B.r[2].w1, B.r[3].w1);
+  B.S[3] = (float)blk4(B.r[0].nw, B.r[1].nw, B.r[2].nw, B.r[3].nw);
 }
 
 // ------------------------------------------------------- upscale border (R4, R5)
-// line(v, n)[c] of L140, given the 16*D values x = v[c>>2], y = v[(c>>2)+1]:
-// k = c & 3;  k == 0 -> x, else ((4-k) x + k y) / 4;  as U: divide by 16.
-__device__ __forceinline__ float line_val(float x16, float y16, int k) {
-  return __fmul_rn(__fadd_rn(__fmul_rn((float)(4 - k), x16), __fmul_rn((float)k, y16)), 1.0f / 64.0f);
-}
-
 // Final value of U at a pixel of the 2-pixel ring (last writer of steps
 // i..vii of L140-L142).  Sc = 16*D of the current D row block (row k) for
 // columns j0-1..j0+2, Sn = the next D row (k+1); j0 = c0/4; r = 4k + a'.
-__device__ float ring_u(int r, int c, int W, int H, int j0, const float Sc[4], const float Sn[4]) {
+__device__ __forceinline__ float ring_u(int r, int c, int W, int H, int j0, const float (&Sc)[4], const float (&Sn)[4]) {
   const int w = W >> 2, h = H >> 2;
   auto col = [&](int j) { return j - j0 + 1; };  // index into Sc/Sn
   if (r >= H - 2 && c >= W - 2) {                 // (vii): third last of last column = D[h-1][w-1]
@@ -250,12 +131,12 @@ __global__ void __launch_bounds__(kThreads) edge_sum_kernel(const uint8_t *__res
 #pragma unroll
         for (int i = 0; i < 4; ++i) pe[i] = 0u;
       }
-      if (c0 == 0) zero_px(pe, 0, 0u);                          // first column
-      if (c0 <= W - 1 && W - 1 < c0 + kPx) zero_px(pe, W - 1 - c0, 0u);  // last column
+      if (c0 == 0) set_px(pe, 0, 0u);                          // first column
+      if (c0 <= W - 1 && W - 1 < c0 + kPx) set_px(pe, W - 1 - c0, 0u);  // last column
       if (c0 + kPx > W) {                                       // pixels beyond the image
 #pragma unroll
         for (int x = 0; x < kPx; ++x)
-          if (c0 + x >= W) zero_px(pe, x, 0u);
+          if (c0 + x >= W) set_px(pe, x, 0u);
       }
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
@@ -303,12 +184,6 @@ __global__ void __launch_bounds__(kThreads) edge_sum_kernel(const uint8_t *__res
 // =========================================================================
 // Pass 2: everything else, fused.
 // =========================================================================
-// Upscale weights (R3): P = [[7,1],[5,3],[3,5],[1,7]] / 8.  For the lane's 8
-// columns x = 0..7 (column 4*j0 + x), the horizontal pair of D columns
-// (relative index jl, jl+1 into S[]) and the left weight *8.
-__device__ __forceinline__ int wl_of(int x) { return (x & 3) == 0 ? 3 : (x & 3) == 1 ? 1 : (x & 3) == 2 ? 7 : 5; }
-__device__ __forceinline__ int jl_of(int x) { return x < 2 ? 0 : (x < 6 ? 1 : 2); }
-
 __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__restrict__ imgs, int W, int H,
                                                            int tiles_x, int tiles_y,
                                                            const float2 *__restrict__ luts,
@@ -363,14 +238,14 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
           }
         }
         if (c0 == 0) {
-          zero_px(pe, 0, 0u);
-          zero_px(MX, 0, kF16_255);
-          zero_px(MN, 0, 0u);
+          set_px(pe, 0, 0u);
+          set_px(MX, 0, kF16_255);
+          set_px(MN, 0, 0u);
         }
         if (c0 <= W - 1 && W - 1 < c0 + kPx) {
-          zero_px(pe, W - 1 - c0, 0u);
-          zero_px(MX, W - 1 - c0, kF16_255);
-          zero_px(MN, W - 1 - c0, 0u);
+          set_px(pe, W - 1 - c0, 0u);
+          set_px(MX, W - 1 - c0, kF16_255);
+          set_px(MN, W - 1 - c0, 0u);
         }
         // Vertical interpolation of the three D-column sums (16*D):
         //   a' = 0,1: U block row k-1, weights (3,5),(1,7) on D rows (k-1,k)
@@ -392,8 +267,8 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
           NU[x] = __fmaf_rn(-(8.0f - wl) * (1.0f / 1024.0f), V[jl + 1], __fmul_rn(-wl * (1.0f / 1024.0f), V[jl]));
         }
         if (r < 2 || r >= H - 2 || ring_cols) {  // the 2-pixel upscale border ring
-          const float *Sc = cur.S;  // D row k: row 0 for rows 0,1; row h-1 for rows H-2,H-1
-          const float *Sn = next.S;
+          const float(&Sc)[4] = cur.S;  // D row k: row 0 for rows 0,1; row h-1 for rows H-2,H-1
+          const float(&Sn)[4] = next.S;
 #pragma unroll
           for (int x = 0; x < 8; ++x) {
             const int c = c0 + x;
@@ -410,7 +285,7 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
           const uint16_t mx_h = hi ? hi16(MX[p]) : lo16(MX[p]);
           const uint16_t mn_h = hi ? hi16(MN[p]) : lo16(MN[p]);
           const uint32_t q = __float_as_uint(add_f32_f16(pe_h, 8388608.0f));  // 2^23 + pEdge
-          const float2 L = lds_v2(q * 8u + lut_base);                        // {adj, osc}
+          const float2 L = lds_f2(q * 8u + lut_base);                        // {adj, osc}
           const float E = add_f32_f16(c_h, NU[x]);                           // pError = O - U (L148)
           const float P = __fmaf_rn(L.x, E, -NU[x]);                         // preliminary (L178)
           const float mxf = add_f32_f16(mx_h, 0.0f), mnf = add_f32_f16(mn_h, 0.0f);

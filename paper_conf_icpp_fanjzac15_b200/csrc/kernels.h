@@ -26,6 +26,15 @@ cudaError_t launch_edge_sum(const uint8_t *imgs, int n, int W, int H, const Para
 cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts,
                            uint8_t *outs, cudaStream_t stream);
 
+// TMA-staged persistent variants (kernels_tma.cu): same contract, used when
+// tma_supported() (W % 16 == 0, 16-byte aligned input, 8-byte aligned output).
+bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);
+cudaError_t launch_edge_sum_tma(const uint8_t *imgs, int n, int W, int H, const Params &p,
+                                unsigned long long *sums, unsigned int *counters, float2 *luts,
+                                double *means, cudaStream_t stream);
+cudaError_t launch_sharpen_tma(const uint8_t *imgs, int n, int W, int H, const float2 *luts,
+                               uint8_t *outs, cudaStream_t stream);
+
 // Kernel launches issued per (pass-1, pass-2) chunk.
 constexpr int kLaunchesPerChunk = 2;
 

@@ -42,6 +42,7 @@ struct sharp_ctx {
   cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
   int nslots = 3;
   int chunk_cfg = 0;
+  bool use_tma = true;  // SHARP_FORCE_GENERIC=1 at sharp_create selects the LDG kernels
   Slot slots[kMaxSlots];
   size_t slot_chunk_frames = 0, slot_stage_bytes = 0;  // capacity of the slot buffers
   unsigned long long *sums = nullptr;
@@ -228,11 +229,19 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   for (size_t f0 = 0; f0 < (size_t)n; f0 += chunk) {
     const int cn = (int)std::min(chunk, (size_t)n - f0);
     const double px = (double)cn * fb;
+    const uint8_t *ci = din + f0 * fb;
+    uint8_t *co = dout + f0 * fb;
+    const bool tma = ctx->use_tma && sharp::tma_supported(ci, co, w, h);
     CK(timed(ctx, st, 1, px, [&] {
-      return sharp::launch_edge_sum(din + f0 * fb, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters,
-                                    slot.luts, ctx->means + frame_base + f0, st);
+      return tma ? sharp::launch_edge_sum_tma(ci, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters,
+                                              slot.luts, ctx->means + frame_base + f0, st)
+                 : sharp::launch_edge_sum(ci, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters,
+                                          slot.luts, ctx->means + frame_base + f0, st);
     }));
-    CK(timed(ctx, st, 2, px, [&] { return sharp::launch_sharpen(din + f0 * fb, cn, w, h, slot.luts, dout + f0 * fb, st); }));
+    CK(timed(ctx, st, 2, px, [&] {
+      return tma ? sharp::launch_sharpen_tma(ci, cn, w, h, slot.luts, co, st)
+                 : sharp::launch_sharpen(ci, cn, w, h, slot.luts, co, st);
+    }));
     *launches += sharp::kLaunchesPerChunk;
   }
   return SHARP_OK;
@@ -359,6 +368,10 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
     return e != cudaSuccess ? SHARP_ECUDA : SHARP_EINVAL;
   }
   ctx->device = dev;
+  {
+    const char *g = getenv("SHARP_FORCE_GENERIC");
+    ctx->use_tma = !(g && g[0] == '1');
+  }
   ctx->nslots = c.streams ? c.streams : 3;
   ctx->chunk_cfg = c.chunk_frames;
   int rc = SHARP_OK;

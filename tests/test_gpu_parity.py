@@ -26,10 +26,19 @@ PARAMS = [
 ]
 
 
-@pytest.fixture(scope="module")
-def sh():
+@pytest.fixture(scope="module", params=["auto", "generic"])
+def sh(request):
+    """A context on the automatic kernel path (TMA-staged persistent kernels
+    when W % 16 == 0) and one forced onto the generic LDG kernels."""
     assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import os
+    old = os.environ.get("SHARP_FORCE_GENERIC")
+    os.environ["SHARP_FORCE_GENERIC"] = "1" if request.param == "generic" else "0"
     s = Sharpener()
+    if old is None:
+        del os.environ["SHARP_FORCE_GENERIC"]
+    else:
+        os.environ["SHARP_FORCE_GENERIC"] = old
     yield s
     s.close()
 
@@ -54,7 +63,9 @@ def assert_parity(sh, img, prm=DEFAULT):
 
 
 SIZES = [(8, 8), (12, 8), (8, 12), (16, 16), (20, 12), (64, 48), (100, 36), (252, 20), (260, 36),
-         (300, 68), (516, 44), (1028, 40)]
+         (300, 68), (516, 44), (1028, 40),
+         # W % 16 == 0 (TMA path): one warp tile, tile + 16, CTA tile edges, ragged rows
+         (16, 8), (32, 12), (240, 36), (256, 40), (480, 68), (960, 36), (976, 44), (1920, 36)]
 
 
 @pytest.mark.parametrize("W,H", SIZES)
