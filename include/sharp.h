@@ -124,11 +124,14 @@ int sharp_get_batch_sums(sharp_ctx *ctx, uint64_t *sums, int n);
 /* Per-kernel device time accounting (CUDA events around every launch, on
  * the launch stream).  enable != 0 starts (and resets) accounting. */
 typedef struct {
-  float pass1_ms;      /* summed duration of edge_sum launches (Sobel+reduction+LUT) */
-  float pass2_ms;      /* summed duration of sharpen launches (fused per-pixel pass)  */
+  float pass1_ms;      /* generic path: summed duration of edge_sum launches        */
+  float pass2_ms;      /* generic path: summed duration of sharpen launches         */
   int pass1_launches;
   int pass2_launches;
-  double pixels;       /* pixels processed by the accounted launches               */
+  float step_ms;       /* TMA path: summed duration of step launches (pass 1 of
+                          chunk c+1 fused with pass 2 of chunk c)                  */
+  int step_launches;
+  double pixels;       /* output pixels completed by the accounted launches         */
 } sharp_kernel_times;
 int sharp_set_profiling(sharp_ctx *ctx, int enable);
 /* Waits for the launch stream, then returns the accumulated times. */

@@ -39,6 +39,7 @@ class SharpStats(ctypes.Structure):
 class SharpKernelTimes(ctypes.Structure):
     _fields_ = [("pass1_ms", ctypes.c_float), ("pass2_ms", ctypes.c_float),
                 ("pass1_launches", ctypes.c_int), ("pass2_launches", ctypes.c_int),
+                ("step_ms", ctypes.c_float), ("step_launches", ctypes.c_int),
                 ("pixels", ctypes.c_double)]
 
 

@@ -48,6 +48,8 @@ struct sharp_ctx {
   unsigned long long *sums = nullptr;
   double *means = nullptr;
   size_t frames_cap = 0;
+  unsigned int *tcounters = nullptr;  // dynamic-scheduling task counters, one per step launch
+  size_t tcounters_cap = 0;
   int last_frames = 0;
   sharp_stats stats{};
   // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2)
@@ -131,6 +133,18 @@ int ensure_frames(sharp_ctx *ctx, size_t n) {
   return SHARP_OK;
 }
 
+int ensure_task_counters(sharp_ctx *ctx, size_t n) {
+  if (n <= ctx->tcounters_cap) return SHARP_OK;
+  CK(cudaStreamSynchronize(ctx->stream));
+  for (int i = 0; i < ctx->nslots; ++i) CK(cudaStreamSynchronize(ctx->slots[i].stream));
+  cudaFree(ctx->tcounters);
+  ctx->tcounters = nullptr;
+  ctx->tcounters_cap = 0;
+  CK(cudaMalloc(&ctx->tcounters, n * sizeof(unsigned int)));
+  ctx->tcounters_cap = n;
+  return SHARP_OK;
+}
+
 void free_slot(Slot &s) {
   cudaFree(s.d_in);
   cudaFree(s.d_out);
@@ -159,7 +173,7 @@ int ensure_slots(sharp_ctx *ctx, size_t chunk, size_t frame_bytes, bool staging)
     free_slot(s);
     CK(cudaMalloc(&s.counters, cap * sizeof(unsigned int)));
     CK(cudaMemset(s.counters, 0, cap * sizeof(unsigned int)));
-    CK(cudaMalloc(&s.luts, cap * sharp::kLutSize * sizeof(float2)));
+    CK(cudaMalloc(&s.luts, 2 * cap * sharp::kLutSize * sizeof(float2)));  // two chunk parities
     if (stage) {
       CK(cudaMalloc(&s.d_in, stage));
       CK(cudaMalloc(&s.d_out, stage));
@@ -221,27 +235,53 @@ cudaError_t timed(sharp_ctx *ctx, cudaStream_t st, int kind, double px, F launch
   return e;
 }
 
-// Device-resident batch: chunks of frames, pass 1 then pass 2 per chunk, on
-// one stream (the chunk's input is still in L2 when pass 2 re-reads it).
+// Device-resident batch on one stream, in chunks of frames.
+//  * TMA path: launch c = pass 1 of chunk c + pass 2 of chunk c-1 (one
+//    dynamically scheduled step kernel); chunk c's input is still in L2 when
+//    launch c+1 re-reads it.  LUT buffers alternate between chunk parities.
+//  * generic path: pass 1 then pass 2 per chunk.
+// `tc` points at this call's zeroed task counters (one per step launch).
 int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, const sharp::Params &prm,
-                   uint8_t *dout, cudaStream_t st, Slot &slot, size_t chunk, size_t frame_base, int *launches) {
+                   uint8_t *dout, cudaStream_t st, Slot &slot, size_t chunk, size_t frame_base, int *launches,
+                   unsigned int *tc) {
   const size_t fb = (size_t)w * h;
+  const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
+  const bool tma = ctx->use_tma && sharp::tma_supported(din, dout, w, h);
+  if (tma) {
+    for (size_t c = 0; c <= nchunks; ++c) {
+      sharp::StepLaunch a;
+      if (c < nchunks) {
+        const size_t f0 = c * chunk;
+        a.in1 = din + f0 * fb;
+        a.n1 = (int)std::min(chunk, (size_t)n - f0);
+        a.sums1 = ctx->sums + frame_base + f0;
+        a.means1 = ctx->means + frame_base + f0;
+        a.counters1 = slot.counters;
+        a.luts1 = slot.luts + (c & 1) * chunk * sharp::kLutSize;
+      }
+      if (c > 0) {
+        const size_t f0 = (c - 1) * chunk;
+        a.in2 = din + f0 * fb;
+        a.n2 = (int)std::min(chunk, (size_t)n - f0);
+        a.luts2 = slot.luts + ((c - 1) & 1) * chunk * sharp::kLutSize;
+        a.out2 = dout + f0 * fb;
+      }
+      a.task_counter = tc + c;
+      CK(timed(ctx, st, 3, (double)a.n2 * fb, [&] { return sharp::launch_step_tma(a, w, h, prm, st); }));
+      *launches += 1;
+    }
+    return SHARP_OK;
+  }
   for (size_t f0 = 0; f0 < (size_t)n; f0 += chunk) {
     const int cn = (int)std::min(chunk, (size_t)n - f0);
     const double px = (double)cn * fb;
     const uint8_t *ci = din + f0 * fb;
     uint8_t *co = dout + f0 * fb;
-    const bool tma = ctx->use_tma && sharp::tma_supported(ci, co, w, h);
     CK(timed(ctx, st, 1, px, [&] {
-      return tma ? sharp::launch_edge_sum_tma(ci, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters,
-                                              slot.luts, ctx->means + frame_base + f0, st)
-                 : sharp::launch_edge_sum(ci, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters,
-                                          slot.luts, ctx->means + frame_base + f0, st);
+      return sharp::launch_edge_sum(ci, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters, slot.luts,
+                                    ctx->means + frame_base + f0, st);
     }));
-    CK(timed(ctx, st, 2, px, [&] {
-      return tma ? sharp::launch_sharpen_tma(ci, cn, w, h, slot.luts, co, st)
-                 : sharp::launch_sharpen(ci, cn, w, h, slot.luts, co, st);
-    }));
+    CK(timed(ctx, st, 2, px, [&] { return sharp::launch_sharpen(ci, cn, w, h, slot.luts, co, st); }));
     *launches += sharp::kLaunchesPerChunk;
   }
   return SHARP_OK;
@@ -269,10 +309,14 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   if ((rc = ensure_frames(ctx, (size_t)n))) return rc;
   if ((rc = ensure_slots(ctx, chunk, fb, staged))) return rc;
   int launches = 0;
+  const size_t nchunks_all = ((size_t)n + chunk - 1) / chunk;
+  if ((rc = ensure_task_counters(ctx, 2 * nchunks_all + 2))) return rc;
   CK(cudaMemsetAsync(ctx->sums, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
-  if (!async) CK(cudaEventRecord(ctx->ev_start, ctx->stream));
+  CK(cudaMemsetAsync(ctx->tcounters, 0, (2 * nchunks_all + 2) * sizeof(unsigned int), ctx->stream));
+  CK(cudaEventRecord(ctx->ev_start, ctx->stream));
   if (!staged) {
-    if ((rc = enqueue_device(ctx, in, n, w, h, prm, out, ctx->stream, ctx->slots[0], chunk, 0, &launches)))
+    if ((rc = enqueue_device(ctx, in, n, w, h, prm, out, ctx->stream, ctx->slots[0], chunk, 0, &launches,
+                             ctx->tcounters)))
       return rc;
   } else {
     // Host pipeline (sec. V-A): chunk c on slot c % nslots; H2D || kernels || D2H.
@@ -302,7 +346,9 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
         dsrc = sl.d_in;
       }
       uint8_t *ddst = (kout == kDevice) ? out + f0 * fb : sl.d_out;
-      if ((rc = enqueue_device(ctx, dsrc, (int)cn, w, h, prm, ddst, sl.stream, sl, cn, f0, &launches))) return rc;
+      if ((rc = enqueue_device(ctx, dsrc, (int)cn, w, h, prm, ddst, sl.stream, sl, cn, f0, &launches,
+                               ctx->tcounters + 2 * c)))
+        return rc;
       if (kout != kDevice) {
         uint8_t *hdst = (kout == kPinned) ? out + f0 * fb : sl.h_out;
         CK(cudaMemcpyAsync(hdst, sl.d_out, bytes, cudaMemcpyDeviceToHost, sl.stream));
@@ -414,6 +460,7 @@ void sharp_destroy(sharp_ctx *ctx) {
   }
   cudaFree(ctx->sums);
   cudaFree(ctx->means);
+  cudaFree(ctx->tcounters);
   for (auto &r : ctx->recs) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -487,10 +534,14 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t) {
     if (r.kind == 1) {
       t->pass1_ms += ms;
       t->pass1_launches++;
-      t->pixels += r.px;
-    } else {
+    } else if (r.kind == 2) {
       t->pass2_ms += ms;
       t->pass2_launches++;
+      t->pixels += r.px;
+    } else {
+      t->step_ms += ms;
+      t->step_launches++;
+      t->pixels += r.px;
     }
   }
   return SHARP_OK;
