@@ -28,25 +28,24 @@ cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float
 
 // TMA-staged, dynamically scheduled step kernel (kernels_tma.cu), used when
 // tma_supported() (W % 16 == 0, 16-byte aligned input, 8-byte aligned output).
-// One launch = pass 1 of chunk "1" (n1 frames, may be 0) + pass 2 of chunk
-// "2" (n2 frames, may be 0).  Chunk 2's LUTs must have been built by an
-// earlier launch; chunk 1's sums must be zero and counters re-armed on entry.
-// task_counter must be zero on entry.
+// One launch = LUT build (mean from the complete sums) + pass 2 of chunk "2"
+// (n2 frames, may be 0) and pass 1 of chunk "1" (n1 frames, may be 0).
+// Chunk 2's sums must be complete (an earlier launch's pass 1); chunk 1's
+// sums, lut_done2 and task_counter must be zero on entry.
 struct StepLaunch {
   const uint8_t *in1 = nullptr;
   int n1 = 0;
   unsigned long long *sums1 = nullptr;
-  double *means1 = nullptr;
-  unsigned int *counters1 = nullptr;
-  float2 *luts1 = nullptr;
   const uint8_t *in2 = nullptr;
   int n2 = 0;
-  const float2 *luts2 = nullptr;
+  const unsigned long long *sums2 = nullptr;
+  double *means2 = nullptr;
+  float2 *luts2 = nullptr;
+  unsigned int *lut_done2 = nullptr;
   uint8_t *out2 = nullptr;
   unsigned int *task_counter = nullptr;
 };
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);
-int tma_tasks(int n, int W, int H);
 cudaError_t launch_step_tma(const StepLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
 
 // Kernel launches issued per (pass-1, pass-2) chunk.

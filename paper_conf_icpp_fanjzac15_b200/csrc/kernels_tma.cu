@@ -1,30 +1,36 @@
-// TMA-staged, dynamically scheduled sm_100a "step" kernel (the main path;
-// needs W % 16 == 0 and 16-byte aligned frames -- the TMA tensor-map rules).
+// TMA-staged, warp-specialised, dynamically scheduled sm_100a "step" kernel
+// (the main path; needs W % 16 == 0 and 16-byte aligned frames -- the TMA
+// tensor-map rules).
 //
-// One launch runs two kinds of tasks, grabbed in order from a global counter
-// by persistent CTAs (2 per SM):
-//   * pass-1 tasks of chunk c+1: Sobel (L158-L172) + reduction (L174, sec.
-//     V-C); the CTA finishing a frame's last pass-1 task computes the frame's
-//     mean and lookup tables (last-block-done);
-//   * pass-2 tasks of chunk c: the fused per-pixel pipeline (downscale L130,
-//     upscale L140-L146, pError L148, Sobel, 3x3 max/min L182, strength L178,
-//     preliminary L178, overshoot L180-L212) -> u8.
-// Pass-1 tasks come first, so the frames' table builds overlap the pass-2
-// tasks of other CTAs, and the chunk's input is re-read from L2 by pass 2 in
-// the next launch.
+// One launch c runs three kinds of tasks, grabbed in this order from a global
+// counter by persistent CTAs (2 per SM):
+//   1. LUT tasks of chunk c-1: the per-frame lookup tables
+//      adj(p) = A (p/m)^gamma (strength, L178) and
+//      osc(p) = clamp(G exp(-p/(K m)), 0, 1) (oscStrength, L184),
+//      128 entries per task, f64 rounded once (R9, R11);
+//   2. pass-1 tasks of chunk c: Sobel (L158-L172) + reduction (L174, sec.
+//      V-C): warp shuffle reduction, u64 atomics, and the last warp of a frame
+//      computes its mean (last-block-done);
+//   3. pass-2 tasks of chunk c-1: the fused per-pixel pipeline (downscale
+//      L130, upscale L140-L146, pError L148, Sobel, 3x3 max/min L182,
+//      strength lookup, preliminary L178, overshoot L180-L212) -> u8.
+// A pass-2 task's producer waits until its frame's LUT tasks are done (they
+// were grabbed earlier, so this cannot deadlock).  The chunk's input is
+// re-read from L2 by pass 2 in the next launch.
 //
-// A task is a CTA tile of 4 warp tiles side by side; a warp tile is 240
-// output columns x 24 rows of one frame.  Its pixels plus halo are fetched by
-// one cp.async.bulk.tensor (TMA) box into shared memory (out-of-image pixels
-// are zero-filled by the TMA unit: no bounds checks in the pixel loops), and
-// the next task's boxes are in flight while the current one is computed.
-// Each lane owns 8 adjacent columns and walks down the rows with a 3-row
-// window; the row loop is unrolled 12 rows (lcm of the 3-row window and the
-// 4-row downscale block) so the window never needs register moves.  Lanes 30
-// and 31 fetch the right/left halo columns and hand them out by shuffle.
+// CTA = 4 compute warps + 1 producer warp.  A pass-1/2 task is a CTA tile of
+// 4 warp tiles side by side; a warp tile is 240 output columns x 24 rows.
+// The producer grabs tasks and issues one cp.async.bulk.tensor (TMA) box per
+// warp tile (out-of-image pixels are zero-filled by the TMA unit: no bounds
+// checks in the pixel loops) plus a bulk copy of the frame's LUT, into one of
+// two smem stages guarded by full/empty mbarriers -- no CTA-wide barrier in
+// the steady state.  Each lane owns 8 adjacent columns and walks down the
+// rows with a 3-row window unrolled by 3 (no register moves); lanes 30 and 31
+// fetch the right/left halo columns and hand them out by shuffle.
 //
-// Image border: rows 0,1,H-2,H-1 by a warp-uniform branch; columns 0,1,W-2,
-// W-1 by a specialised scalar pass of the warps whose tile touches them.
+// Image border (the 2-pixel ring: upscale border lines L140-L142, Sobel frame
+// L160, overshoot frame L208): recomputed by a specialised scalar pass of the
+// warps whose tile touches it, after the interior code wrote the tile.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
@@ -41,26 +47,30 @@ namespace {
 using namespace dev;
 
 constexpr int kTW = 240;     // output columns per warp tile (lanes 0..29 x 8 px)
-constexpr int kTH = 24;      // output rows per warp tile (two 12-row bodies)
-constexpr int kWarpsT = 4;   // warp tiles per CTA tile
+constexpr int kTH = 12;      // output rows per warp tile
+constexpr int kCtasPerSm = 3;  // smem ~67 KB per CTA
+constexpr int kWarpsT = 4;   // compute warps = warp tiles per CTA tile
 constexpr int kCtaCols = kTW * kWarpsT;
-constexpr int kThreadsT = 32 * kWarpsT;
+constexpr int kThreadsT = 32 * (kWarpsT + 1);  // + producer warp
+constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task
+constexpr int kLutTasks = kLutSize / kLutPerTask;
 // The TMA box's innermost start coordinate must be 16-byte aligned and a box
 // dimension is at most 256, so frames are viewed as 4-D [n][H][W/16][16] and
 // a warp tile's box is {16, 17 chunks, rows, 1}: 272 columns from C0w-16.
 constexpr int kChunks = 17;
 constexpr int kPitch = 16 * kChunks;  // smem row pitch: columns C0w-16 .. C0w+255
 constexpr int kCol0 = 16;             // smem column of C0w
-constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+27
-constexpr int kRows1 = kTH + 2;       // pass-1 box rows: R0-1 .. R0+24
-constexpr int kBox2 = kPitch * kRows2;  // 8704 = 68 * 128
-constexpr int kBox1 = kPitch * kRows1;  // 7072
-constexpr int kSlot = kBox2;            // per-warp smem slot (128-B aligned)
+constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+kTH+3
+constexpr int kRows1 = kTH + 2;       // pass-1 box rows: R0-1 .. R0+kTH
+constexpr int kBox2 = kPitch * kRows2;
+constexpr int kBox1 = kPitch * kRows1;
+constexpr int kSlot = (kBox2 + 127) / 128 * 128;  // per-warp smem slot (128-B aligned)
 constexpr int kLutBytes = kLutSize * 8;
 constexpr int kStage = kWarpsT * kSlot + kLutBytes;
 constexpr int kSmem = 2 * kStage + 64;
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
-static_assert(kTH % 12 == 0, "row loop is unrolled by 12");
+static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
+static_assert(kLutSize % kLutPerTask == 0, "LUT tasks");
 
 // ------------------------------------------------------------ TMA / mbarrier
 __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
@@ -69,12 +79,15 @@ __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
 __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n"
       ".reg .pred p;\n"
       "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 1000000;\n"  // suspend (not spin) up to 1 ms
       "@!p bra WAIT_%=;\n"
       "}\n" ::"r"(bar),
       "r"(parity)
@@ -95,8 +108,19 @@ __device__ __forceinline__ void bulk_copy(uint32_t dst, const void *src, uint32_
                "l"(src), "r"(bytes), "r"(bar)
                : "memory");
 }
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void fence_barrier_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__device__ __forceinline__ unsigned int ld_acquire(const unsigned int *p) {
+  unsigned int v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// LDS address q*8 + base in one integer op.
+__device__ __forceinline__ uint32_t mad8(uint32_t q, uint32_t base) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, 8, %2;" : "=r"(r) : "r"(q), "r"(base));
+  return r;
+}
 
 // ----------------------------------------------------------- packed f32x2
 __device__ __forceinline__ unsigned long long f2pack(float a, float b) {
@@ -109,13 +133,12 @@ __device__ __forceinline__ float2 f2unpack(unsigned long long r) {
   asm("mov.b64 {%0, %1}, %2;" : "=f"(v.x), "=f"(v.y) : "l"(r));
   return v;
 }
-// (a*x + b*y) for a lane pair with the same (x, y): two single-rounding ops
-// (FMUL2 then FFMA2), bit-identical to the scalar fmul/fma pair.
-__device__ __forceinline__ float2 lin2(float x, float y, float a0, float a1, float b0, float b1) {
+// (a*x + b*y) for a lane pair with the same (x, y): FMUL2 then FFMA2, each
+// single-rounding per lane -- bit-identical to the scalar fmul/fma pair.
+__device__ __forceinline__ float2 lin2(float x, float y, unsigned long long a, unsigned long long b) {
   unsigned long long t, r;
-  const unsigned long long xx = f2pack(x, x), yy = f2pack(y, y);
-  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(t) : "l"(xx), "l"(f2pack(a0, a1)));
-  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(yy), "l"(f2pack(b0, b1)), "l"(t));
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(t) : "l"(f2pack(x, x)), "l"(a));
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(f2pack(y, y)), "l"(b), "l"(t));
   return f2unpack(r);
 }
 __device__ __forceinline__ float2 sub2(float2 a, float2 b) {
@@ -140,13 +163,15 @@ __device__ __forceinline__ void tile_of(const Geo &g, int t, int &f, int &C0, in
 
 struct StepParams {
   Geo g;
-  int n1, n2;  // pass-1 / pass-2 task counts
+  int nL, n1, n2;  // LUT / pass-1 / pass-2 task counts (in this order)
   Params prm;
+  // pass 1 (chunk c)
   unsigned long long *sums1;
-  double *means1;
-  unsigned int *counters1;
-  float2 *luts1;
-  const float2 *luts2;
+  // LUT + pass 2 (chunk c-1)
+  const unsigned long long *sums2;
+  double *means2;
+  float2 *luts2;
+  unsigned int *lut_done2;
   uint8_t *out2;
   unsigned int *task_counter;
 };
@@ -260,13 +285,13 @@ __device__ uint32_t pixel_generic(uint32_t tile, uint32_t lut, int r, int c, int
 }
 
 // ========================================================== pass 2, one row
-// Output row r (window rows a = r-1, b = r, c = r+1) of this lane.  T / B are
-// the D rows above / below for the vertical interpolation; Dc is D row k
-// (for the border lines of rows 0,1,H-2,H-1).
-template <int kA>  // r - 4k, 0..3
-__device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &T,
-                                       const float4 &B, const float4 &Dc, int r, int c0, int W, int H,
-                                       uint32_t lut_q, uint8_t *orow, bool store) {
+// Output row of this lane (window rows a = r-1, b = r, c = r+1), interior
+// formulas only.  V = vertical interpolation (x 128) of the four D columns.
+struct Wts {  // packed horizontal weights -w/1024 for pixel pairs (x, x+1)
+  unsigned long long a01, b01, a23, b23;
+};
+__device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
+                                       const Wts &wt, uint32_t lut_q, uint8_t *orow, bool store) {
   uint32_t pe[4], MX[4], MN[4];
   sobel(ra, rb, rc, pe);
 #pragma unroll
@@ -274,33 +299,13 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
     MX[i] = __vimax3_u16x2(ra.mx[i], rb.mx[i], rc.mx[i]);
     MN[i] = __vimin3_u16x2(ra.mn[i], rb.mn[i], rc.mn[i]);
   }
-  // Upscale body (L146, R3): vertical weights (wt, 8-wt) on D rows (T, B),
-  // then horizontal; NU = -U, exact.
-  constexpr float wt = (float)wt_of(kA), wb = 8.0f - wt;
-  const float V0 = __fmaf_rn(wb, B.x, __fmul_rn(wt, T.x));
-  const float V1 = __fmaf_rn(wb, B.y, __fmul_rn(wt, T.y));
-  const float V2 = __fmaf_rn(wb, B.z, __fmul_rn(wt, T.z));
-  const float V3 = __fmaf_rn(wb, B.w, __fmul_rn(wt, T.w));
-  constexpr float s = -1.0f / 1024.0f;
-  float2 nu01 = lin2(V0, V1, 3 * s, 1 * s, 5 * s, 7 * s);   // x = 0,1: (3,5), (1,7) on (V0, V1)
-  float2 nu23 = lin2(V1, V2, 7 * s, 5 * s, 1 * s, 3 * s);   // x = 2,3: (7,1), (5,3) on (V1, V2)
-  float2 nu45 = lin2(V1, V2, 3 * s, 1 * s, 5 * s, 7 * s);   // x = 4,5
-  float2 nu67 = lin2(V2, V3, 7 * s, 5 * s, 1 * s, 3 * s);   // x = 6,7
-  if (r < 2 || r >= H - 2) {  // border rows (warp-uniform): upscale border lines (L140) + frame
-    const float q0 = Dc.y, q1 = Dc.z, q2 = Dc.w;  // D row 0 (rows 0,1) or h-1 (rows H-2,H-1)
-    nu01 = make_float2(-__fmul_rn(q0, 1.0f / 16.0f), -line_val(q0, q1, 1));
-    nu23 = make_float2(-line_val(q0, q1, 2), -line_val(q0, q1, 3));
-    nu45 = make_float2(-__fmul_rn(q1, 1.0f / 16.0f), (c0 + 5 == W - 3) ? -__fmul_rn(q1, 1.0f / 16.0f) : -line_val(q1, q2, 1));
-    nu67 = make_float2(-line_val(q1, q2, 2), -line_val(q1, q2, 3));
-    if (r == 0 || r == H - 1) {  // frame: Sobel 0 (L160), no overshoot window (L208)
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        pe[i] = 0u;
-        MX[i] = kF16_255 | (kF16_255 << 16);
-        MN[i] = 0u;
-      }
-    }
-  }
+  // Upscale body (L146, R3), horizontal step on pixel pairs; NU = -U, exact.
+  //   x = 0,1: (3,5),(1,7) on (V0,V1);  x = 2,3: (7,1),(5,3) on (V1,V2)
+  //   x = 4,5: (3,5),(1,7) on (V1,V2);  x = 6,7: (7,1),(5,3) on (V2,V3)
+  const float2 nu01 = lin2(V.x, V.y, wt.a01, wt.b01);
+  const float2 nu23 = lin2(V.y, V.z, wt.a23, wt.b23);
+  const float2 nu45 = lin2(V.y, V.z, wt.a01, wt.b01);
+  const float2 nu67 = lin2(V.z, V.w, wt.a23, wt.b23);
   const float NU[8] = {nu01.x, nu01.y, nu23.x, nu23.y, nu45.x, nu45.y, nu67.x, nu67.y};
   float P[8], T8[8], osc[8];
 #pragma unroll
@@ -308,7 +313,7 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
     const int p = pair_of(x);
     const bool hi = half_of(x);
     const uint32_t qb = __float_as_uint(add_f32_f16(hi ? hi16(pe[p]) : lo16(pe[p]), 8388608.0f));  // 2^23 + pEdge
-    const float2 L = lds_f2(qb * 8u + lut_q);                                                      // {adj, osc}
+    const float2 L = lds_f2(mad8(qb, lut_q));                                                      // {adj, osc}
     const float E = add_f32_f16(hi ? hi16(rb.c[p]) : lo16(rb.c[p]), NU[x]);                       // O - U (L148)
     P[x] = __fmaf_rn(L.x, E, -NU[x]);                                                              // L178
     const float mxf = add_f32_f16(hi ? hi16(MX[p]) : lo16(MX[p]), 0.0f);
@@ -326,29 +331,15 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   if (store) *reinterpret_cast<uint2 *>(orow) = pack8(o);
 }
 
-// 12 output rows r0 .. r0+11 (r0 = R0 + 12 m, a multiple of 4); window and D
-// rows carried in/out by reference (the unrolled body renames registers).
-__device__ __forceinline__ void p2_body12(uint32_t aw, int s0, int lane, RowD &ra, RowD &rb, float4 &Dp, float4 &Dc,
-                                          int r0, int c0, int W, int H, uint32_t lut_q, uint8_t *orow, bool active) {
-#pragma unroll
-  for (int blk = 0; blk < 3; ++blk) {
-    const float4 Dn = dblock(aw, s0 + 4 * blk + 4, lane);  // D row k+1 (smem rows of block k+1)
-#pragma unroll
-    for (int a = 0; a < 4; ++a) {
-      const int r = r0 + 4 * blk + a;
-      const RowD rc = derive_w<true>(row_words(aw, s0 + 4 * blk + a + 1), lane);
-      const bool st = active && r < H;
-      uint8_t *op = orow + (size_t)(4 * blk + a) * W;
-      if (a == 0) p2_row<0>(ra, rb, rc, Dp, Dc, Dc, r, c0, W, H, lut_q, op, st);
-      if (a == 1) p2_row<1>(ra, rb, rc, Dp, Dc, Dc, r, c0, W, H, lut_q, op, st);
-      if (a == 2) p2_row<2>(ra, rb, rc, Dc, Dn, Dc, r, c0, W, H, lut_q, op, st);
-      if (a == 3) p2_row<3>(ra, rb, rc, Dc, Dn, Dc, r, c0, W, H, lut_q, op, st);
-      ra = rb;
-      rb = rc;
-    }
-    Dp = Dc;
-    Dc = Dn;
-  }
+__device__ __forceinline__ float4 f4fma(float a, const float4 &x, const float4 &y) {  // a*x + y, exact here
+  return make_float4(__fmaf_rn(a, x.x, y.x), __fmaf_rn(a, x.y, y.y), __fmaf_rn(a, x.z, y.z), __fmaf_rn(a, x.w, y.w));
+}
+__device__ __forceinline__ float4 f4add(const float4 &x, const float4 &y) {
+  return make_float4(__fadd_rn(x.x, y.x), __fadd_rn(x.y, y.y), __fadd_rn(x.z, y.z), __fadd_rn(x.w, y.w));
+}
+__device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y) {  // 2 (x - y), exact here
+  return make_float4(__fmul_rn(2.0f, __fsub_rn(x.x, y.x)), __fmul_rn(2.0f, __fsub_rn(x.y, y.y)),
+                     __fmul_rn(2.0f, __fsub_rn(x.z, y.z)), __fmul_rn(2.0f, __fsub_rn(x.w, y.w)));
 }
 
 __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__restrict__ out, int W, int H, int C0w,
@@ -356,28 +347,73 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
   const uint32_t aw = tile + (uint32_t)(kCol0 + 8 * (lane < 31 ? lane : -1));
-  const uint32_t lut_q = lut - (0x4B000000u << 3);  // LDS address of entry p from the bits of (2^23 + p)
-  // smem row of global row R0-4 is 0: row r -> r - R0 + 4.
-  float4 Dp = dblock(aw, 0, lane);  // D row k0-1
-  float4 Dc = dblock(aw, 4, lane);  // D row k0
+  // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (kept
+  // opaque so the compiler emits one IMAD instead of folding the constant).
+  uint32_t lut_q;
+  asm volatile("mov.u32 %0, %1;" : "=r"(lut_q) : "r"(lut - (0x4B000000u << 3)));
+  constexpr float s = -1.0f / 1024.0f;
+  const Wts wt{f2pack(3 * s, 1 * s), f2pack(5 * s, 7 * s), f2pack(7 * s, 5 * s), f2pack(1 * s, 3 * s)};
+  // smem row of global row R0-4 is 0: row r -> smem row r - R0 + 4.
+  // Vertical interpolation (L146, R3) of D rows (i, i+1) is linear in r on
+  // r = 4i+2 .. 4i+5: V(r+1) = V(r) + 2 (D_{i+1} - D_i), restarted at
+  // r = 4i+2 with V = 7 D_i + D_{i+1} (all exact integers, x 128).
+  const float4 Dp = dblock(aw, 0, lane);  // D row k0-1
+  float4 Dc = dblock(aw, 4, lane);        // D row k0 (= row r>>2)
+  float4 V = f4fma(5.0f, Dc, f4fma(3.0f, Dp, make_float4(0.f, 0.f, 0.f, 0.f)));  // r = R0 (a' = 0): (3,5)
+  float4 slope = f4twice_diff(Dc, Dp);
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
   uint8_t *orow = out + (size_t)R0 * W + c0;
-  p2_body12(aw, 4, lane, ra, rb, Dp, Dc, R0, c0, W, H, lut_q, orow, active);
-  if (R0 + 12 < H)
-    p2_body12(aw, 16, lane, ra, rb, Dp, Dc, R0 + 12, c0, W, H, lut_q, orow + (size_t)12 * W, active);
+  const int rend = min(R0 + kTH, H);
+#pragma unroll 1
+  for (int r = R0; r < rend; r += 3) {
+    // 3 rows per iteration: the window rotation has period 3, so the
+    // unrolled body needs no register moves.
+#pragma unroll
+    for (int u = 0; u < 3; ++u) {
+      const int rr = r + u;
+      const int sm = rr - R0 + 4;
+      if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
+        const float4 Dn = dblock(aw, sm + 2, lane);
+        V = f4fma(7.0f, Dc, Dn);
+        slope = f4twice_diff(Dn, Dc);
+        Dc = Dn;  // (D row k is no longer needed)
+      }
+      const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
+      p2_row(ra, rb, rc, V, wt, lut_q, orow, active && rr < rend);
+      V = f4add(V, slope);
+      orow += W;
+      ra = rb;
+      rb = rc;
+    }
+  }
 
-  // Specialised border pass: columns 0,1 and W-2,W-1 inside this tile.
+  // Specialised border pass: the 2-pixel ring inside this tile -- rows 0,1
+  // and H-2,H-1, columns 0,1 and W-2,W-1 -- recomputed with the scalar rules.
+  const bool top = (R0 == 0), bot = (R0 + kTH >= H - 2);
   const bool left = (C0w == 0), right = (C0w <= W - 2 && W - 2 < C0w + kTW);
-  if (left || right) {
+  if (top || bot || left || right) {
     __syncwarp();
-    const int nr = min(R0 + kTH, H) - R0;
-    const int ncol = (left ? 2 : 0) + (right ? 2 : 0);
-    for (int idx = lane; idx < nr * ncol; idx += 32) {
-      const int r = R0 + idx / ncol;
-      const int k = idx % ncol;  // left: columns 0,1; then W-2, W-1
-      const int c = left ? (k < 2 ? k : W - 4 + k) : W - 2 + k;
-      out[(size_t)r * W + c] = (uint8_t)pixel_generic(tile, lut, r, c, W, H, R0, C0w);
+    const int ncols = min(kTW, W - C0w);
+    if (top || bot) {
+      const int r0 = top ? 0 : H - 2;
+      const int nrow = (top && bot) ? 4 : 2;  // tiny images: both
+      for (int idx = lane; idx < nrow * ncols; idx += 32) {
+        const int q = idx / ncols;
+        const int r = (top && bot) ? (q < 2 ? q : H - 4 + q) : r0 + q;
+        if (r < R0 || r >= rend) continue;
+        const int c = C0w + idx % ncols;
+        out[(size_t)r * W + c] = (uint8_t)pixel_generic(tile, lut, r, c, W, H, R0, C0w);
+      }
+    }
+    if (left || right) {
+      const int ncol = (left ? 2 : 0) + (right ? 2 : 0);
+      for (int idx = lane; idx < (rend - R0) * ncol; idx += 32) {
+        const int r = R0 + idx / ncol;
+        const int k = idx % ncol;  // left: columns 0,1; then W-2, W-1
+        const int c = left ? (k < 2 ? k : W - 4 + k) : W - 2 + k;
+        out[(size_t)r * W + c] = (uint8_t)pixel_generic(tile, lut, r, c, W, H, R0, C0w);
+      }
     }
   }
 }
@@ -391,135 +427,135 @@ __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, i
 #pragma unroll
   for (int x = 0; x < 8; ++x) vmask |= (uint32_t)(c0 + x >= 1 && c0 + x <= W - 2) << x;
   if (lane >= 30) vmask = 0;
-  const bool edge = vmask != 0xffu;
   // smem row of global row R0-1 is 0: row r -> r - R0 + 1.
   RowD ra = derive_w<false>(row_words(aw, 0), lane);
   RowD rb = derive_w<false>(row_words(aw, 1), lane);
-  float acc = 0.0f;  // exact: < 8 px * 24 rows * 1530 < 2^24
+  // One accumulator per pixel column (exact: < 24 rows * 1530 < 2^24); the
+  // column mask is applied once at the end, so the row loop has no
+  // per-lane branches.
+  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 #pragma unroll 1
-  for (int m = 0; m < kTH; m += 12) {
+  for (int m = 0; m < kTH; m += 3) {
 #pragma unroll
-    for (int a = 0; a < 12; ++a) {
+    for (int a = 0; a < 3; ++a) {
       const int r = R0 + m + a;
       const RowD rc = derive_w<false>(row_words(aw, m + a + 2), lane);
       uint32_t pe[4];
       sobel(ra, rb, rc, pe);
-      if (r >= 1 && r < H - 1) {  // Sobel border rows are 0 (L160); rows >= H skipped
-        if (!edge) {
+      if ((unsigned)(r - 1) < (unsigned)(H - 2)) {  // Sobel frame rows are 0 (L160); rows >= H skipped
 #pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            acc = add_f32_f16(lo16(pe[i]), acc);
-            acc = add_f32_f16(hi16(pe[i]), acc);
-          }
-        } else {
-#pragma unroll
-          for (int x = 0; x < 8; ++x)
-            if (vmask >> x & 1) acc = add_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), acc);
-        }
+        for (int x = 0; x < 8; ++x)
+          acc[x] = add_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), acc[x]);
       }
       ra = rb;
       rb = rc;
     }
   }
-  return acc;
+  float sum = 0.0f;
+#pragma unroll
+  for (int x = 0; x < 8; ++x) sum = __fadd_rn(sum, (vmask >> x & 1) ? acc[x] : 0.0f);
+  return sum;
 }
 
-// Last-block-done (sec. V-C stage 2): the frame's mean and lookup tables,
-// adj(p) = A (p/m)^gamma and osc(p) = clamp(G exp(-p/(K m)), 0, 1) in f64,
-// rounded once to f32 (R9, R11), exactly the oracle's expressions.
-__device__ void build_lut(const StepParams &sp, int f) {
-  __threadfence();
-  const unsigned long long S = atomicAdd(&sp.sums1[f], 0ull);
-  const double mean = (double)S / ((double)sp.g.W * (double)sp.g.H);
-  const double m = mean > 1.0 ? mean : 1.0;
-  for (int p = threadIdx.x; p < kLutSize; p += blockDim.x) {
-    float adj = 0.0f, osc = 0.0f;
-    if (p <= 1530) {
-      adj = (float)((double)sp.prm.amount * pow((double)p / m, (double)sp.prm.gamma));
-      osc = (float)fmin(fmax((double)sp.prm.osc_gain * exp(-(double)p / ((double)sp.prm.osc_scale * m)), 0.0), 1.0);
-    }
-    sp.luts1[(size_t)f * kLutSize + p] = make_float2(adj, osc);
-  }
-  if (threadIdx.x == 0) {
-    sp.means1[f] = mean;
-    sp.counters1[f] = 0u;  // re-arm for the next launch
-  }
-}
-
-__global__ void __launch_bounds__(kThreadsT, 2)
+// ============================================================== the kernel
+__global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     step_kernel(const __grid_constant__ CUtensorMap map1, const __grid_constant__ CUtensorMap map2, StepParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ uint32_t warp_sum[kWarpsT];
-  __shared__ int next_task[2];
-  __shared__ int last_frame;
+  __shared__ int stage_task[2];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t sbase = smem_u32(smem);
-  const uint32_t bar0 = sbase + 2 * kStage;
-  const int ntasks = sp.n1 + sp.n2;
+  const uint32_t full0 = sbase + 2 * kStage, empty0 = full0 + 16;
+  const int t1 = sp.nL, t2 = sp.nL + sp.n1, ntasks = sp.nL + sp.n1 + sp.n2;
   const Geo &g = sp.g;
 
   if (threadIdx.x == 0) {
-    mbar_init(bar0, 1);
-    mbar_init(bar0 + 8, 1);
+    mbar_init(full0, 1);
+    mbar_init(full0 + 8, 1);
+    mbar_init(empty0, kWarpsT);
+    mbar_init(empty0 + 8, kWarpsT);
     fence_barrier_init();
   }
-  // Producer: grab the next task and start its loads into stage b.
-  auto issue = [&](int b) {
-    const int t = (int)atomicAdd(sp.task_counter, 1u);
-    next_task[b] = t;
-    if (t >= ntasks) return;
-    const bool p1 = t < sp.n1;
-    int f, C0, R0;
-    tile_of(g, p1 ? t : t - sp.n1, f, C0, R0);
-    int nw = 0;
-#pragma unroll
-    for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
-    const uint32_t bar = bar0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
-    fence_proxy_async();
-    if (p1) {
-      mbar_expect_tx(bar, (uint32_t)(nw * kBox1));
-      for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, &map1, C0 + w * kTW, R0 - 1, f, bar);
-    } else {
-      mbar_expect_tx(bar, (uint32_t)(nw * kBox2 + kLutBytes));
-      for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, &map2, C0 + w * kTW, R0 - 4, f, bar);
-      bulk_copy(st + kWarpsT * kSlot, sp.luts2 + (size_t)f * kLutSize, kLutBytes, bar);
-    }
-  };
-  if (threadIdx.x == 0) issue(0);
   __syncthreads();
 
+  if (warp == kWarpsT) {
+    // ------------------------------------------------------------ producer
+    if (lane != 0) return;
+    for (int i = 0;; ++i) {
+      const int b = i & 1;
+      if (i >= 2) mbar_wait(empty0 + 8u * b, (uint32_t)(((i >> 1) - 1) & 1));
+      const int t = (int)atomicAdd(sp.task_counter, 1u);
+      stage_task[b] = t;
+      const uint32_t full = full0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
+      if (t < t1 || t >= ntasks) {  // LUT task (no data) or the end marker
+        mbar_arrive(full);
+        if (t >= ntasks) break;
+        continue;
+      }
+      const bool p1 = t < t2;
+      int f, C0, R0;
+      tile_of(g, p1 ? t - t1 : t - t2, f, C0, R0);
+      int nw = 0;
+#pragma unroll
+      for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
+      if (p1) {
+        mbar_expect_tx(full, (uint32_t)(nw * kBox1));
+        for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, &map1, C0 + w * kTW, R0 - 1, f, full);
+      } else {
+        // the frame's LUT tasks (grabbed earlier) must have finished
+        while (ld_acquire(&sp.lut_done2[f]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(256);
+        fence_proxy_async_global();
+        mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
+        for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, &map2, C0 + w * kTW, R0 - 4, f, full);
+        bulk_copy(st + kWarpsT * kSlot, sp.luts2 + (size_t)f * kLutSize, kLutBytes, full);
+      }
+    }
+    return;
+  }
+
+  // -------------------------------------------------------------- consumers
   for (int i = 0;; ++i) {
     const int b = i & 1;
-    const int t = next_task[b];
+    mbar_wait(full0 + 8u * b, (uint32_t)((i >> 1) & 1));
+    const int t = stage_task[b];
     if (t >= ntasks) break;
-    if (threadIdx.x == 0) issue(b ^ 1);  // stage b^1 was released by the barrier ending iteration i-1
-    mbar_wait(bar0 + 8u * b, (uint32_t)((i >> 1) & 1));
     const uint32_t st = sbase + (uint32_t)(b * kStage);
-    const bool p1 = t < sp.n1;
-    int f, C0, R0;
-    tile_of(g, p1 ? t : t - sp.n1, f, C0, R0);
-    const int C0w = C0 + warp * kTW;
-    if (!p1) {
+    if (t < t1) {
+      // LUT task: entries q*128 .. q*128+127 of frame f (R9, R11; f64, one rounding)
+      const int f = t / kLutTasks, p = (t % kLutTasks) * kLutPerTask + threadIdx.x;
+      // L174: mean of pEdge over all W*H elements (R8), from the exact sum.
+      const double mean = (double)sp.sums2[f] / ((double)g.W * (double)g.H);
+      if (p == 0) sp.means2[f] = mean;
+      const double m = mean > 1.0 ? mean : 1.0;
+      float adj = 0.0f, osc = 0.0f;
+      if (p <= 1530) {
+        adj = (float)((double)sp.prm.amount * pow((double)p / m, (double)sp.prm.gamma));
+        osc = (float)fmin(fmax((double)sp.prm.osc_gain * exp(-(double)p / ((double)sp.prm.osc_scale * m)), 0.0), 1.0);
+      }
+      sp.luts2[(size_t)f * kLutSize + p] = make_float2(adj, osc);
+      __threadfence();
+      __syncwarp();
+      if (lane == 0) atomicAdd(&sp.lut_done2[f], 1u);
+    } else if (t < t2) {
+      int f, C0, R0;
+      tile_of(g, t - t1, f, C0, R0);
+      const int C0w = C0 + warp * kTW;
+      const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.H, C0w, R0, lane) : 0.0f;
+      // Reduction (sec. V-C): warp reduction, u64 atomic per warp; the last
+      // warp of the frame (last-block-done) computes the mean (L174).
+      // (the frame's mean is taken from the complete sum by its LUT tasks in
+      // the next launch: the kernel boundary is the global barrier, so no
+      // fence / last-block ticket is needed here)
+      const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
+      if (lane == 0 && ws) atomicAdd(&sp.sums1[f], (unsigned long long)ws);
+    } else {
+      int f, C0, R0;
+      tile_of(g, t - t2, f, C0, R0);
+      const int C0w = C0 + warp * kTW;
       if (C0w < g.W)
         p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out2 + (size_t)f * g.W * g.H, g.W, g.H, C0w, R0, lane);
-    } else {
-      const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.H, C0w, R0, lane) : 0.0f;
-      const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
-      if (lane == 0) warp_sum[warp] = ws;
-      __syncthreads();
-      if (threadIdx.x == 0) {
-        unsigned long long part = 0;
-#pragma unroll
-        for (int w = 0; w < kWarpsT; ++w) part += warp_sum[w];
-        atomicAdd(&sp.sums1[f], part);
-        __threadfence();
-        const unsigned int ticket = atomicAdd(&sp.counters1[f], 1u);
-        last_frame = (ticket == (unsigned)g.per_frame - 1) ? f : -1;
-      }
-      __syncthreads();
-      if (last_frame >= 0) build_lut(sp, last_frame);
     }
-    __syncthreads();  // stage b is free again
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty0 + 8u * b);  // stage b may be refilled
   }
 }
 
@@ -566,11 +602,6 @@ bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
          encode_fn() != nullptr;
 }
 
-int tma_tasks(int n, int W, int H) {
-  const int tx = (W + kCtaCols - 1) / kCtaCols, ty = (H + kTH - 1) / kTH;
-  return tx * ty * n;
-}
-
 cudaError_t launch_step_tma(const StepLaunch &a, int W, int H, const Params &p, cudaStream_t stream) {
   static bool attr = false;
   if (!attr) {
@@ -587,19 +618,20 @@ cudaError_t launch_step_tma(const StepLaunch &a, int W, int H, const Params &p, 
   sp.g.H = H;
   sp.g.tiles_x = (W + kCtaCols - 1) / kCtaCols;
   sp.g.per_frame = sp.g.tiles_x * ((H + kTH - 1) / kTH);
+  sp.nL = a.n2 * kLutTasks;
   sp.n1 = a.n1 * sp.g.per_frame;
   sp.n2 = a.n2 * sp.g.per_frame;
   sp.prm = p;
   sp.sums1 = a.sums1;
-  sp.means1 = a.means1;
-  sp.counters1 = a.counters1;
-  sp.luts1 = a.luts1;
+  sp.sums2 = a.sums2;
+  sp.means2 = a.means2;
   sp.luts2 = a.luts2;
+  sp.lut_done2 = a.lut_done2;
   sp.out2 = a.out2;
   sp.task_counter = a.task_counter;
-  const int tasks = sp.n1 + sp.n2;
+  const int tasks = sp.nL + sp.n1 + sp.n2;
   if (tasks == 0) return cudaSuccess;
-  const int grid = std::min(tasks, 2 * num_sms());
+  const int grid = std::min(tasks, kCtasPerSm * num_sms());
   step_kernel<<<grid, kThreadsT, kSmem, stream>>>(m1, m2, sp);
   return cudaGetLastError();
 }

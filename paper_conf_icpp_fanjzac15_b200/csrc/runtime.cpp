@@ -50,6 +50,7 @@ struct sharp_ctx {
   size_t frames_cap = 0;
   unsigned int *tcounters = nullptr;  // dynamic-scheduling task counters, one per step launch
   size_t tcounters_cap = 0;
+  unsigned int *lut_done = nullptr;   // per frame: finished LUT-task warps (step kernel)
   int last_frames = 0;
   sharp_stats stats{};
   // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2)
@@ -124,11 +125,14 @@ int ensure_frames(sharp_ctx *ctx, size_t n) {
   if (n <= ctx->frames_cap) return SHARP_OK;
   cudaFree(ctx->sums);
   cudaFree(ctx->means);
+  cudaFree(ctx->lut_done);
   ctx->sums = nullptr;
   ctx->means = nullptr;
+  ctx->lut_done = nullptr;
   ctx->frames_cap = 0;
   CK(cudaMalloc(&ctx->sums, n * sizeof(unsigned long long)));
   CK(cudaMalloc(&ctx->means, n * sizeof(double)));
+  CK(cudaMalloc(&ctx->lut_done, n * sizeof(unsigned int)));
   ctx->frames_cap = n;
   return SHARP_OK;
 }
@@ -255,15 +259,15 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
         a.in1 = din + f0 * fb;
         a.n1 = (int)std::min(chunk, (size_t)n - f0);
         a.sums1 = ctx->sums + frame_base + f0;
-        a.means1 = ctx->means + frame_base + f0;
-        a.counters1 = slot.counters;
-        a.luts1 = slot.luts + (c & 1) * chunk * sharp::kLutSize;
       }
       if (c > 0) {
         const size_t f0 = (c - 1) * chunk;
         a.in2 = din + f0 * fb;
         a.n2 = (int)std::min(chunk, (size_t)n - f0);
+        a.sums2 = ctx->sums + frame_base + f0;
+        a.means2 = ctx->means + frame_base + f0;
         a.luts2 = slot.luts + ((c - 1) & 1) * chunk * sharp::kLutSize;
+        a.lut_done2 = ctx->lut_done + frame_base + f0;
         a.out2 = dout + f0 * fb;
       }
       a.task_counter = tc + c;
@@ -312,6 +316,7 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   const size_t nchunks_all = ((size_t)n + chunk - 1) / chunk;
   if ((rc = ensure_task_counters(ctx, 2 * nchunks_all + 2))) return rc;
   CK(cudaMemsetAsync(ctx->sums, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
+  CK(cudaMemsetAsync(ctx->lut_done, 0, (size_t)n * sizeof(unsigned int), ctx->stream));
   CK(cudaMemsetAsync(ctx->tcounters, 0, (2 * nchunks_all + 2) * sizeof(unsigned int), ctx->stream));
   CK(cudaEventRecord(ctx->ev_start, ctx->stream));
   if (!staged) {
@@ -460,6 +465,7 @@ void sharp_destroy(sharp_ctx *ctx) {
   }
   cudaFree(ctx->sums);
   cudaFree(ctx->means);
+  cudaFree(ctx->lut_done);
   cudaFree(ctx->tcounters);
   for (auto &r : ctx->recs) {
     cudaEventDestroy(r.a);
