@@ -191,7 +191,10 @@ def main():
     h_out = torch.empty_like(h_in).pin_memory()
     d_in = h_in.to(f"cuda:{local}")
     d_out = torch.empty_like(d_in)
-    stream = torch.cuda.current_stream()
+    # A dedicated (non-default) stream: the library launches on it and the
+    # CUDA events below are recorded on it.
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
     sh = Sharpener(device=local)
     sh.set_stream(stream)
 

@@ -96,7 +96,8 @@ void sharp_default_params(sharp_params *p);
 
 /* Kernels are launched on `stream` (a cudaStream_t of the context's device,
  * e.g. torch.cuda.current_stream().cuda_stream); NULL restores the
- * context's own stream. */
+ * context's own (non-blocking) stream -- pass cudaStreamLegacy ((void *)1)
+ * for the legacy default stream. */
 int sharp_set_stream(sharp_ctx *ctx, void *stream);
 
 /* One image: img, out are w*h bytes.  params NULL -> defaults. */

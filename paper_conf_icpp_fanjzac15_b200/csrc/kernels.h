@@ -26,27 +26,23 @@ cudaError_t launch_edge_sum(const uint8_t *imgs, int n, int W, int H, const Para
 cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts,
                            uint8_t *outs, cudaStream_t stream);
 
-// TMA-staged, dynamically scheduled step kernel (kernels_tma.cu), used when
-// tma_supported() (W % 16 == 0, 16-byte aligned input, 8-byte aligned output).
-// One launch = LUT build (mean from the complete sums) + pass 2 of chunk "2"
-// (n2 frames, may be 0) and pass 1 of chunk "1" (n1 frames, may be 0).
-// Chunk 2's sums must be complete (an earlier launch's pass 1); chunk 1's
-// sums, lut_done2 and task_counter must be zero on entry.
-struct StepLaunch {
-  const uint8_t *in1 = nullptr;
-  int n1 = 0;
-  unsigned long long *sums1 = nullptr;
-  const uint8_t *in2 = nullptr;
-  int n2 = 0;
-  const unsigned long long *sums2 = nullptr;
-  double *means2 = nullptr;
-  float2 *luts2 = nullptr;
-  unsigned int *lut_done2 = nullptr;
-  uint8_t *out2 = nullptr;
-  unsigned int *task_counter = nullptr;
+// TMA-staged, persistent, dynamically scheduled kernel (kernels_tma.cu) for a
+// whole batch in ONE launch (pass 1, per-frame LUT build and pass 2 as tasks
+// with in-kernel dependencies), used when tma_supported() (W % 16 == 0,
+// W*H <= 2^29, 16-byte aligned input, 8-byte aligned output).
+struct BatchLaunch {
+  const uint8_t *in = nullptr;  // [n][H][W]
+  int n = 0;
+  uint8_t *out = nullptr;       // [n][H][W]
+  unsigned long long *acc = nullptr;   // n; zero on entry
+  unsigned long long *sums = nullptr;  // n; out: S per frame
+  double *means = nullptr;             // n; out: S / (W H)
+  float2 *luts = nullptr;              // n * kLutSize (scratch)
+  unsigned int *lut_done = nullptr;    // n; zero on entry
+  unsigned int *task_counter = nullptr;  // 1; zero on entry
 };
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);
-cudaError_t launch_step_tma(const StepLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
+cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
 
 // Kernel launches issued per (pass-1, pass-2) chunk.
 constexpr int kLaunchesPerChunk = 2;

@@ -54,17 +54,21 @@ constexpr int kCtaCols = kTW * kWarpsT;
 constexpr int kThreadsT = 32 * (kWarpsT + 1);  // + producer warp
 constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task
 constexpr int kLutTasks = kLutSize / kLutPerTask;
-// The TMA box's innermost start coordinate must be 16-byte aligned and a box
-// dimension is at most 256, so frames are viewed as 4-D [n][H][W/16][16] and
-// a warp tile's box is {16, 17 chunks, rows, 1}: 272 columns from C0w-16.
-constexpr int kChunks = 17;
-constexpr int kPitch = 16 * kChunks;  // smem row pitch: columns C0w-16 .. C0w+255
-constexpr int kCol0 = 16;             // smem column of C0w
+// A warp tile needs columns C0w-8 .. C0w+247.  TMA box starts must be
+// 16-byte aligned in the innermost dimension and a box dimension is at most
+// 256, so each warp tile is fetched as two boxes of the [n][H][W] frames:
+//   region A: 256 columns C0w-16 .. C0w+239  (smem pitch 256)
+//   region B:  16 columns C0w+240 .. C0w+255 (smem pitch 16; only lane 30,
+//             the right halo, reads it)
+constexpr int kPitch = 256;           // region A pitch
+constexpr int kPitchB = 16;           // region B pitch
+constexpr int kCol0 = 16;             // region-A column of C0w
 constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+kTH+3
 constexpr int kRows1 = kTH + 2;       // pass-1 box rows: R0-1 .. R0+kTH
-constexpr int kBox2 = kPitch * kRows2;
-constexpr int kBox1 = kPitch * kRows1;
+constexpr int kBox2 = (kPitch + kPitchB) * kRows2;
+constexpr int kBox1 = (kPitch + kPitchB) * kRows1;
 constexpr int kSlot = (kBox2 + 127) / 128 * 128;  // per-warp smem slot (128-B aligned)
+static_assert((kPitch * kRows1) % 128 == 0 && (kPitch * kRows2) % 128 == 0, "region B alignment");
 constexpr int kLutBytes = kLutSize * 8;
 constexpr int kStage = kWarpsT * kSlot + kLutBytes;
 constexpr int kSmem = 2 * kStage + 64;
@@ -93,15 +97,19 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
-// Box of the warp tile whose first output column is C0w (a multiple of 16):
-// columns C0w-16 .. C0w+255, rows r .. r+rows-1 of frame f.
-__device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, int C0w, int r, int f, uint32_t bar) {
-  const int chunk = (C0w - kCol0) / 16;
+// One 3-D box {cols, rows, 1} of the [n][H][W] frames at (x, r, f) (x 16-B aligned).
+__device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, int x, int r, int f, uint32_t bar) {
   asm volatile(
-      "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], "
-      "[%6];" ::"r"(dst),
-      "l"(map), "r"(0), "r"(chunk), "r"(r), "r"(f), "r"(bar)
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+      "[%5];" ::"r"(dst),
+      "l"(map), "r"(x), "r"(r), "r"(f), "r"(bar)
       : "memory");
+}
+// Both boxes of a warp tile (region A then region B at dst + kPitch*rows).
+__device__ __forceinline__ void tma_tile(uint32_t dst, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0w,
+                                         int r, int rows, int f, uint32_t bar) {
+  tma_box(dst, mapA, C0w - kCol0, r, f, bar);
+  tma_box(dst + (uint32_t)(kPitch * rows), mapB, C0w + 256 - kCol0, r, f, bar);
 }
 __device__ __forceinline__ void bulk_copy(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
@@ -161,25 +169,78 @@ __device__ __forceinline__ void tile_of(const Geo &g, int t, int &f, int &C0, in
   R0 = ty * kTH;
 }
 
+// The task sequence is a list of rounds; round rho holds
+//   [pass-1 tasks of frame rho][LUT tasks of frame rho-L1][pass-2 tasks of frame rho-L2]
+// (slots for frames outside [0, n) are empty tasks).  The lags L1 < L2 are
+// chosen so that a frame's dependencies were grabbed long before (they are
+// normally complete when the producer checks them).
+enum TaskType { kEmpty = 0, kP1 = 1, kLut = 2, kP2 = 3, kEnd = -1 };
 struct StepParams {
   Geo g;
-  int nL, n1, n2;  // LUT / pass-1 / pass-2 task counts (in this order)
+  int n;          // frames
+  int L1, L2;     // round lags of the LUT and pass-2 tasks
+  int per_round;  // 2 * per_frame + kLutTasks
+  int ntasks;     // (n + L2) * per_round
   Params prm;
-  // pass 1 (chunk c)
-  unsigned long long *sums1;
-  // LUT + pass 2 (chunk c-1)
-  const unsigned long long *sums2;
-  double *means2;
-  float2 *luts2;
-  unsigned int *lut_done2;
-  uint8_t *out2;
-  unsigned int *task_counter;
+  unsigned long long *acc;  // per frame: (pass-1 warp arrivals << 40) + sum of pEdge; zero on entry
+  unsigned long long *sums; // per frame: S (written by the frame's first LUT task)
+  double *means;            // per frame: S / (W H)
+  float2 *luts;             // per frame: kLutSize entries {adj, osc}
+  unsigned int *lut_done;   // per frame: finished LUT-task warps; zero on entry
+  uint8_t *out;
+  unsigned int *task_counter;  // zero on entry
 };
+// acc packing: S <= 1530 * W * H < 2^40 for W * H <= 2^29 (tma_supported),
+// and the arrival count (4 per task) stays far below 2^24.
+constexpr int kAccShift = 40;
+__device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type, frame, sub, 0}
+  if (t >= sp.ntasks) return make_int4(kEnd, 0, 0, 0);
+  const int rho = t / sp.per_round, k = t - rho * sp.per_round;
+  const int pf = sp.g.per_frame;
+  if (k < pf) return rho < sp.n ? make_int4(kP1, rho, k, 0) : make_int4(kEmpty, 0, 0, 0);
+  if (k < pf + kLutTasks) {
+    const int f = rho - sp.L1;
+    return (f >= 0 && f < sp.n) ? make_int4(kLut, f, k - pf, 0) : make_int4(kEmpty, 0, 0, 0);
+  }
+  const int f = rho - sp.L2;
+  return (f >= 0 && f < sp.n) ? make_int4(kP2, f, k - pf - kLutTasks, 0) : make_int4(kEmpty, 0, 0, 0);
+}
+__device__ __forceinline__ void tile_xy(const Geo &g, int sub, int &C0, int &R0) {
+  const int ty = sub / g.tiles_x;
+  C0 = (sub - ty * g.tiles_x) * kCtaCols;
+  R0 = ty * kTH;
+}
+// Polling loads: relaxed (no L1 invalidation per poll); the caller issues
+// one acquire fence after the awaited value was seen.
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned int ld_relaxed_u32(const unsigned int *p) {
+  unsigned int v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void fence_acquire() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 // ------------------------------------------------------------- row window
-// Lane words of smem row s: lanes 0..29 own columns C0w+8l..+7; lane 30 the
-// right halo C0w+240..247, lane 31 the left halo C0w-8..C0w-1.
-__device__ __forceinline__ uint2 row_words(uint32_t a, int s) { return lds_u64(a + (uint32_t)s * kPitch); }
+// Lane words of smem row s: lanes 0..29 own columns C0w+8l..+7 (region A);
+// lane 31 the left halo C0w-8..C0w-1 (region A); lane 30 the right halo
+// C0w+240..247 (region B, pitch 16).
+struct LaneRow {
+  uint32_t base, pitch;
+};
+__device__ __forceinline__ LaneRow lane_row(uint32_t tile, int rows, int lane) {
+  if (lane == 30) return LaneRow{tile + (uint32_t)(kPitch * rows), (uint32_t)kPitchB};
+  return LaneRow{tile + (uint32_t)(kCol0 + 8 * (lane < 31 ? lane : -1)), (uint32_t)kPitch};
+}
+__device__ __forceinline__ uint2 row_words(const LaneRow &a, int s) { return lds_u64(a.base + (uint32_t)s * a.pitch); }
+// smem address of (tile row s, column C0w - kCol0 + rel), either region.
+__device__ __forceinline__ uint32_t tile_addr(uint32_t tile, int rows, int s, int rel) {
+  return rel < kPitch ? tile + (uint32_t)(s * kPitch + rel)
+                      : tile + (uint32_t)(kPitch * rows + s * kPitchB + (rel - kPitch));
+}
 
 // Converts a row of words into the window data.  Neighbour pairs come from
 // the adjacent lanes (shuffle), so each lane loads only its own 8 bytes.
@@ -209,9 +270,9 @@ __device__ __forceinline__ RowD derive_w(uint2 w, int lane) {
 }
 
 // D sums (16*D) of the block at smem rows s..s+3 for D columns j0-1..j0+2.
-__device__ __forceinline__ float4 dblock(uint32_t a, int s, int lane) {
-  const uint32_t o = a + (uint32_t)s * kPitch;
-  const uint2 r0 = lds_u64(o), r1 = lds_u64(o + kPitch), r2 = lds_u64(o + 2 * kPitch), r3 = lds_u64(o + 3 * kPitch);
+__device__ __forceinline__ float4 dblock(const LaneRow &a, int s, int lane) {
+  const uint32_t o = a.base + (uint32_t)s * a.pitch;
+  const uint2 r0 = lds_u64(o), r1 = lds_u64(o + a.pitch), r2 = lds_u64(o + 2 * a.pitch), r3 = lds_u64(o + 3 * a.pitch);
   const float d0 = (float)blk4(r0.x, r1.x, r2.x, r3.x);
   const float d1 = (float)blk4(r0.y, r1.y, r2.y, r3.y);
   const float dm1 = __shfl_sync(0xffffffffu, d1, (lane + 31) & 31);
@@ -220,9 +281,11 @@ __device__ __forceinline__ float4 dblock(uint32_t a, int s, int lane) {
 }
 
 // ------------------------------------------------------- scalar border pixel
+// (pass-2 tiles: kRows2 rows, smem row 0 = global row R0-4)
 __device__ __forceinline__ float dsum_at(uint32_t tile, int i, int j, int R0, int C0w) {
-  const uint32_t a = tile + (uint32_t)(4 * i - R0 + 4) * kPitch + (uint32_t)(4 * j - C0w + kCol0);
-  return (float)blk4(lds_u32(a), lds_u32(a + kPitch), lds_u32(a + 2 * kPitch), lds_u32(a + 3 * kPitch));
+  const int s = 4 * i - R0 + 4, rel = 4 * j - C0w + kCol0;
+  return (float)blk4(lds_u32(tile_addr(tile, kRows2, s, rel)), lds_u32(tile_addr(tile, kRows2, s + 1, rel)),
+                     lds_u32(tile_addr(tile, kRows2, s + 2, rel)), lds_u32(tile_addr(tile, kRows2, s + 3, rel)));
 }
 
 // U at (r, c), any pixel: body formula of L146 or the border rules of
@@ -256,15 +319,15 @@ __device__ float u_any(uint32_t tile, int r, int c, int W, int H, int R0, int C0
 
 // The whole pipeline for one pixel with scalar code (specialised border pass).
 __device__ uint32_t pixel_generic(uint32_t tile, uint32_t lut, int r, int c, int W, int H, int R0, int C0w) {
-  const uint32_t base = tile + (uint32_t)(r - R0 + 4) * kPitch + (uint32_t)(c - C0w + kCol0);
-  const int o = (int)lds_u8(base);
+  const int s0 = r - R0 + 4, rel0 = c - C0w + kCol0;
+  const int o = (int)lds_u8(tile_addr(tile, kRows2, s0, rel0));
   int pe = 0, mx = 255, mn = 0;
   if (!(r == 0 || r == H - 1 || c == 0 || c == W - 1)) {  // Sobel frame (L160) / overshoot frame (L208)
     int v[3][3];
 #pragma unroll
     for (int u = 0; u < 3; ++u)
 #pragma unroll
-      for (int q = 0; q < 3; ++q) v[u][q] = (int)lds_u8(base + (uint32_t)((u - 1) * kPitch + (q - 1)));
+      for (int q = 0; q < 3; ++q) v[u][q] = (int)lds_u8(tile_addr(tile, kRows2, s0 + u - 1, rel0 + q - 1));
     const int gx = (v[0][2] + 2 * v[1][2] + v[2][2]) - (v[0][0] + 2 * v[1][0] + v[2][0]);
     const int gy = (v[2][0] + 2 * v[2][1] + v[2][2]) - (v[0][0] + 2 * v[0][1] + v[0][2]);
     pe = abs(gx) + abs(gy);
@@ -346,7 +409,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
                                         int R0, int lane) {
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
-  const uint32_t aw = tile + (uint32_t)(kCol0 + 8 * (lane < 31 ? lane : -1));
+  const LaneRow aw = lane_row(tile, kRows2, lane);
   // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (kept
   // opaque so the compiler emits one IMAD instead of folding the constant).
   uint32_t lut_q;
@@ -421,7 +484,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
 // ========================================================== pass 1 (warp)
 __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, int R0, int lane) {
   const int c0 = C0w + 8 * lane;
-  const uint32_t aw = tile + (uint32_t)(kCol0 + 8 * (lane < 31 ? lane : -1));
+  const LaneRow aw = lane_row(tile, kRows1, lane);
   // Sobel-body pixels of this lane (not frame columns, not beyond the image).
   uint32_t vmask = 0;
 #pragma unroll
@@ -459,13 +522,14 @@ __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, i
 
 // ============================================================== the kernel
 __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
-    step_kernel(const __grid_constant__ CUtensorMap map1, const __grid_constant__ CUtensorMap map2, StepParams sp) {
+    step_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
+                const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, StepParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ int stage_task[2];
+  __shared__ int4 stage_task[2];                 // {type, frame, sub, 0}
+  __shared__ unsigned long long stage_sum[2];    // LUT tasks: the frame's S
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t sbase = smem_u32(smem);
   const uint32_t full0 = sbase + 2 * kStage, empty0 = full0 + 16;
-  const int t1 = sp.nL, t2 = sp.nL + sp.n1, ntasks = sp.nL + sp.n1 + sp.n2;
   const Geo &g = sp.g;
 
   if (threadIdx.x == 0) {
@@ -480,33 +544,41 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
   if (warp == kWarpsT) {
     // ------------------------------------------------------------ producer
     if (lane != 0) return;
+    const unsigned long long arrivals = (unsigned long long)(g.per_frame * kWarpsT) << kAccShift;
     for (int i = 0;; ++i) {
       const int b = i & 1;
       if (i >= 2) mbar_wait(empty0 + 8u * b, (uint32_t)(((i >> 1) - 1) & 1));
-      const int t = (int)atomicAdd(sp.task_counter, 1u);
-      stage_task[b] = t;
+      const int4 d = decode(sp, (int)atomicAdd(sp.task_counter, 1u));
+      stage_task[b] = d;
       const uint32_t full = full0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
-      if (t < t1 || t >= ntasks) {  // LUT task (no data) or the end marker
-        mbar_arrive(full);
-        if (t >= ntasks) break;
-        continue;
-      }
-      const bool p1 = t < t2;
-      int f, C0, R0;
-      tile_of(g, p1 ? t - t1 : t - t2, f, C0, R0);
-      int nw = 0;
+      if (d.x == kP1 || d.x == kP2) {
+        int C0, R0;
+        tile_xy(g, d.z, C0, R0);
+        int nw = 0;
 #pragma unroll
-      for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
-      if (p1) {
-        mbar_expect_tx(full, (uint32_t)(nw * kBox1));
-        for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, &map1, C0 + w * kTW, R0 - 1, f, full);
+        for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
+        if (d.x == kP1) {
+          mbar_expect_tx(full, (uint32_t)(nw * kBox1));
+          for (int w = 0; w < nw; ++w) tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1, kRows1, d.y, full);
+        } else {
+          // dependency: the frame's LUT tasks (grabbed earlier) have finished
+          while (ld_relaxed_u32(&sp.lut_done[d.y]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(500);
+          fence_acquire();
+          fence_proxy_async_global();
+          mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
+          for (int w = 0; w < nw; ++w) tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4, kRows2, d.y, full);
+          bulk_copy(st + kWarpsT * kSlot, sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
+        }
       } else {
-        // the frame's LUT tasks (grabbed earlier) must have finished
-        while (ld_acquire(&sp.lut_done2[f]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(256);
-        fence_proxy_async_global();
-        mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
-        for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, &map2, C0 + w * kTW, R0 - 4, f, full);
-        bulk_copy(st + kWarpsT * kSlot, sp.luts2 + (size_t)f * kLutSize, kLutBytes, full);
+        if (d.x == kLut) {
+          // dependency: every pass-1 warp of the frame has added its partial
+          // (the global barrier of L174's reduction)
+          unsigned long long a;
+          while (((a = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(500);
+          stage_sum[b] = a & ((1ull << kAccShift) - 1);
+        }
+        mbar_arrive(full);  // no data: LUT, empty or end task
+        if (d.x == kEnd) break;
       }
     }
     return;
@@ -516,43 +588,46 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
   for (int i = 0;; ++i) {
     const int b = i & 1;
     mbar_wait(full0 + 8u * b, (uint32_t)((i >> 1) & 1));
-    const int t = stage_task[b];
-    if (t >= ntasks) break;
+    const int4 d = stage_task[b];
+    if (d.x == kEnd) break;
     const uint32_t st = sbase + (uint32_t)(b * kStage);
-    if (t < t1) {
+    if (d.x == kLut) {
       // LUT task: entries q*128 .. q*128+127 of frame f (R9, R11; f64, one rounding)
-      const int f = t / kLutTasks, p = (t % kLutTasks) * kLutPerTask + threadIdx.x;
+      const int f = d.y, p = d.z * kLutPerTask + threadIdx.x;
       // L174: mean of pEdge over all W*H elements (R8), from the exact sum.
-      const double mean = (double)sp.sums2[f] / ((double)g.W * (double)g.H);
-      if (p == 0) sp.means2[f] = mean;
+      const unsigned long long S = stage_sum[b];
+      const double mean = (double)S / ((double)g.W * (double)g.H);
+      if (p == 0) {
+        sp.sums[f] = S;
+        sp.means[f] = mean;
+      }
       const double m = mean > 1.0 ? mean : 1.0;
       float adj = 0.0f, osc = 0.0f;
       if (p <= 1530) {
         adj = (float)((double)sp.prm.amount * pow((double)p / m, (double)sp.prm.gamma));
         osc = (float)fmin(fmax((double)sp.prm.osc_gain * exp(-(double)p / ((double)sp.prm.osc_scale * m)), 0.0), 1.0);
       }
-      sp.luts2[(size_t)f * kLutSize + p] = make_float2(adj, osc);
+      sp.luts[(size_t)f * kLutSize + p] = make_float2(adj, osc);
       __threadfence();
       __syncwarp();
-      if (lane == 0) atomicAdd(&sp.lut_done2[f], 1u);
-    } else if (t < t2) {
-      int f, C0, R0;
-      tile_of(g, t - t1, f, C0, R0);
+      if (lane == 0) atomicAdd(&sp.lut_done[f], 1u);
+    } else if (d.x == kP1) {
+      int C0, R0;
+      tile_xy(g, d.z, C0, R0);
       const int C0w = C0 + warp * kTW;
       const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.H, C0w, R0, lane) : 0.0f;
-      // Reduction (sec. V-C): warp reduction, u64 atomic per warp; the last
-      // warp of the frame (last-block-done) computes the mean (L174).
-      // (the frame's mean is taken from the complete sum by its LUT tasks in
-      // the next launch: the kernel boundary is the global barrier, so no
-      // fence / last-block ticket is needed here)
+      // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
+      // atomic per warp adding (1 << 40) + partial: the frame's arrival count
+      // and sum in one word, so its LUT tasks can tell when S is complete
+      // without any fence.
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
-      if (lane == 0 && ws) atomicAdd(&sp.sums1[f], (unsigned long long)ws);
-    } else {
-      int f, C0, R0;
-      tile_of(g, t - t2, f, C0, R0);
+      if (lane == 0) atomicAdd(&sp.acc[d.y], (1ull << kAccShift) + (unsigned long long)ws);
+    } else if (d.x == kP2) {
+      int C0, R0;
+      tile_xy(g, d.z, C0, R0);
       const int C0w = C0 + warp * kTW;
       if (C0w < g.W)
-        p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out2 + (size_t)f * g.W * g.H, g.W, g.H, C0w, R0, lane);
+        p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H, C0w, R0, lane);
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(empty0 + 8u * b);  // stage b may be refilled
@@ -572,14 +647,14 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, int box_rows) {
+bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, int box_cols, int box_rows) {
   auto fn = encode_fn();
   if (!fn) return false;
-  const cuuint64_t dims[4] = {16, (cuuint64_t)W / 16, (cuuint64_t)H, (cuuint64_t)n};  // [n][H][W/16][16]
-  const cuuint64_t strides[3] = {16, (cuuint64_t)W, (cuuint64_t)W * H};
-  const cuuint32_t box[4] = {16, (cuuint32_t)kChunks, (cuuint32_t)box_rows, 1};
-  const cuuint32_t estr[4] = {1, 1, 1, 1};
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, (void *)imgs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+  const cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)n};  // [n][H][W]
+  const cuuint64_t strides[2] = {(cuuint64_t)W, (cuuint64_t)W * H};
+  const cuuint32_t box[3] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows, 1};
+  const cuuint32_t estr[3] = {1, 1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, (void *)imgs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
@@ -599,40 +674,46 @@ int num_sms() {
 
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
   return (W % 16) == 0 && (((uintptr_t)imgs) & 15) == 0 && (((uintptr_t)outs) & 7) == 0 && H >= 8 &&
-         encode_fn() != nullptr;
+         (size_t)W * H <= (1u << 29) && encode_fn() != nullptr;
 }
 
-cudaError_t launch_step_tma(const StepLaunch &a, int W, int H, const Params &p, cudaStream_t stream) {
+cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream) {
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
     attr = true;
   }
-  CUtensorMap m1, m2;
-  memset(&m1, 0, sizeof(m1));
-  memset(&m2, 0, sizeof(m2));
-  if (a.n1 > 0 && !make_map(&m1, a.in1, a.n1, W, H, kRows1)) return cudaErrorInvalidValue;
-  if (a.n2 > 0 && !make_map(&m2, a.in2, a.n2, W, H, kRows2)) return cudaErrorInvalidValue;
+  if (a.n <= 0) return cudaSuccess;
+  CUtensorMap m1A, m1B, m2A, m2B;  // the same frames: pass-1 / pass-2 box heights, regions A / B
+  if (!make_map(&m1A, a.in, a.n, W, H, kPitch, kRows1) || !make_map(&m1B, a.in, a.n, W, H, kPitchB, kRows1) ||
+      !make_map(&m2A, a.in, a.n, W, H, kPitch, kRows2) || !make_map(&m2B, a.in, a.n, W, H, kPitchB, kRows2))
+    return cudaErrorInvalidValue;
   StepParams sp;
   sp.g.W = W;
   sp.g.H = H;
   sp.g.tiles_x = (W + kCtaCols - 1) / kCtaCols;
   sp.g.per_frame = sp.g.tiles_x * ((H + kTH - 1) / kTH);
-  sp.nL = a.n2 * kLutTasks;
-  sp.n1 = a.n1 * sp.g.per_frame;
-  sp.n2 = a.n2 * sp.g.per_frame;
+  sp.n = a.n;
+  sp.per_round = 2 * sp.g.per_frame + kLutTasks;
+  const int grid = kCtasPerSm * num_sms();
+  // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
+  // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
+  // one more round separates those from its pass-2 tasks.
+  const int in_flight = 3 * grid;
+  sp.L1 = (in_flight + sp.per_round - 1) / sp.per_round + 1;
+  // LUT tasks take a few microseconds (f64 pow/exp): leave >= ~2 grid's worth
+  // of grabs before the frame's pass-2 tasks.
+  sp.L2 = sp.L1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
+  sp.ntasks = (a.n + sp.L2) * sp.per_round;
   sp.prm = p;
-  sp.sums1 = a.sums1;
-  sp.sums2 = a.sums2;
-  sp.means2 = a.means2;
-  sp.luts2 = a.luts2;
-  sp.lut_done2 = a.lut_done2;
-  sp.out2 = a.out2;
+  sp.acc = a.acc;
+  sp.sums = a.sums;
+  sp.means = a.means;
+  sp.luts = a.luts;
+  sp.lut_done = a.lut_done;
+  sp.out = a.out;
   sp.task_counter = a.task_counter;
-  const int tasks = sp.nL + sp.n1 + sp.n2;
-  if (tasks == 0) return cudaSuccess;
-  const int grid = std::min(tasks, kCtasPerSm * num_sms());
-  step_kernel<<<grid, kThreadsT, kSmem, stream>>>(m1, m2, sp);
+  step_kernel<<<grid, kThreadsT, kSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
   return cudaGetLastError();
 }
 

@@ -50,7 +50,9 @@ struct sharp_ctx {
   size_t frames_cap = 0;
   unsigned int *tcounters = nullptr;  // dynamic-scheduling task counters, one per step launch
   size_t tcounters_cap = 0;
-  unsigned int *lut_done = nullptr;   // per frame: finished LUT-task warps (step kernel)
+  unsigned int *lut_done = nullptr;   // per frame: finished LUT-task warps (batch kernel)
+  unsigned long long *acc = nullptr;  // per frame: pass-1 arrivals << 40 | partial sum (batch kernel)
+  float2 *luts = nullptr;             // per frame lookup tables (batch kernel)
   int last_frames = 0;
   sharp_stats stats{};
   // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2)
@@ -123,16 +125,24 @@ int classify(sharp_ctx *ctx, const void *p, Kind *k) {
 
 int ensure_frames(sharp_ctx *ctx, size_t n) {
   if (n <= ctx->frames_cap) return SHARP_OK;
+  CK(cudaStreamSynchronize(ctx->stream));
+  for (int i = 0; i < ctx->nslots; ++i) CK(cudaStreamSynchronize(ctx->slots[i].stream));
   cudaFree(ctx->sums);
   cudaFree(ctx->means);
   cudaFree(ctx->lut_done);
+  cudaFree(ctx->acc);
+  cudaFree(ctx->luts);
   ctx->sums = nullptr;
   ctx->means = nullptr;
   ctx->lut_done = nullptr;
+  ctx->acc = nullptr;
+  ctx->luts = nullptr;
   ctx->frames_cap = 0;
   CK(cudaMalloc(&ctx->sums, n * sizeof(unsigned long long)));
   CK(cudaMalloc(&ctx->means, n * sizeof(double)));
   CK(cudaMalloc(&ctx->lut_done, n * sizeof(unsigned int)));
+  CK(cudaMalloc(&ctx->acc, n * sizeof(unsigned long long)));
+  CK(cudaMalloc(&ctx->luts, n * sharp::kLutSize * sizeof(float2)));
   ctx->frames_cap = n;
   return SHARP_OK;
 }
@@ -251,31 +261,22 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   const size_t fb = (size_t)w * h;
   const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
   const bool tma = ctx->use_tma && sharp::tma_supported(din, dout, w, h);
-  if (tma) {
-    for (size_t c = 0; c <= nchunks; ++c) {
-      sharp::StepLaunch a;
-      if (c < nchunks) {
-        const size_t f0 = c * chunk;
-        a.in1 = din + f0 * fb;
-        a.n1 = (int)std::min(chunk, (size_t)n - f0);
-        a.sums1 = ctx->sums + frame_base + f0;
-      }
-      if (c > 0) {
-        const size_t f0 = (c - 1) * chunk;
-        a.in2 = din + f0 * fb;
-        a.n2 = (int)std::min(chunk, (size_t)n - f0);
-        a.sums2 = ctx->sums + frame_base + f0;
-        a.means2 = ctx->means + frame_base + f0;
-        a.luts2 = slot.luts + ((c - 1) & 1) * chunk * sharp::kLutSize;
-        a.lut_done2 = ctx->lut_done + frame_base + f0;
-        a.out2 = dout + f0 * fb;
-      }
-      a.task_counter = tc + c;
-      CK(timed(ctx, st, 3, (double)a.n2 * fb, [&] { return sharp::launch_step_tma(a, w, h, prm, st); }));
-      *launches += 1;
-    }
+  if (tma) {  // the whole batch in one persistent launch
+    sharp::BatchLaunch a;
+    a.in = din;
+    a.n = n;
+    a.out = dout;
+    a.acc = ctx->acc + frame_base;
+    a.sums = ctx->sums + frame_base;
+    a.means = ctx->means + frame_base;
+    a.luts = ctx->luts + frame_base * sharp::kLutSize;
+    a.lut_done = ctx->lut_done + frame_base;
+    a.task_counter = tc;
+    CK(timed(ctx, st, 3, (double)n * fb, [&] { return sharp::launch_batch_tma(a, w, h, prm, st); }));
+    *launches += 1;
     return SHARP_OK;
   }
+  (void)nchunks;
   for (size_t f0 = 0; f0 < (size_t)n; f0 += chunk) {
     const int cn = (int)std::min(chunk, (size_t)n - f0);
     const double px = (double)cn * fb;
@@ -317,6 +318,7 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   if ((rc = ensure_task_counters(ctx, 2 * nchunks_all + 2))) return rc;
   CK(cudaMemsetAsync(ctx->sums, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
   CK(cudaMemsetAsync(ctx->lut_done, 0, (size_t)n * sizeof(unsigned int), ctx->stream));
+  CK(cudaMemsetAsync(ctx->acc, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
   CK(cudaMemsetAsync(ctx->tcounters, 0, (2 * nchunks_all + 2) * sizeof(unsigned int), ctx->stream));
   CK(cudaEventRecord(ctx->ev_start, ctx->stream));
   if (!staged) {
@@ -466,6 +468,8 @@ void sharp_destroy(sharp_ctx *ctx) {
   cudaFree(ctx->sums);
   cudaFree(ctx->means);
   cudaFree(ctx->lut_done);
+  cudaFree(ctx->acc);
+  cudaFree(ctx->luts);
   cudaFree(ctx->tcounters);
   for (auto &r : ctx->recs) {
     cudaEventDestroy(r.a);

@@ -114,6 +114,23 @@ def test_batch_frames_independent_and_equal_to_oracle(sh):
     assert sums == [int(s) for s in ref_sums]
 
 
+@pytest.mark.parametrize("n,W,H", [(1, 16, 8), (3, 16, 16), (40, 256, 40), (9, 976, 44), (2, 3840, 2160)])
+def test_batch_single_launch_dependencies(n, W, H):
+    """TMA batch kernel: pass 1 -> LUT -> pass 2 dependencies resolved inside
+    one launch (rounds with lags; empty tasks at the ends)."""
+    imgs = synth.frames(n, W, H, "natural", seed=n * 7 + W)
+    with Sharpener() as s:
+        d = torch.from_numpy(imgs).cuda()
+        o = torch.empty_like(d)
+        s.run_batch(d, DEFAULT, o)
+        sums = s.batch_sums(n)
+        st = s.stats()
+    ref, ref_sums = oracle.sharpen_batch(imgs, *DEFAULT)
+    np.testing.assert_array_equal(o.cpu().numpy(), ref)
+    assert sums == [int(x) for x in ref_sums]
+    assert st.edge_sum == int(ref_sums[0])
+
+
 def test_batch_chunking_many_chunks():
     # chunk_frames=3 forces several pass-1/pass-2 chunk pairs on one stream
     imgs = synth.frames(10, 128, 64, "natural", seed=9)
