@@ -17,7 +17,7 @@ SYNTH_CFLAGS  := -std=c11 -O2 -fopenmp -fPIC -shared -Wall -Wextra
 # --fmad=false: no implicit FMA contraction; every fused multiply-add in the
 # kernels is an explicit __fmaf_rn / fma.rn (bit-exact parity, R15).
 NVCC_FLAGS := $(ARCH) -O3 -lineinfo -std=c++17 --fmad=false -Xptxas -v \
-              -Xcompiler -fPIC,-O2,-Wall -I include -I $(PKG)/csrc
+              -Xcompiler -fPIC,-O2,-Wall -I include -I $(PKG)/csrc $(EXTRA_NVCC_FLAGS)
 
 SHARP_SRCS := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 SHARP_HDRS := $(wildcard $(PKG)/csrc/*.cuh) $(wildcard $(PKG)/csrc/*.h) include/sharp.h

@@ -203,7 +203,8 @@ __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type,
     return (f >= 0 && f < sp.n) ? make_int4(kLut, f, k - pf, 0) : make_int4(kEmpty, 0, 0, 0);
   }
   const int f = rho - sp.L2;
-  return (f >= 0 && f < sp.n) ? make_int4(kP2, f, k - pf - kLutTasks, 0) : make_int4(kEmpty, 0, 0, 0);
+  if (f < 0 || f >= sp.n) return make_int4(kEmpty, 0, 0, 0);
+  return make_int4(kP2, f, k - pf - kLutTasks, 0);
 }
 __device__ __forceinline__ void tile_xy(const Geo &g, int sub, int &C0, int &R0) {
   const int ty = sub / g.tiles_x;
@@ -280,81 +281,75 @@ __device__ __forceinline__ float4 dblock(const LaneRow &a, int s, int lane) {
   return make_float4(dm1, d0, d1, d2);
 }
 
-// ------------------------------------------------------- scalar border pixel
-// (pass-2 tiles: kRows2 rows, smem row 0 = global row R0-4)
-__device__ __forceinline__ float dsum_at(uint32_t tile, int i, int j, int R0, int C0w) {
-  const int s = 4 * i - R0 + 4, rel = 4 * j - C0w + kCol0;
-  return (float)blk4(lds_u32(tile_addr(tile, kRows2, s, rel)), lds_u32(tile_addr(tile, kRows2, s + 1, rel)),
-                     lds_u32(tile_addr(tile, kRows2, s + 2, rel)), lds_u32(tile_addr(tile, kRows2, s + 3, rel)));
-}
-
-// U at (r, c), any pixel: body formula of L146 or the border rules of
-// L140-L142 (the last writer of steps i..vii), from the smem tile.
-__device__ float u_any(uint32_t tile, int r, int c, int W, int H, int R0, int C0w) {
-  const int w = W >> 2, h = H >> 2;
-  const bool ring = r < 2 || r >= H - 2 || c < 2 || c >= W - 2;
-  if (!ring) {
-    const int i = (r - 2) >> 2, a = (r - 2) & 3, j = (c - 2) >> 2, b = (c - 2) & 3;
-    const float wt = (float)wt_of((a + 2) & 3), wl = (float)wl_of((b + 2) & 3);
-    const float v0 = __fmaf_rn(8.0f - wt, dsum_at(tile, i + 1, j, R0, C0w), __fmul_rn(wt, dsum_at(tile, i, j, R0, C0w)));
-    const float v1 =
-        __fmaf_rn(8.0f - wt, dsum_at(tile, i + 1, j + 1, R0, C0w), __fmul_rn(wt, dsum_at(tile, i, j + 1, R0, C0w)));
-    return __fmaf_rn((8.0f - wl) * (1.0f / 1024.0f), v1, __fmul_rn(wl * (1.0f / 1024.0f), v0));
-  }
-  if (r >= H - 2 && c >= W - 2) return __fmul_rn(dsum_at(tile, h - 1, w - 1, R0, C0w), 1.0f / 16.0f);  // (vii)
-  if ((c <= 1 || c >= W - 2) && r <= H - 3) {                                                             // columns
-    const int j = (c <= 1) ? 0 : w - 1;
-    if (c <= 1 && r <= 1) return __fmul_rn(dsum_at(tile, 0, 0, R0, C0w), 1.0f / 16.0f);  // (v) then (vi)
-    const int rr = (r == H - 3) ? H - 4 : r;  // third last <- fourth last
-    const int i = rr >> 2, k = rr & 3;
-    const float x = dsum_at(tile, i, j, R0, C0w);
-    return k == 0 ? __fmul_rn(x, 1.0f / 16.0f) : line_val(x, dsum_at(tile, i + 1, j, R0, C0w), k);
-  }
-  const int i = (r <= 1) ? 0 : h - 1;  // rows 0/1: line of D row 0; rows H-2/H-1: D row h-1
-  const int cc = (c == W - 3) ? W - 4 : c;
-  const int j = cc >> 2, k = cc & 3;
-  const float x = dsum_at(tile, i, j, R0, C0w);
-  return k == 0 ? __fmul_rn(x, 1.0f / 16.0f) : line_val(x, dsum_at(tile, i, j + 1, R0, C0w), k);
-}
-
-// The whole pipeline for one pixel with scalar code (specialised border pass).
-__device__ uint32_t pixel_generic(uint32_t tile, uint32_t lut, int r, int c, int W, int H, int R0, int C0w) {
-  const int s0 = r - R0 + 4, rel0 = c - C0w + kCol0;
-  const int o = (int)lds_u8(tile_addr(tile, kRows2, s0, rel0));
-  int pe = 0, mx = 255, mn = 0;
-  if (!(r == 0 || r == H - 1 || c == 0 || c == W - 1)) {  // Sobel frame (L160) / overshoot frame (L208)
-    int v[3][3];
-#pragma unroll
-    for (int u = 0; u < 3; ++u)
-#pragma unroll
-      for (int q = 0; q < 3; ++q) v[u][q] = (int)lds_u8(tile_addr(tile, kRows2, s0 + u - 1, rel0 + q - 1));
-    const int gx = (v[0][2] + 2 * v[1][2] + v[2][2]) - (v[0][0] + 2 * v[1][0] + v[2][0]);
-    const int gy = (v[2][0] + 2 * v[2][1] + v[2][2]) - (v[0][0] + 2 * v[0][1] + v[0][2]);
-    pe = abs(gx) + abs(gy);
-    mx = 0;
-    mn = 255;
-#pragma unroll
-    for (int u = 0; u < 3; ++u)
-#pragma unroll
-      for (int q = 0; q < 3; ++q) {
-        mx = max(mx, v[u][q]);
-        mn = min(mn, v[u][q]);
-      }
-  }
-  const float U = u_any(tile, r, c, W, H, R0, C0w);
-  const float2 L = lds_f2(lut + 8u * (uint32_t)pe);
-  const float E = __fsub_rn((float)o, U);
-  return sharpen_px(L.x, L.y, E, U, (float)mx, (float)mn);
-}
-
 // ========================================================== pass 2, one row
-// Output row of this lane (window rows a = r-1, b = r, c = r+1), interior
-// formulas only.  V = vertical interpolation (x 128) of the four D columns.
+// Output row of this lane (window rows a = r-1, b = r, c = r+1).
+// V = vertical interpolation (x 128) of the four D columns (body, L146);
+// D0 / D1 = 16*D of D rows r>>2 and (r>>2)+1 for the lane's D columns
+// j0-1..j0+2 (border lines).  edge: 1 if the lane holds image columns 0,1,
+// 2 if it holds W-2,W-1 (W % 16 == 0: only c0 == 0 / c0 == W-8), else 0.
 struct Wts {  // packed horizontal weights -w/1024 for pixel pairs (x, x+1)
   unsigned long long a01, b01, a23, b23;
 };
+__device__ __forceinline__ float div16(float s) { return __fmul_rn(s, 1.0f / 16.0f); }
+
+// The 2-pixel ring (L140-L142 upscale border, L160 Sobel frame, L208
+// overshoot frame): overrides of -U, pEdge and the overshoot window.
+__device__ __forceinline__ void set_frame_px(uint32_t pe[4], uint32_t MX[4], uint32_t MN[4], int x) {
+  set_px(pe, x, 0u);         // Sobel frame: 0
+  set_px(MX, x, kF16_255);   // overshoot frame: the clamped preliminary value,
+  set_px(MN, x, 0u);         // i.e. window [0, 255]
+}
+// Rows 0,1 (line of D row 0) and H-2,H-1 (line of D row h-1): here D0 is
+// that D row; the corners follow the step order (v)-(vii).
+__device__ __forceinline__ void ring_rows(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4],
+                                          const float4 &D0, const float4 &D1, int r, int c0, int W, int H,
+                                          int edge) {
+  const float q0 = D0.y, q1 = D0.z, q2 = D0.w;
+  float u[8] = {div16(q0),         line_val(q0, q1, 1), line_val(q0, q1, 2), line_val(q0, q1, 3),
+                div16(q1),         line_val(q1, q2, 1), line_val(q1, q2, 2), line_val(q1, q2, 3)};
+  if (c0 + 5 == W - 3) u[5] = div16(q1);  // third last <- fourth last
+  const bool top = r < 2;
+  if (edge == 1 && top) u[1] = div16(q0);  // (v)+(vi): top-left 2x2 = D[0][0]
+  if (edge == 2) {                         // columns W-2, W-1 (D column w-1 = j0+1)
+    const float v = (top && r == 1) ? line_val(D0.z, D1.z, 1) : div16(D0.z);
+    u[6] = v;
+    u[7] = v;
+  }
+#pragma unroll
+  for (int x = 0; x < 8; ++x) NU[x] = -u[x];
+  if (edge == 1) set_frame_px(pe, MX, MN, 0);  // column 0 (rows 1, H-2)
+  if (edge == 2) set_frame_px(pe, MX, MN, 7);  // column W-1
+  if (r == 0 || r == H - 1) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      pe[i] = 0u;
+      MX[i] = kF16_255 | (kF16_255 << 16);
+      MN[i] = 0u;
+    }
+  }
+}
+// Columns 0,1 / W-2,W-1 on rows 2..H-3 (lines of D columns 0 / w-1).
+__device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4],
+                                          const float4 &D0, const float4 &D1, int r, int H, int edge) {
+  const int rr = (r == H - 3) ? H - 4 : r;  // third last <- fourth last
+  const int k = rr & 3;
+  const float x0 = edge == 1 ? D0.y : D0.z, x1 = edge == 1 ? D1.y : D1.z;
+  const float v = -(k == 0 ? div16(x0) : line_val(x0, x1, k));
+  if (edge == 1) {
+    NU[0] = v;
+    NU[1] = v;
+    set_frame_px(pe, MX, MN, 0);
+  } else if (edge == 2) {
+    NU[6] = v;
+    NU[7] = v;
+    set_frame_px(pe, MX, MN, 7);
+  }
+}
+
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
-                                       const Wts &wt, uint32_t lut_q, uint8_t *orow, bool store) {
+                                       const float4 &D0, const float4 &D1, const Wts &wt, uint32_t lut_q,
+                                       uint8_t *orow, bool store, int r, int c0, int W, int H, bool edge_warp,
+                                       int edge) {
   uint32_t pe[4], MX[4], MN[4];
   sobel(ra, rb, rc, pe);
 #pragma unroll
@@ -369,7 +364,12 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   const float2 nu23 = lin2(V.y, V.z, wt.a23, wt.b23);
   const float2 nu45 = lin2(V.y, V.z, wt.a01, wt.b01);
   const float2 nu67 = lin2(V.z, V.w, wt.a23, wt.b23);
-  const float NU[8] = {nu01.x, nu01.y, nu23.x, nu23.y, nu45.x, nu45.y, nu67.x, nu67.y};
+  float NU[8] = {nu01.x, nu01.y, nu23.x, nu23.y, nu45.x, nu45.y, nu67.x, nu67.y};
+  if (r < 2 || r >= H - 2) {  // warp-uniform
+    ring_rows(NU, pe, MX, MN, D0, D1, r, c0, W, H, edge);
+  } else if (edge_warp) {     // warp-uniform; only the edge lane changes
+    ring_cols(NU, pe, MX, MN, D0, D1, r, H, edge);
+  }
   float P[8], T8[8], osc[8];
 #pragma unroll
   for (int x = 0; x < 8; ++x) {
@@ -409,6 +409,10 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
                                         int R0, int lane) {
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
+  // W % 16 == 0: image columns 0,1 are in the lane with c0 == 0, columns
+  // W-2,W-1 in the lane with c0 == W-8.
+  const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
+  const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
   const LaneRow aw = lane_row(tile, kRows2, lane);
   // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (kept
   // opaque so the compiler emits one IMAD instead of folding the constant).
@@ -421,9 +425,10 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   // r = 4i+2 .. 4i+5: V(r+1) = V(r) + 2 (D_{i+1} - D_i), restarted at
   // r = 4i+2 with V = 7 D_i + D_{i+1} (all exact integers, x 128).
   const float4 Dp = dblock(aw, 0, lane);  // D row k0-1
-  float4 Dc = dblock(aw, 4, lane);        // D row k0 (= row r>>2)
-  float4 V = f4fma(5.0f, Dc, f4fma(3.0f, Dp, make_float4(0.f, 0.f, 0.f, 0.f)));  // r = R0 (a' = 0): (3,5)
-  float4 slope = f4twice_diff(Dc, Dp);
+  float4 D0 = dblock(aw, 4, lane);        // D row r>>2
+  float4 D1 = dblock(aw, 8, lane);        // D row (r>>2)+1
+  float4 V = f4fma(5.0f, D0, f4fma(3.0f, Dp, make_float4(0.f, 0.f, 0.f, 0.f)));  // r = R0 (a' = 0): (3,5)
+  float4 slope = f4twice_diff(D0, Dp);
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
   uint8_t *orow = out + (size_t)R0 * W + c0;
@@ -436,47 +441,19 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
     for (int u = 0; u < 3; ++u) {
       const int rr = r + u;
       const int sm = rr - R0 + 4;
-      if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
-        const float4 Dn = dblock(aw, sm + 2, lane);
-        V = f4fma(7.0f, Dc, Dn);
-        slope = f4twice_diff(Dn, Dc);
-        Dc = Dn;  // (D row k is no longer needed)
+      if ((rr & 3) == 0 && rr != R0) {  // next D block row
+        D0 = D1;
+        D1 = dblock(aw, sm + 4, lane);
+      } else if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
+        V = f4fma(7.0f, D0, D1);
+        slope = f4twice_diff(D1, D0);
       }
       const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
-      p2_row(ra, rb, rc, V, wt, lut_q, orow, active && rr < rend);
+      p2_row(ra, rb, rc, V, D0, D1, wt, lut_q, orow, active && rr < rend, rr, c0, W, H, edge_warp, edge);
       V = f4add(V, slope);
       orow += W;
       ra = rb;
       rb = rc;
-    }
-  }
-
-  // Specialised border pass: the 2-pixel ring inside this tile -- rows 0,1
-  // and H-2,H-1, columns 0,1 and W-2,W-1 -- recomputed with the scalar rules.
-  const bool top = (R0 == 0), bot = (R0 + kTH >= H - 2);
-  const bool left = (C0w == 0), right = (C0w <= W - 2 && W - 2 < C0w + kTW);
-  if (top || bot || left || right) {
-    __syncwarp();
-    const int ncols = min(kTW, W - C0w);
-    if (top || bot) {
-      const int r0 = top ? 0 : H - 2;
-      const int nrow = (top && bot) ? 4 : 2;  // tiny images: both
-      for (int idx = lane; idx < nrow * ncols; idx += 32) {
-        const int q = idx / ncols;
-        const int r = (top && bot) ? (q < 2 ? q : H - 4 + q) : r0 + q;
-        if (r < R0 || r >= rend) continue;
-        const int c = C0w + idx % ncols;
-        out[(size_t)r * W + c] = (uint8_t)pixel_generic(tile, lut, r, c, W, H, R0, C0w);
-      }
-    }
-    if (left || right) {
-      const int ncol = (left ? 2 : 0) + (right ? 2 : 0);
-      for (int idx = lane; idx < (rend - R0) * ncol; idx += 32) {
-        const int r = R0 + idx / ncol;
-        const int k = idx % ncol;  // left: columns 0,1; then W-2, W-1
-        const int c = left ? (k < 2 ? k : W - 4 + k) : W - 2 + k;
-        out[(size_t)r * W + c] = (uint8_t)pixel_generic(tile, lut, r, c, W, H, R0, C0w);
-      }
     }
   }
 }
@@ -545,10 +522,26 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     // ------------------------------------------------------------ producer
     if (lane != 0) return;
     const unsigned long long arrivals = (unsigned long long)(g.per_frame * kWarpsT) << kAccShift;
+    int t_next = (int)atomicAdd(sp.task_counter, 1u);
     for (int i = 0;; ++i) {
       const int b = i & 1;
+      const int4 d = decode(sp, t_next);
+      // Resolve the task's dependency first (before waiting for the stage).
+      unsigned long long S = 0;
+      if (d.x == kLut) {
+        // every pass-1 warp of the frame has added its partial (the global
+        // barrier of L174's reduction)
+        while (((S = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(500);
+      } else if (d.x == kP2) {
+        // the frame's LUT tasks (grabbed earlier) have finished
+        while (ld_relaxed_u32(&sp.lut_done[d.y]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(500);
+        fence_acquire();
+        fence_proxy_async_global();
+      }
       if (i >= 2) mbar_wait(empty0 + 8u * b, (uint32_t)(((i >> 1) - 1) & 1));
-      const int4 d = decode(sp, (int)atomicAdd(sp.task_counter, 1u));
+      // Grab the following task now: the atomic's latency overlaps this
+      // task's loads and the next empty-wait.
+      if (d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
       stage_task[b] = d;
       const uint32_t full = full0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
       if (d.x == kP1 || d.x == kP2) {
@@ -561,22 +554,18 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
           mbar_expect_tx(full, (uint32_t)(nw * kBox1));
           for (int w = 0; w < nw; ++w) tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1, kRows1, d.y, full);
         } else {
-          // dependency: the frame's LUT tasks (grabbed earlier) have finished
-          while (ld_relaxed_u32(&sp.lut_done[d.y]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(500);
-          fence_acquire();
-          fence_proxy_async_global();
+#ifdef SHARP_EXP_NO_LUT  // timing experiment only (stale LUTs)
+          mbar_expect_tx(full, (uint32_t)(nw * kBox2));
+#else
           mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
+#endif
           for (int w = 0; w < nw; ++w) tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4, kRows2, d.y, full);
+#ifndef SHARP_EXP_NO_LUT
           bulk_copy(st + kWarpsT * kSlot, sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
+#endif
         }
       } else {
-        if (d.x == kLut) {
-          // dependency: every pass-1 warp of the frame has added its partial
-          // (the global barrier of L174's reduction)
-          unsigned long long a;
-          while (((a = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(500);
-          stage_sum[b] = a & ((1ull << kAccShift) - 1);
-        }
+        if (d.x == kLut) stage_sum[b] = S & ((1ull << kAccShift) - 1);
         mbar_arrive(full);  // no data: LUT, empty or end task
         if (d.x == kEnd) break;
       }
