@@ -64,7 +64,8 @@ constexpr int kPitch = 256;           // region A pitch
 constexpr int kPitchB = 16;           // region B pitch
 constexpr int kCol0 = 16;             // region-A column of C0w
 constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+kTH+3
-constexpr int kRows1 = kTH + 2;       // pass-1 box rows: R0-1 .. R0+kTH
+constexpr int kTH1 = 18;              // pass-1 output rows per warp tile (fits the same slot)
+constexpr int kRows1 = kTH1 + 2;      // pass-1 box rows: R0-1 .. R0+kTH1
 constexpr int kBox2 = (kPitch + kPitchB) * kRows2;
 constexpr int kBox1 = (kPitch + kPitchB) * kRows1;
 constexpr int kSlot = (kBox2 + 127) / 128 * 128;  // per-warp smem slot (128-B aligned)
@@ -74,6 +75,7 @@ constexpr int kStage = kWarpsT * kSlot + kLutBytes;
 constexpr int kSmem = 2 * kStage + 64;
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
+static_assert(kTH1 % 3 == 0 && kBox1 <= kSlot, "pass-1 tiles");
 static_assert(kLutSize % kLutPerTask == 0, "LUT tasks");
 
 // ------------------------------------------------------------ TMA / mbarrier
@@ -158,16 +160,10 @@ __device__ __forceinline__ float2 sub2(float2 a, float2 b) {
 // ------------------------------------------------------------------ tasks
 struct Geo {
   int W, H;
-  int tiles_x;    // CTA tiles per row band (ceil(W / 960))
-  int per_frame;  // CTA tiles per frame
+  int tiles_x;     // CTA tiles per row band (ceil(W / 960))
+  int per_frame;   // pass-2 CTA tiles per frame (kTH rows)
+  int per_frame1;  // pass-1 CTA tiles per frame (kTH1 rows)
 };
-__device__ __forceinline__ void tile_of(const Geo &g, int t, int &f, int &C0, int &R0) {
-  f = t / g.per_frame;
-  const int rem = t - f * g.per_frame;
-  const int ty = rem / g.tiles_x;
-  C0 = (rem - ty * g.tiles_x) * kCtaCols;
-  R0 = ty * kTH;
-}
 
 // The task sequence is a list of rounds; round rho holds
 //   [pass-1 tasks of frame rho][LUT tasks of frame rho-L1][pass-2 tasks of frame rho-L2]
@@ -196,20 +192,20 @@ constexpr int kAccShift = 40;
 __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type, frame, sub, 0}
   if (t >= sp.ntasks) return make_int4(kEnd, 0, 0, 0);
   const int rho = t / sp.per_round, k = t - rho * sp.per_round;
-  const int pf = sp.g.per_frame;
-  if (k < pf) return rho < sp.n ? make_int4(kP1, rho, k, 0) : make_int4(kEmpty, 0, 0, 0);
-  if (k < pf + kLutTasks) {
+  const int pf1 = sp.g.per_frame1;
+  if (k < pf1) return rho < sp.n ? make_int4(kP1, rho, k, 0) : make_int4(kEmpty, 0, 0, 0);
+  if (k < pf1 + kLutTasks) {
     const int f = rho - sp.L1;
-    return (f >= 0 && f < sp.n) ? make_int4(kLut, f, k - pf, 0) : make_int4(kEmpty, 0, 0, 0);
+    return (f >= 0 && f < sp.n) ? make_int4(kLut, f, k - pf1, 0) : make_int4(kEmpty, 0, 0, 0);
   }
   const int f = rho - sp.L2;
   if (f < 0 || f >= sp.n) return make_int4(kEmpty, 0, 0, 0);
-  return make_int4(kP2, f, k - pf - kLutTasks, 0);
+  return make_int4(kP2, f, k - pf1 - kLutTasks, 0);
 }
-__device__ __forceinline__ void tile_xy(const Geo &g, int sub, int &C0, int &R0) {
+__device__ __forceinline__ void tile_xy(const Geo &g, int sub, int th, int &C0, int &R0) {
   const int ty = sub / g.tiles_x;
   C0 = (sub - ty * g.tiles_x) * kCtaCols;
-  R0 = ty * kTH;
+  R0 = ty * th;
 }
 // Polling loads: relaxed (no L1 invalidation per poll); the caller issues
 // one acquire fence after the awaited value was seen.
@@ -407,6 +403,9 @@ __device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y)
 
 __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__restrict__ out, int W, int H, int C0w,
                                         int R0, int lane) {
+#ifdef SHARP_EXP_NO_P2  // timing experiment only
+  return;
+#endif
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
   // W % 16 == 0: image columns 0,1 are in the lane with c0 == 0, columns
@@ -460,6 +459,9 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
 
 // ========================================================== pass 1 (warp)
 __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, int R0, int lane) {
+#ifdef SHARP_EXP_NO_P1  // timing experiment only
+  return 0.0f;
+#endif
   const int c0 = C0w + 8 * lane;
   const LaneRow aw = lane_row(tile, kRows1, lane);
   // Sobel-body pixels of this lane (not frame columns, not beyond the image).
@@ -475,7 +477,7 @@ __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, i
   // per-lane branches.
   float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 #pragma unroll 1
-  for (int m = 0; m < kTH; m += 3) {
+  for (int m = 0; m < kTH1; m += 3) {
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
       const int r = R0 + m + a;
@@ -521,7 +523,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
   if (warp == kWarpsT) {
     // ------------------------------------------------------------ producer
     if (lane != 0) return;
-    const unsigned long long arrivals = (unsigned long long)(g.per_frame * kWarpsT) << kAccShift;
+    const unsigned long long arrivals = (unsigned long long)(g.per_frame1 * kWarpsT) << kAccShift;
     int t_next = (int)atomicAdd(sp.task_counter, 1u);
     for (int i = 0;; ++i) {
       const int b = i & 1;
@@ -546,7 +548,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       const uint32_t full = full0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
       if (d.x == kP1 || d.x == kP2) {
         int C0, R0;
-        tile_xy(g, d.z, C0, R0);
+        tile_xy(g, d.z, d.x == kP1 ? kTH1 : kTH, C0, R0);
         int nw = 0;
 #pragma unroll
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
@@ -602,7 +604,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       if (lane == 0) atomicAdd(&sp.lut_done[f], 1u);
     } else if (d.x == kP1) {
       int C0, R0;
-      tile_xy(g, d.z, C0, R0);
+      tile_xy(g, d.z, kTH1, C0, R0);
       const int C0w = C0 + warp * kTW;
       const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.H, C0w, R0, lane) : 0.0f;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
@@ -613,7 +615,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       if (lane == 0) atomicAdd(&sp.acc[d.y], (1ull << kAccShift) + (unsigned long long)ws);
     } else if (d.x == kP2) {
       int C0, R0;
-      tile_xy(g, d.z, C0, R0);
+      tile_xy(g, d.z, kTH, C0, R0);
       const int C0w = C0 + warp * kTW;
       if (C0w < g.W)
         p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H, C0w, R0, lane);
@@ -682,8 +684,9 @@ cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p
   sp.g.H = H;
   sp.g.tiles_x = (W + kCtaCols - 1) / kCtaCols;
   sp.g.per_frame = sp.g.tiles_x * ((H + kTH - 1) / kTH);
+  sp.g.per_frame1 = sp.g.tiles_x * ((H + kTH1 - 1) / kTH1);
   sp.n = a.n;
-  sp.per_round = 2 * sp.g.per_frame + kLutTasks;
+  sp.per_round = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
   const int grid = kCtasPerSm * num_sms();
   // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
   // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
@@ -693,6 +696,11 @@ cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p
   // LUT tasks take a few microseconds (f64 pow/exp): leave >= ~2 grid's worth
   // of grabs before the frame's pass-2 tasks.
   sp.L2 = sp.L1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
+#ifndef SHARP_EXP_LAG_MUL
+#define SHARP_EXP_LAG_MUL 2  // measured: 2x the minimal lags removes most dependency waits
+#endif
+  sp.L1 *= SHARP_EXP_LAG_MUL;
+  sp.L2 *= SHARP_EXP_LAG_MUL;
   sp.ntasks = (a.n + sp.L2) * sp.per_round;
   sp.prm = p;
   sp.acc = a.acc;
