@@ -100,18 +100,47 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       : "memory");
 }
 // One 3-D box {cols, rows, 1} of the [n][H][W] frames at (x, r, f) (x 16-B aligned).
-__device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, int x, int r, int f, uint32_t bar) {
+// L2 eviction-priority policies (createpolicy): pass-1 loads keep the frame
+// in L2 for its pass-2 re-read (evict_last); pass-2 loads and the output
+// stores are the last touch (evict_first).
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+#ifdef SHARP_EXP_NORMAL_FIRST
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+#else
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+#endif
+  return p;
+}
+__device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, int x, int r, int f, uint32_t bar,
+                                        uint64_t policy) {
   asm volatile(
-      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
-      "[%5];" ::"r"(dst),
-      "l"(map), "r"(x), "r"(r), "r"(f), "r"(bar)
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, "
+      "{%2, %3, %4}], [%5], %6;" ::"r"(dst),
+      "l"(map), "r"(x), "r"(r), "r"(f), "r"(bar), "l"(policy)
       : "memory");
 }
 // Both boxes of a warp tile (region A then region B at dst + kPitch*rows).
 __device__ __forceinline__ void tma_tile(uint32_t dst, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0w,
-                                         int r, int rows, int f, uint32_t bar) {
-  tma_box(dst, mapA, C0w - kCol0, r, f, bar);
-  tma_box(dst + (uint32_t)(kPitch * rows), mapB, C0w + 256 - kCol0, r, f, bar);
+                                         int r, int rows, int f, uint32_t bar, uint64_t policy) {
+  tma_box(dst, mapA, C0w - kCol0, r, f, bar, policy);
+  tma_box(dst + (uint32_t)(kPitch * rows), mapB, C0w + 256 - kCol0, r, f, bar, policy);
+}
+// Output store.  (Measured: an L2::cache_hint store costs ~5% of the step
+// through extra issue; plain STG.64 it is -- SHARP_EXP_HINT_STORE to compare.)
+__device__ __forceinline__ void st_stream_u64(uint8_t *p, uint2 v, uint64_t policy) {
+#ifndef SHARP_EXP_HINT_STORE
+  (void)policy;
+  *reinterpret_cast<uint2 *>(p) = v;
+#else
+  asm volatile("st.global.L2::cache_hint.v2.b32 [%0], {%1, %2}, %3;" ::"l"(p), "r"(v.x), "r"(v.y), "l"(policy)
+               : "memory");
+#endif
 }
 __device__ __forceinline__ void bulk_copy(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
@@ -344,7 +373,8 @@ __device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t 
 
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
                                        const float4 &D0, const float4 &D1, const Wts &wt, uint32_t lut_q,
-                                       uint8_t *orow, bool store, int r, int c0, int W, int H, bool edge_warp,
+                                       uint8_t *orow, uint64_t pol_out, bool store, int r, int c0, int W, int H,
+                                       bool edge_warp,
                                        int edge) {
   uint32_t pe[4], MX[4], MN[4];
   sobel(ra, rb, rc, pe);
@@ -387,7 +417,7 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
     o[x] = cvt_u8(__fmaf_rn(osc[x], d.x, T8[x]));  // osc max / osc min / P, clamp, RNE
     o[x + 1] = cvt_u8(__fmaf_rn(osc[x + 1], d.y, T8[x + 1]));
   }
-  if (store) *reinterpret_cast<uint2 *>(orow) = pack8(o);
+  if (store) st_stream_u64(orow, pack8(o), pol_out);
 }
 
 __device__ __forceinline__ float4 f4fma(float a, const float4 &x, const float4 &y) {  // a*x + y, exact here
@@ -413,6 +443,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
   const LaneRow aw = lane_row(tile, kRows2, lane);
+  const uint64_t pol_out = policy_evict_first();  // output: written once, never re-read
   // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (kept
   // opaque so the compiler emits one IMAD instead of folding the constant).
   uint32_t lut_q;
@@ -448,7 +479,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
         slope = f4twice_diff(D1, D0);
       }
       const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
-      p2_row(ra, rb, rc, V, D0, D1, wt, lut_q, orow, active && rr < rend, rr, c0, W, H, edge_warp, edge);
+      p2_row(ra, rb, rc, V, D0, D1, wt, lut_q, orow, pol_out, active && rr < rend, rr, c0, W, H, edge_warp, edge);
       V = f4add(V, slope);
       orow += W;
       ra = rb;
@@ -524,6 +555,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     // ------------------------------------------------------------ producer
     if (lane != 0) return;
     const unsigned long long arrivals = (unsigned long long)(g.per_frame1 * kWarpsT) << kAccShift;
+    const uint64_t pol_keep = policy_evict_last(), pol_drop = policy_evict_first();
     int t_next = (int)atomicAdd(sp.task_counter, 1u);
     for (int i = 0;; ++i) {
       const int b = i & 1;
@@ -554,14 +586,16 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
         if (d.x == kP1) {
           mbar_expect_tx(full, (uint32_t)(nw * kBox1));
-          for (int w = 0; w < nw; ++w) tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1, kRows1, d.y, full);
+          for (int w = 0; w < nw; ++w)
+            tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1, kRows1, d.y, full, pol_keep);
         } else {
 #ifdef SHARP_EXP_NO_LUT  // timing experiment only (stale LUTs)
           mbar_expect_tx(full, (uint32_t)(nw * kBox2));
 #else
           mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
 #endif
-          for (int w = 0; w < nw; ++w) tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4, kRows2, d.y, full);
+          for (int w = 0; w < nw; ++w)
+            tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4, kRows2, d.y, full, pol_drop);
 #ifndef SHARP_EXP_NO_LUT
           bulk_copy(st + kWarpsT * kSlot, sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
 #endif
