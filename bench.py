@@ -100,10 +100,20 @@ def dist_setup():
     return world, rank, local
 
 
-def split(n, world, rank):
-    base, rem = divmod(n, world)
-    start = rank * base + min(rank, rem)
-    return start, base + (1 if rank < rem else 0)
+def traffic_per_launch(px_per_launch):
+    """DRAM bytes (read + write) per launch of the dominant kernel, from the
+    committed ncu --set full capture of this kernel (profiles/<round>/
+    traffic.json: dram bytes per output pixel), scaled to this launch; None
+    if no capture is committed."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "traffic.json")))
+    if not files:
+        return None
+    try:
+        t = json.load(open(files[-1]))
+        return float(t["dram_bytes_per_px"]) * px_per_launch
+    except Exception:
+        return None
 
 
 def cpu_oracle_rate(frames, threads):
@@ -178,12 +188,13 @@ def main():
 
     import synth
     from paper_conf_icpp_fanjzac15_b200 import Sharpener
+    from paper_conf_icpp_fanjzac15_b200 import shard
 
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     W, H = args.width, args.height
-    start, n = split(args.frames, world, rank)
+    start, n = shard.frame_range(args.frames, world, rank)
     fb = W * H
     # Inputs: pinned host (for e2e) and a device copy (device-resident value).
     h_in = torch.empty((n, H, W), dtype=torch.uint8).pin_memory()
@@ -198,16 +209,10 @@ def main():
     sh = Sharpener(device=local)
     sh.set_stream(stream)
 
-    def barrier():
-        if world > 1:
-            dist.barrier()
+    barrier = shard.barrier
 
     def max_over_ranks(x):
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=f"cuda:{local}")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return shard.max_over_ranks(x, device=f"cuda:{local}")
 
     # ---- device-resident timed region
     for _ in range(args.warmup):
@@ -287,13 +292,13 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": workload_config(args, world),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None,
+                         "frac": achieved / peak, "traffic": traffic_per_launch(px_per_launch),
                          "kernel": kname, "peak_source": pk_src,
                          "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px_per_launch,
                          "kernel_avg_ms": k_avg_ms, "kernel_launches": k_launches,
                          "kernel_share_of_step": k_share, "step_frac": step_achieved / peak},
-            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": total_px // world,
-                    "d2h_bytes_per_step": total_px // world, "ms_per_step": e2e_ms,
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": total_px,
+                    "d2h_bytes_per_step": total_px, "ms_per_step": e2e_ms,
                     "api": "sharp_run_batch(pinned host in, pinned host out)"},
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clk.summary(),
