@@ -1,36 +1,34 @@
 // TMA-staged, warp-specialised, dynamically scheduled sm_100a "step" kernel
 // (the main path; needs W % 16 == 0 and 16-byte aligned frames -- the TMA
-// tensor-map rules).
+// tensor-map rules).  ONE launch processes a whole batch of frames.
 //
-// One launch c runs three kinds of tasks, grabbed in this order from a global
-// counter by persistent CTAs (2 per SM):
-//   1. LUT tasks of chunk c-1: the per-frame lookup tables
-//      adj(p) = A (p/m)^gamma (strength, L178) and
-//      osc(p) = clamp(G exp(-p/(K m)), 0, 1) (oscStrength, L184),
-//      128 entries per task, f64 rounded once (R9, R11);
-//   2. pass-1 tasks of chunk c: Sobel (L158-L172) + reduction (L174, sec.
-//      V-C): warp shuffle reduction, u64 atomics, and the last warp of a frame
-//      computes its mean (last-block-done);
-//   3. pass-2 tasks of chunk c-1: the fused per-pixel pipeline (downscale
-//      L130, upscale L140-L146, pError L148, Sobel, 3x3 max/min L182,
-//      strength lookup, preliminary L178, overshoot L180-L212) -> u8.
-// A pass-2 task's producer waits until its frame's LUT tasks are done (they
-// were grabbed earlier, so this cannot deadlock).  The chunk's input is
-// re-read from L2 by pass 2 in the next launch.
+// Persistent CTAs (3 per SM) grab tasks from a global counter.  The task list
+// is a sequence of rounds; round rho holds
+//   [pass-1 tasks of frame rho][LUT tasks of frame rho-L1][pass-2 tasks of frame rho-L2]
+//   * pass 1: Sobel (L158-L172) + reduction (L174, sec. V-C): warp-shuffle
+//     reduction and one packed u64 atomic per warp (arrival count | partial S);
+//   * LUT: per-frame tables adj(p) = A (p/m)^gamma (strength, L178) and
+//     osc(p) = clamp(G exp(-p/(K m)), 0, 1) (oscStrength, L184), 128 entries
+//     per task, f64 rounded once (R9, R11), once the frame's S is complete;
+//   * pass 2: the fused per-pixel pipeline (downscale L130, upscale L140-L146,
+//     pError L148, Sobel, 3x3 max/min L182, strength lookup, preliminary
+//     L178, overshoot L180-L212) -> u8, once the frame's LUT is written.
+// The lags L1 < L2 make the dependencies (checked by the producer before it
+// fills a stage) normally complete long before they are needed; a frame's
+// input is re-read by pass 2 from L2 (pass-1 loads carry evict_last).
 //
 // CTA = 4 compute warps + 1 producer warp.  A pass-1/2 task is a CTA tile of
-// 4 warp tiles side by side; a warp tile is 240 output columns x 24 rows.
-// The producer grabs tasks and issues one cp.async.bulk.tensor (TMA) box per
-// warp tile (out-of-image pixels are zero-filled by the TMA unit: no bounds
-// checks in the pixel loops) plus a bulk copy of the frame's LUT, into one of
-// two smem stages guarded by full/empty mbarriers -- no CTA-wide barrier in
-// the steady state.  Each lane owns 8 adjacent columns and walks down the
-// rows with a 3-row window unrolled by 3 (no register moves); lanes 30 and 31
-// fetch the right/left halo columns and hand them out by shuffle.
-//
-// Image border (the 2-pixel ring: upscale border lines L140-L142, Sobel frame
-// L160, overshoot frame L208): recomputed by a specialised scalar pass of the
-// warps whose tile touches it, after the interior code wrote the tile.
+// 4 warp tiles side by side; a warp tile is 240 output columns x 12 rows
+// (pass 2) or 18 rows (pass 1).  The producer issues two TMA boxes per warp
+// tile (out-of-image pixels are zero-filled: no bounds checks in the pixel
+// loops) plus a bulk copy of the frame's LUT, into one of two smem stages
+// guarded by full/empty mbarriers -- no CTA-wide barrier in the steady state.
+// Each lane owns 8 adjacent columns and walks down the rows with a 3-row
+// window unrolled by 3 (no register moves); lanes 30 and 31 fetch the
+// right/left halo columns and hand them out by shuffle.  The 2-pixel image
+// ring (upscale border lines L140-L142, Sobel frame L160, overshoot frame
+// L208) is handled in the same vectorised loop: a warp-uniform branch for
+// the ring rows, lane-predicated overrides for the ring columns.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
@@ -94,6 +92,18 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       ".reg .pred p;\n"
       "WAIT_%=:\n"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 1000000;\n"  // suspend (not spin) up to 1 ms
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+// Plain polling wait (no suspend-time hint).
+__device__ __forceinline__ void mbar_wait_spin(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
       "@!p bra WAIT_%=;\n"
       "}\n" ::"r"(bar),
       "r"(parity)
@@ -312,9 +322,13 @@ __device__ __forceinline__ float4 dblock(const LaneRow &a, int s, int lane) {
 // D0 / D1 = 16*D of D rows r>>2 and (r>>2)+1 for the lane's D columns
 // j0-1..j0+2 (border lines).  edge: 1 if the lane holds image columns 0,1,
 // 2 if it holds W-2,W-1 (W % 16 == 0: only c0 == 0 / c0 == W-8), else 0.
-struct Wts {  // packed horizontal weights -w/1024 for pixel pairs (x, x+1)
-  unsigned long long a01, b01, a23, b23;
-};
+// Packed horizontal weights -w/1024 for pixel pairs (x, x+1), in the constant
+// bank (loaded with LDC where used; as literals, ptxas kept rematerialising
+// them on every row under the 128-register cap -- measured 4% slower).
+// {lo, hi} = {-3, -1}, {-5, -7}, {-7, -5}, {-1, -3} / 1024 as f32 bit pairs.
+__constant__ unsigned long long c_wts[4] = {0xba800000bb400000ull, 0xbbe00000bba00000ull, 0xbba00000bbe00000ull,
+                                            0xbb400000ba800000ull};
+__device__ __forceinline__ unsigned long long cwt(int i) { return c_wts[i]; }
 __device__ __forceinline__ float div16(float s) { return __fmul_rn(s, 1.0f / 16.0f); }
 
 // The 2-pixel ring (L140-L142 upscale border, L160 Sobel frame, L208
@@ -372,7 +386,7 @@ __device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t 
 }
 
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
-                                       const float4 &D0, const float4 &D1, const Wts &wt, uint32_t lut_q,
+                                       const float4 &D0, const float4 &D1, uint32_t lut_q,
                                        uint8_t *orow, uint64_t pol_out, bool store, int r, int c0, int W, int H,
                                        bool edge_warp,
                                        int edge) {
@@ -386,10 +400,10 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   // Upscale body (L146, R3), horizontal step on pixel pairs; NU = -U, exact.
   //   x = 0,1: (3,5),(1,7) on (V0,V1);  x = 2,3: (7,1),(5,3) on (V1,V2)
   //   x = 4,5: (3,5),(1,7) on (V1,V2);  x = 6,7: (7,1),(5,3) on (V2,V3)
-  const float2 nu01 = lin2(V.x, V.y, wt.a01, wt.b01);
-  const float2 nu23 = lin2(V.y, V.z, wt.a23, wt.b23);
-  const float2 nu45 = lin2(V.y, V.z, wt.a01, wt.b01);
-  const float2 nu67 = lin2(V.z, V.w, wt.a23, wt.b23);
+  const float2 nu01 = lin2(V.x, V.y, cwt(0), cwt(1));
+  const float2 nu23 = lin2(V.y, V.z, cwt(2), cwt(3));
+  const float2 nu45 = lin2(V.y, V.z, cwt(0), cwt(1));
+  const float2 nu67 = lin2(V.z, V.w, cwt(2), cwt(3));
   float NU[8] = {nu01.x, nu01.y, nu23.x, nu23.y, nu45.x, nu45.y, nu67.x, nu67.y};
   if (r < 2 || r >= H - 2) {  // warp-uniform
     ring_rows(NU, pe, MX, MN, D0, D1, r, c0, W, H, edge);
@@ -423,8 +437,12 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
 __device__ __forceinline__ float4 f4fma(float a, const float4 &x, const float4 &y) {  // a*x + y, exact here
   return make_float4(__fmaf_rn(a, x.x, y.x), __fmaf_rn(a, x.y, y.y), __fmaf_rn(a, x.z, y.z), __fmaf_rn(a, x.w, y.w));
 }
-__device__ __forceinline__ float4 f4add(const float4 &x, const float4 &y) {
-  return make_float4(__fadd_rn(x.x, y.x), __fadd_rn(x.y, y.y), __fadd_rn(x.z, y.z), __fadd_rn(x.w, y.w));
+__device__ __forceinline__ float4 f4add(const float4 &x, const float4 &y) {  // two packed f32x2 adds
+  unsigned long long lo, hi;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(lo) : "l"(f2pack(x.x, x.y)), "l"(f2pack(y.x, y.y)));
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(hi) : "l"(f2pack(x.z, x.w)), "l"(f2pack(y.z, y.w)));
+  const float2 a = f2unpack(lo), b = f2unpack(hi);
+  return make_float4(a.x, a.y, b.x, b.y);
 }
 __device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y) {  // 2 (x - y), exact here
   return make_float4(__fmul_rn(2.0f, __fsub_rn(x.x, y.x)), __fmul_rn(2.0f, __fsub_rn(x.y, y.y)),
@@ -446,10 +464,9 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   const uint64_t pol_out = policy_evict_first();  // output: written once, never re-read
   // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (kept
   // opaque so the compiler emits one IMAD instead of folding the constant).
-  uint32_t lut_q;
-  asm volatile("mov.u32 %0, %1;" : "=r"(lut_q) : "r"(lut - (0x4B000000u << 3)));
-  constexpr float s = -1.0f / 1024.0f;
-  const Wts wt{f2pack(3 * s, 1 * s), f2pack(5 * s, 7 * s), f2pack(7 * s, 5 * s), f2pack(1 * s, 3 * s)};
+  // (a shuffle hides the value from ptxas, which would otherwise split the
+  // constant back out into one extra IADD per pixel)
+  const uint32_t lut_q = __shfl_sync(0xffffffffu, lut - (0x4B000000u << 3), 0);
   // smem row of global row R0-4 is 0: row r -> smem row r - R0 + 4.
   // Vertical interpolation (L146, R3) of D rows (i, i+1) is linear in r on
   // r = 4i+2 .. 4i+5: V(r+1) = V(r) + 2 (D_{i+1} - D_i), restarted at
@@ -463,6 +480,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
   uint8_t *orow = out + (size_t)R0 * W + c0;
   const int rend = min(R0 + kTH, H);
+  const int rend_l = active ? rend : R0;  // this lane stores rows < rend_l
 #pragma unroll 1
   for (int r = R0; r < rend; r += 3) {
     // 3 rows per iteration: the window rotation has period 3, so the
@@ -479,7 +497,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
         slope = f4twice_diff(D1, D0);
       }
       const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
-      p2_row(ra, rb, rc, V, D0, D1, wt, lut_q, orow, pol_out, active && rr < rend, rr, c0, W, H, edge_warp, edge);
+      p2_row(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
       V = f4add(V, slope);
       orow += W;
       ra = rb;
@@ -535,7 +553,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     step_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
                 const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, StepParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ int4 stage_task[2];                 // {type, frame, sub, 0}
+  __shared__ int4 stage_task[2];                 // {type, frame, C0, R0} (LUT tasks: {type, frame, q, 0})
   __shared__ unsigned long long stage_sum[2];    // LUT tasks: the frame's S
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t sbase = smem_u32(smem);
@@ -576,11 +594,11 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       // Grab the following task now: the atomic's latency overlaps this
       // task's loads and the next empty-wait.
       if (d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
-      stage_task[b] = d;
       const uint32_t full = full0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
       if (d.x == kP1 || d.x == kP2) {
         int C0, R0;
         tile_xy(g, d.z, d.x == kP1 ? kTH1 : kTH, C0, R0);
+        stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
         int nw = 0;
 #pragma unroll
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
@@ -601,6 +619,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
 #endif
         }
       } else {
+        stage_task[b] = d;
         if (d.x == kLut) stage_sum[b] = S & ((1ull << kAccShift) - 1);
         mbar_arrive(full);  // no data: LUT, empty or end task
         if (d.x == kEnd) break;
@@ -612,7 +631,11 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
   // -------------------------------------------------------------- consumers
   for (int i = 0;; ++i) {
     const int b = i & 1;
+#ifdef SHARP_EXP_SPIN_WAIT
+    mbar_wait_spin(full0 + 8u * b, (uint32_t)((i >> 1) & 1));
+#else
     mbar_wait(full0 + 8u * b, (uint32_t)((i >> 1) & 1));
+#endif
     const int4 d = stage_task[b];
     if (d.x == kEnd) break;
     const uint32_t st = sbase + (uint32_t)(b * kStage);
@@ -637,8 +660,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       __syncwarp();
       if (lane == 0) atomicAdd(&sp.lut_done[f], 1u);
     } else if (d.x == kP1) {
-      int C0, R0;
-      tile_xy(g, d.z, kTH1, C0, R0);
+      const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
       const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.H, C0w, R0, lane) : 0.0f;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
@@ -648,8 +670,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
       if (lane == 0) atomicAdd(&sp.acc[d.y], (1ull << kAccShift) + (unsigned long long)ws);
     } else if (d.x == kP2) {
-      int C0, R0;
-      tile_xy(g, d.z, kTH, C0, R0);
+      const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
       if (C0w < g.W)
         p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H, C0w, R0, lane);

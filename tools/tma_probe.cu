@@ -5,6 +5,7 @@
 #include <stdio.h>
 #include <stdint.h>
 #include <vector>
+#include <stdlib.h>
 
 __device__ __forceinline__ uint32_t su(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -30,7 +31,7 @@ __global__ void probe(const __grid_constant__ CUtensorMap m, int c, int r, uint8
   for (int i = threadIdx.x; i < nbytes; i += blockDim.x) out[i] = sm[i];
 }
 
-int main() {
+int main(int argc, char** argv) {
   cudaDriverEntryPointQueryResult q; void* p = nullptr;
   cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q);
   auto enc = (PFN_cuTensorMapEncodeTiled_v12000)p;
@@ -38,7 +39,13 @@ int main() {
   Case cases[] = {{1024, 64, 256, 40, 2, 0, 0}, {1024, 64, 256, 40, 2, -8, -4}, {16, 16, 256, 40, 2, 0, 0},
                   {16, 16, 256, 40, 2, -8, -4}, {1024, 64, 256, 40, 3, -8, -4}, {16, 16, 256, 40, 3, -8, -4},
                   {16, 16, 16, 8, 2, 0, 0}, {1024, 64, 128, 40, 2, 0, 0}};
-  for (auto& cs : cases) {
+  if (argc > 1) {  // one custom case: W H bw bh dims c r
+    Case c1{atoi(argv[1]), atoi(argv[2]), atoi(argv[3]), atoi(argv[4]), atoi(argv[5]), atoi(argv[6]), atoi(argv[7])};
+    cases[0] = c1;
+  }
+  int ncase = argc > 1 ? 1 : (int)(sizeof(cases) / sizeof(cases[0]));
+  for (int ci = 0; ci < ncase; ++ci) {
+    auto& cs = cases[ci];
     std::vector<uint8_t> h(cs.W * cs.H);
     for (int i = 0; i < cs.W * cs.H; ++i) h[i] = (uint8_t)(i * 7 + 3);
     uint8_t *d, *o; cudaMalloc(&d, h.size()); cudaMalloc(&o, 256 * 256);
