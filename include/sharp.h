@@ -26,9 +26,9 @@
  *  - Ownership: the caller owns every image buffer; the library never retains
  *    them past return and never frees them.  The context owns all device
  *    scratch, streams, events and pinned staging; sharp_destroy releases them.
- *  - Synchrony: sharp_run / sharp_run_batch / sharp_run_bands return after the
- *    output is complete.  sharp_enqueue_batch is asynchronous on the
- *    context's stream (device pointers only).
+ *  - Synchrony: sharp_run / sharp_run_batch return after the output is
+ *    complete.  sharp_enqueue_batch and the row-band calls are asynchronous
+ *    on the context's stream (device pointers only).
  *  - Threads: a context is used by one thread at a time.
  *  - After a sticky CUDA error the context is poisoned: every later call
  *    returns SHARP_ESTATE until sharp_destroy.
@@ -121,6 +121,33 @@ int sharp_get_stats(const sharp_ctx *ctx, sharp_stats *s);
 /* Per-frame pEdge sums S of the last run / enqueued batch (waits for the
  * context's stream).  n must not exceed the number of frames of that call. */
 int sharp_get_batch_sums(sharp_ctx *ctx, uint64_t *sums, int n);
+
+/* ---- Row-band sharding of ONE image.
+ * The image is split into row bands, one per process / GPU.  The only
+ * coupling between bands is the global pEdge mean ("the
+ * arithmetic mean of the elements in this matrix"), so a band runs in two
+ * calls around one all-reduce of a 64-bit sum:
+ *   1. sharp_band_edge_sum  -> *d_partial = sum of pEdge over rows [row0, row1)
+ *   2. the caller sums the partials of all bands into *d_total (e.g. NCCL
+ *      all-reduce through torch.distributed)
+ *   3. sharp_band_sharpen   -> output rows [row0, row1), bit-identical to the
+ *      same rows of sharp_run on the whole image.
+ * Geometry: band g owns output rows [row0, row1), multiples of 4 with
+ * 0 <= row0 < row1 <= h, so no 4x4 downscale block straddles two bands.  Its
+ * input `band` holds image rows [in0, in1) = [max(row0-4, 0), min(row1+4, h))
+ * (sharp_band_halo): the band plus 4 halo rows on each side -- the upscale of
+ * rows row0 .. row1-1 reads D rows row0/4-1 .. row1/4 (L146), the Sobel and
+ * the 3x3 overshoot window one row (L158-L172, L182).  Rows are dense, pitch w.
+ * Requirements: DEVICE pointers on the context's device; w % 16 == 0, `band`
+ * 16-byte aligned, `out` 8-byte aligned (the TMA path), w*h < 2^29 -- else
+ * SHARP_EUNSUPPORTED / SHARP_EINVAL.  d_partial / d_total: device uint64.
+ * Both calls are asynchronous on the context's stream (sharp_set_stream);
+ * `out` ((row1-row0) x w bytes) must not overlap `band`. */
+int sharp_band_halo(int h, int row0, int row1, int *in0, int *in1);
+int sharp_band_edge_sum(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
+                        uint64_t *d_partial);
+int sharp_band_sharpen(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
+                       const uint64_t *d_total, const sharp_params *params, uint8_t *out);
 
 /* Per-kernel device time accounting (CUDA events around every launch, on
  * the launch stream).  enable != 0 starts (and resets) accounting. */

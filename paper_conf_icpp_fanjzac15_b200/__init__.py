@@ -39,4 +39,7 @@ from .binding import (  # noqa: F401
     sharp_set_stream,
     sharp_strerror,
     sharp_version,
+    sharp_band_halo,
+    sharp_band_edge_sum,
+    sharp_band_sharpen,
 )

@@ -1,0 +1,104 @@
+"""Row-band sharding of ONE image over the ranks of a process group
+(DESIGN.md sec. 9).
+
+One process per GPU.  Rank g owns output rows [row0, row1) (multiples of 4,
+so no 4x4 downscale block of PAPER.md L130 straddles two bands).  The method
+couples the bands in exactly two places:
+
+* halo rows: the upscale of rows row0..row1-1 reads D rows row0/4-1 .. row1/4
+  (L146) and the Sobel / 3x3 overshoot window one row (L158-L172, L182), so a
+  band's input buffer holds 4 extra image rows above and below
+  (`halo_rows`, the C ABI's sharp_band_halo); `exchange_halos` fetches them
+  from the neighbouring ranks (point-to-point send/recv; NCCL over NVLink on
+  GPUs, gloo on CPU);
+* the pEdge mean (L174): each rank sums pEdge over its own rows
+  (sharp_band_edge_sum), one all-reduce of a 64-bit integer adds the partials,
+  and every rank builds the identical LUTs from the identical S
+  (sharp_band_sharpen) -- so the bands are bit-identical to the same rows of
+  the whole-image result.
+
+torch.distributed is plumbing only (the collective and the P2P transfers);
+every pixel is computed by libsharp.so.
+"""
+import torch
+import torch.distributed as dist
+
+HALO = 4  # image rows of halo per side
+
+
+def band_rows(h, world, rank):
+    """Rows [row0, row1) of rank `rank`: the h/4 downscale block rows split
+    as evenly as possible (the first (h/4) % world ranks get one more)."""
+    if h % 4 or h < 8 or world < 1 or not 0 <= rank < world:
+        raise ValueError("bad band request")
+    blocks = h // 4
+    if blocks < world:
+        raise ValueError(f"{h} rows cannot feed {world} bands of >= 4 rows")
+    base, rem = divmod(blocks, world)
+    start = rank * base + min(rank, rem)
+    count = base + (1 if rank < rem else 0)
+    return 4 * start, 4 * (start + count)
+
+
+def halo_rows(h, row0, row1):
+    """Image rows [in0, in1) a band's input buffer holds (sharp_band_halo)."""
+    return max(row0 - HALO, 0), min(row1 + HALO, h)
+
+
+def _world(group):
+    if not (dist.is_available() and dist.is_initialized()):
+        return 1, 0
+    return dist.get_world_size(group), dist.get_rank(group)
+
+
+def exchange_halos(own, h, row0, row1, group=None):
+    """own: this rank's rows [row0, row1) ([rows, w] uint8, any device).
+    Returns the band buffer of rows [in0, in1): own plus up to HALO rows from
+    each neighbour (rank-1 above, rank+1 below), by point-to-point transfers.
+    Every rank must call it (it pairs sends with the neighbours' receives)."""
+    world, rank = _world(group)
+    in0, in1 = halo_rows(h, row0, row1)
+    rows, w = own.shape
+    if rows != row1 - row0:
+        raise ValueError("own rows do not match [row0, row1)")
+    band = torch.empty((in1 - in0, w), dtype=own.dtype, device=own.device)
+    top, bot = row0 - in0, in1 - row1
+    band[top:top + rows].copy_(own)
+    if world == 1:
+        if top or bot:
+            raise ValueError("a single rank must own the whole image")
+        return band
+    ops = []
+    up_recv = band[:top] if top else None
+    dn_recv = band[top + rows:] if bot else None
+    peer = (lambda r: dist.get_global_rank(group, r)) if group is not None else (lambda r: r)
+    if rank > 0:  # exchange with the band above: it needs our first rows, we need its last
+        ops.append(dist.P2POp(dist.isend, own[:HALO].contiguous(), peer(rank - 1), group))
+        ops.append(dist.P2POp(dist.irecv, up_recv, peer(rank - 1), group))
+    if rank < world - 1:
+        ops.append(dist.P2POp(dist.isend, own[rows - HALO:].contiguous(), peer(rank + 1), group))
+        ops.append(dist.P2POp(dist.irecv, dn_recv, peer(rank + 1), group))
+    for req in dist.batch_isend_irecv(ops):
+        req.wait()
+    return band
+
+
+def sharpen_band(sharpener, band, w, h, row0, row1, params=None, out=None, group=None):
+    """Sharpen this rank's rows [row0, row1) of a w x h image.
+
+    band: CUDA uint8 tensor of image rows halo_rows(h, row0, row1).
+    Runs sharp_band_edge_sum -> all-reduce(sum) of the u64 partial over the
+    group (skipped when not distributed) -> sharp_band_sharpen, all on the
+    current CUDA stream.  Returns (out, S): out = [row1-row0, w] uint8 and S
+    the image's pEdge sum (a 1-element int64 CUDA tensor)."""
+    if out is None:
+        out = torch.empty((row1 - row0, w), dtype=torch.uint8, device=band.device)
+    stream = torch.cuda.current_stream(band.device)
+    sharpener.set_stream(stream)
+    s = torch.zeros(1, dtype=torch.int64, device=band.device)  # u64 bits; S < 2^40
+    sharpener.band_edge_sum(band, w, h, row0, row1, s)
+    world, _ = _world(group)
+    if world > 1:
+        dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)  # the L174 reduction across bands
+    sharpener.band_sharpen(band, w, h, row0, row1, s, out, params)
+    return out, s

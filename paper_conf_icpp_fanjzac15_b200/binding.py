@@ -60,6 +60,9 @@ _SIGS = {
     "sharp_strerror": ([_I], ctypes.c_char_p),
     "sharp_last_error": ([_P], ctypes.c_char_p),
     "sharp_version": ([], ctypes.c_char_p),
+    "sharp_band_halo": ([_I, _I, _I, ctypes.POINTER(_I), ctypes.POINTER(_I)], _I),
+    "sharp_band_edge_sum": ([_P, _P, _I, _I, _I, _I, _P], _I),
+    "sharp_band_sharpen": ([_P, _P, _I, _I, _I, _I, _P, ctypes.POINTER(SharpParams), _P], _I),
 }
 
 _lib = None
@@ -150,8 +153,13 @@ def sharp_default_params():
 
 
 def sharp_set_stream(ctx, stream):
-    """stream: torch.cuda.Stream, raw cudaStream_t int, or None (context's own)."""
+    """stream: torch.cuda.Stream, raw cudaStream_t int, or None (context's own).
+    torch's default stream has cuda_stream == 0, i.e. the legacy default
+    stream: it is passed as cudaStreamLegacy ((void *) 1), because a NULL
+    handle means "the context's own stream" in the C ABI."""
     s = getattr(stream, "cuda_stream", stream)
+    if hasattr(stream, "cuda_stream") and s == 0:
+        s = 1  # cudaStreamLegacy
     return _check(lib().sharp_set_stream(ctx, s), ctx)
 
 
@@ -204,6 +212,24 @@ def sharp_last_error(ctx):
 
 def sharp_version():
     return lib().sharp_version().decode()
+
+
+def sharp_band_halo(h, row0, row1):
+    """-> (in0, in1): the image rows a band's input buffer must hold."""
+    a, b = _I(), _I()
+    rc = lib().sharp_band_halo(h, row0, row1, ctypes.byref(a), ctypes.byref(b))
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_band_halo: {sharp_strerror(rc)}")
+    return a.value, b.value
+
+
+def sharp_band_edge_sum(ctx, band, w, h, row0, row1, d_partial):
+    return _check(lib().sharp_band_edge_sum(ctx, _addr(band), w, h, row0, row1, _addr(d_partial)), ctx)
+
+
+def sharp_band_sharpen(ctx, band, w, h, row0, row1, d_total, params, out):
+    return _check(lib().sharp_band_sharpen(ctx, _addr(band), w, h, row0, row1, _addr(d_total), _pp(params),
+                                           _addr(out)), ctx)
 
 
 # ---------------------------------------------------------------- convenience
@@ -277,3 +303,10 @@ class Sharpener:
 
     def kernel_times(self):
         return sharp_get_kernel_times(self.ctx)
+
+    # row bands of one image (orchestration in bands.py)
+    def band_edge_sum(self, band, w, h, row0, row1, d_partial):
+        sharp_band_edge_sum(self.ctx, band, w, h, row0, row1, d_partial)
+
+    def band_sharpen(self, band, w, h, row0, row1, d_total, out, params=None):
+        sharp_band_sharpen(self.ctx, band, w, h, row0, row1, d_total, params, out)

@@ -40,9 +40,22 @@ struct BatchLaunch {
   float2 *luts = nullptr;              // n * kLutSize (scratch)
   unsigned int *lut_done = nullptr;    // n; zero on entry
   unsigned int *task_counter = nullptr;  // 1; zero on entry
+  // row-band launches only (launch_band_tma):
+  unsigned long long *partial = nullptr;      // pass 1 out: the band's S
+  const unsigned long long *total = nullptr;  // pass 2 in: the all-reduced S
 };
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);
 cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
+
+// One row band [row_lo, row_hi) of a W x H image (sec. 8(e)): a.in holds
+// image rows [y0, y0 + rows_in) (the band plus its halo rows), a.out the
+// band's rows (a.out = first output row).  mode kStepPass1 sums the band's
+// pEdge into *a.partial (a.acc, a.task_counter zero on entry); kStepPass2
+// builds the LUT from *a.total and writes the band (3 launches: arm, step,
+// nothing else).  n = 1 frame; a.out is offset internally.
+enum StepMode { kStepAll = 0, kStepPass1 = 1, kStepPass2 = 2 };
+cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int row_lo, int row_hi, int y0, int rows_in,
+                            const Params &p, cudaStream_t stream);
 
 // Kernel launches issued per (pass-1, pass-2) chunk.
 constexpr int kLaunchesPerChunk = 2;

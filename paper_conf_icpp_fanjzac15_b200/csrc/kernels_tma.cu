@@ -198,10 +198,15 @@ __device__ __forceinline__ float2 sub2(float2 a, float2 b) {
 
 // ------------------------------------------------------------------ tasks
 struct Geo {
-  int W, H;
+  int W, H;        // the whole image (ring rows, Sobel frame, mean denominator)
   int tiles_x;     // CTA tiles per row band (ceil(W / 960))
   int per_frame;   // pass-2 CTA tiles per frame (kTH rows)
   int per_frame1;  // pass-1 CTA tiles per frame (kTH1 rows)
+  // Rows processed: [row_lo, row_hi) of the image (the whole image, or one
+  // row band, sec. 8(e)); the tensor map's row 0 is image row y0 (a band's
+  // buffer starts with its upper halo); rmax1 = min(H-2, row_hi-1) is the
+  // last row whose pEdge this launch sums.
+  int row_lo, row_hi, y0, rmax1;
 };
 
 // The task sequence is a list of rounds; round rho holds
@@ -212,6 +217,7 @@ struct Geo {
 enum TaskType { kEmpty = 0, kP1 = 1, kLut = 2, kP2 = 3, kEnd = -1 };
 struct StepParams {
   Geo g;
+  int mode;       // kStepAll, or a row band's kStepPass1 / kStepPass2
   int n;          // frames
   int L1, L2;     // round lags of the LUT and pass-2 tasks
   int per_round;  // 2 * per_frame + kLutTasks
@@ -230,6 +236,10 @@ struct StepParams {
 constexpr int kAccShift = 40;
 __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type, frame, sub, 0}
   if (t >= sp.ntasks) return make_int4(kEnd, 0, 0, 0);
+  // A row band's two launches (one frame): pass-1 tasks only; or the LUT
+  // tasks (S preset by band_prep_kernel) followed by the pass-2 tasks.
+  if (sp.mode == kStepPass1) return make_int4(kP1, 0, t, 0);
+  if (sp.mode == kStepPass2) return t < kLutTasks ? make_int4(kLut, 0, t, 0) : make_int4(kP2, 0, t - kLutTasks, 0);
   const int rho = t / sp.per_round, k = t - rho * sp.per_round;
   const int pf1 = sp.g.per_frame1;
   if (k < pf1) return rho < sp.n ? make_int4(kP1, rho, k, 0) : make_int4(kEmpty, 0, 0, 0);
@@ -244,7 +254,7 @@ __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type,
 __device__ __forceinline__ void tile_xy(const Geo &g, int sub, int th, int &C0, int &R0) {
   const int ty = sub / g.tiles_x;
   C0 = (sub - ty * g.tiles_x) * kCtaCols;
-  R0 = ty * th;
+  R0 = g.row_lo + ty * th;
 }
 // Polling loads: relaxed (no L1 invalidation per poll); the caller issues
 // one acquire fence after the awaited value was seen.
@@ -449,8 +459,9 @@ __device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y)
                      __fmul_rn(2.0f, __fsub_rn(x.z, y.z)), __fmul_rn(2.0f, __fsub_rn(x.w, y.w)));
 }
 
-__device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__restrict__ out, int W, int H, int C0w,
-                                        int R0, int lane) {
+// out: first row of the output rows [row_lo, row_hi).
+__device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__restrict__ out, int W, int H,
+                                        int row_lo, int row_hi, int C0w, int R0, int lane) {
 #ifdef SHARP_EXP_NO_P2  // timing experiment only
   return;
 #endif
@@ -478,8 +489,8 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   float4 slope = f4twice_diff(D0, Dp);
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
-  uint8_t *orow = out + (size_t)R0 * W + c0;
-  const int rend = min(R0 + kTH, H);
+  uint8_t *orow = out + (size_t)(R0 - row_lo) * W + c0;
+  const int rend = min(R0 + kTH, row_hi);
   const int rend_l = active ? rend : R0;  // this lane stores rows < rend_l
 #pragma unroll 1
   for (int r = R0; r < rend; r += 3) {
@@ -507,7 +518,7 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
 }
 
 // ========================================================== pass 1 (warp)
-__device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, int R0, int lane) {
+__device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int C0w, int R0, int lane) {
 #ifdef SHARP_EXP_NO_P1  // timing experiment only
   return 0.0f;
 #endif
@@ -533,7 +544,7 @@ __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int H, int C0w, i
       const RowD rc = derive_w<false>(row_words(aw, m + a + 2), lane);
       uint32_t pe[4];
       sobel(ra, rb, rc, pe);
-      if ((unsigned)(r - 1) < (unsigned)(H - 2)) {  // Sobel frame rows are 0 (L160); rows >= H skipped
+      if ((unsigned)(r - 1) < (unsigned)rmax1) {  // 1 <= r <= rmax1: Sobel frame rows are 0 (L160)
 #pragma unroll
         for (int x = 0; x < 8; ++x)
           acc[x] = add_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), acc[x]);
@@ -605,7 +616,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
         if (d.x == kP1) {
           mbar_expect_tx(full, (uint32_t)(nw * kBox1));
           for (int w = 0; w < nw; ++w)
-            tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1, kRows1, d.y, full, pol_keep);
+            tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1 - g.y0, kRows1, d.y, full, pol_keep);
         } else {
 #ifdef SHARP_EXP_NO_LUT  // timing experiment only (stale LUTs)
           mbar_expect_tx(full, (uint32_t)(nw * kBox2));
@@ -613,7 +624,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
           mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
 #endif
           for (int w = 0; w < nw; ++w)
-            tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4, kRows2, d.y, full, pol_drop);
+            tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4 - g.y0, kRows2, d.y, full, pol_drop);
 #ifndef SHARP_EXP_NO_LUT
           bulk_copy(st + kWarpsT * kSlot, sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
 #endif
@@ -662,7 +673,7 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
-      const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.H, C0w, R0, lane) : 0.0f;
+      const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.rmax1, C0w, R0, lane) : 0.0f;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
       // atomic per warp adding (1 << 40) + partial: the frame's arrival count
       // and sum in one word, so its LUT tasks can tell when S is complete
@@ -673,7 +684,8 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
       if (C0w < g.W)
-        p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H, C0w, R0, lane);
+        p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H, g.row_lo,
+                g.row_hi, C0w, R0, lane);
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(empty0 + 8u * b);  // stage b may be refilled
@@ -723,40 +735,80 @@ bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
          (size_t)W * H <= (1u << 29) && encode_fn() != nullptr;
 }
 
-cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream) {
+// Row-band helpers (one thread): arm a band's pass-2 launch with the
+// all-reduced S (arrival count complete, so the LUT tasks start at once), and
+// export a band's pass-1 partial S.
+__global__ void band_prep_kernel(unsigned long long *acc, unsigned int *lut_done, unsigned int *task_counter,
+                                 const unsigned long long *total, unsigned long long arrivals) {
+  acc[0] = arrivals | (total[0] & ((1ull << kAccShift) - 1));
+  lut_done[0] = 0;
+  task_counter[0] = 0;
+}
+__global__ void band_finish_kernel(const unsigned long long *acc, unsigned long long *partial) {
+  partial[0] = acc[0] & ((1ull << kAccShift) - 1);
+}
+
+struct StepGeometry {
+  int n, rows_in;               // tensor-map frames and rows
+  int row_lo, row_hi, y0;       // rows processed; image row of map row 0
+};
+
+cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, int W, int H, const Params &p,
+                        cudaStream_t stream) {
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
     attr = true;
   }
-  if (a.n <= 0) return cudaSuccess;
+  if (sg.n <= 0 || sg.row_hi <= sg.row_lo) return cudaSuccess;
   CUtensorMap m1A, m1B, m2A, m2B;  // the same frames: pass-1 / pass-2 box heights, regions A / B
-  if (!make_map(&m1A, a.in, a.n, W, H, kPitch, kRows1) || !make_map(&m1B, a.in, a.n, W, H, kPitchB, kRows1) ||
-      !make_map(&m2A, a.in, a.n, W, H, kPitch, kRows2) || !make_map(&m2B, a.in, a.n, W, H, kPitchB, kRows2))
+  const int R = sg.rows_in;
+  if (!make_map(&m1A, a.in, sg.n, W, R, kPitch, kRows1) || !make_map(&m1B, a.in, sg.n, W, R, kPitchB, kRows1) ||
+      !make_map(&m2A, a.in, sg.n, W, R, kPitch, kRows2) || !make_map(&m2B, a.in, sg.n, W, R, kPitchB, kRows2))
     return cudaErrorInvalidValue;
   StepParams sp;
   sp.g.W = W;
   sp.g.H = H;
+  sp.g.row_lo = sg.row_lo;
+  sp.g.row_hi = sg.row_hi;
+  sp.g.y0 = sg.y0;
+  sp.g.rmax1 = std::min(H - 2, sg.row_hi - 1);
+  const int rows = sg.row_hi - sg.row_lo;
   sp.g.tiles_x = (W + kCtaCols - 1) / kCtaCols;
-  sp.g.per_frame = sp.g.tiles_x * ((H + kTH - 1) / kTH);
-  sp.g.per_frame1 = sp.g.tiles_x * ((H + kTH1 - 1) / kTH1);
-  sp.n = a.n;
+  sp.g.per_frame = sp.g.tiles_x * ((rows + kTH - 1) / kTH);
+  sp.g.per_frame1 = sp.g.tiles_x * ((rows + kTH1 - 1) / kTH1);
+  sp.mode = mode;
+  sp.n = sg.n;
   sp.per_round = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
   const int grid = kCtasPerSm * num_sms();
-  // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
-  // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
-  // one more round separates those from its pass-2 tasks.
-  const int in_flight = 3 * grid;
-  sp.L1 = (in_flight + sp.per_round - 1) / sp.per_round + 1;
-  // LUT tasks take a few microseconds (f64 pow/exp): leave >= ~2 grid's worth
-  // of grabs before the frame's pass-2 tasks.
-  sp.L2 = sp.L1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
+  if (mode == kStepPass1) {
+    sp.L1 = sp.L2 = 0;
+    sp.ntasks = sp.g.per_frame1;
+  } else if (mode == kStepPass2) {
+    sp.L1 = sp.L2 = 0;
+    sp.ntasks = kLutTasks + sp.g.per_frame;
+  } else {
+    // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
+    // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
+    // LUT tasks (a few microseconds of f64 pow/exp) are followed by >= ~2
+    // grids' worth of grabs before the frame's pass-2 tasks.
+    const int in_flight = 3 * grid;
+    sp.L1 = (in_flight + sp.per_round - 1) / sp.per_round + 1;
+    sp.L2 = sp.L1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
 #ifndef SHARP_EXP_LAG_MUL
 #define SHARP_EXP_LAG_MUL 2  // measured: 2x the minimal lags removes most dependency waits
 #endif
-  sp.L1 *= SHARP_EXP_LAG_MUL;
-  sp.L2 *= SHARP_EXP_LAG_MUL;
-  sp.ntasks = (a.n + sp.L2) * sp.per_round;
+    sp.L1 *= SHARP_EXP_LAG_MUL;
+    sp.L2 *= SHARP_EXP_LAG_MUL;
+    // The lag rounds past the last frame hold only empty tasks: for a short
+    // batch use the minimal lags (a dependency wait stalls one producer; it
+    // cannot deadlock -- every dependency was grabbed, and issued, earlier).
+    if (sg.n < sp.L2) {
+      sp.L1 = 1;
+      sp.L2 = 2;
+    }
+    sp.ntasks = (sg.n + sp.L2) * sp.per_round;
+  }
   sp.prm = p;
   sp.acc = a.acc;
   sp.sums = a.sums;
@@ -765,8 +817,23 @@ cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p
   sp.lut_done = a.lut_done;
   sp.out = a.out;
   sp.task_counter = a.task_counter;
+  if (mode == kStepPass2) {
+    band_prep_kernel<<<1, 1, 0, stream>>>(a.acc, a.lut_done, a.task_counter, a.total,
+                                          (unsigned long long)(sp.g.per_frame1 * kWarpsT) << kAccShift);
+  }
   step_kernel<<<grid, kThreadsT, kSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
+  if (mode == kStepPass1) band_finish_kernel<<<1, 1, 0, stream>>>(a.acc, a.partial);
   return cudaGetLastError();
+}
+
+cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream) {
+  return launch_step(a, StepGeometry{a.n, H, 0, H, 0}, kStepAll, W, H, p, stream);
+}
+
+cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int row_lo, int row_hi, int y0, int rows_in,
+                            const Params &p, cudaStream_t stream) {
+  if (mode != kStepPass1 && mode != kStepPass2) return cudaErrorInvalidValue;
+  return launch_step(a, StepGeometry{1, rows_in, row_lo, row_hi, y0}, mode, W, H, p, stream);
 }
 
 }  // namespace sharp

@@ -389,9 +389,93 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   return SHARP_OK;
 }
 
+// Row bands (sec. 8(e) of SURVEY.md / DESIGN.md sec. 9).
+int band_halo(int h, int row0, int row1, int *in0, int *in1) {
+  if (h < 8 || (h & 3) || row0 < 0 || row1 > h || row0 >= row1 || (row0 & 3) || (row1 & 3)) return SHARP_EINVAL;
+  *in0 = std::max(row0 - 4, 0);
+  *in1 = std::min(row1 + 4, h);
+  return SHARP_OK;
+}
+
+int band_impl(sharp_ctx *ctx, int mode, const uint8_t *band, int w, int h, int row0, int row1,
+              unsigned long long *partial, const unsigned long long *total, const sharp_params *pp, uint8_t *out) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  int in0 = 0, in1 = 0;
+  if (!band || (mode == sharp::kStepPass1 ? !partial : (!total || !out)))
+    return set_err(ctx, SHARP_EINVAL, "%s", "NULL pointer");
+  if (w < 8 || (w & 3) || band_halo(h, row0, row1, &in0, &in1))
+    return set_err(ctx, SHARP_EINVAL, "%s", "bad band geometry (multiples of 4, 0 <= row0 < row1 <= h)");
+  if ((long long)w * h >= (1ll << 29) || w > 65536 || h > 65536)
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "image larger than 2^29 pixels");
+  if (pp && !params_ok(*pp)) return set_err(ctx, SHARP_EINVAL, "%s", "parameter out of range or not finite");
+  Kind k;
+  int rc;
+  if ((rc = classify(ctx, band, &k))) return rc;
+  if (k != kDevice) return set_err(ctx, SHARP_EINVAL, "%s", "band calls take device pointers only");
+  if (mode == sharp::kStepPass2) {
+    if ((rc = classify(ctx, out, &k))) return rc;
+    if (k != kDevice) return set_err(ctx, SHARP_EINVAL, "%s", "band calls take device pointers only");
+    const uintptr_t a = (uintptr_t)band, b = (uintptr_t)out;
+    const size_t na = (size_t)(in1 - in0) * w, nb = (size_t)(row1 - row0) * w;
+    if (a < b + nb && b < a + na) return set_err(ctx, SHARP_EINVAL, "%s", "input and output overlap");
+  }
+  if (!ctx->use_tma || !sharp::tma_supported(band, mode == sharp::kStepPass2 ? out : (uint8_t *)band, w, h))
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
+                   "row bands need the TMA path (w % 16 == 0, 16-byte aligned band, 8-byte aligned out)");
+  sharp_params p;
+  if (pp) p = *pp;
+  else sharp_default_params(&p);
+  const sharp::Params prm{p.amount, p.gamma, p.osc_gain, p.osc_scale};
+  CK(cudaSetDevice(ctx->device));
+  if ((rc = ensure_frames(ctx, 1))) return rc;
+  if ((rc = ensure_task_counters(ctx, 1))) return rc;
+  sharp::BatchLaunch a;
+  a.in = band;
+  a.n = 1;
+  a.out = out;
+  a.acc = ctx->acc;
+  a.sums = ctx->sums;
+  a.means = ctx->means;
+  a.luts = ctx->luts;
+  a.lut_done = ctx->lut_done;
+  a.task_counter = ctx->tcounters;
+  a.partial = partial;
+  a.total = total;
+  if (mode == sharp::kStepPass1) {
+    CK(cudaMemsetAsync(ctx->acc, 0, sizeof(unsigned long long), ctx->stream));
+    CK(cudaMemsetAsync(ctx->tcounters, 0, sizeof(unsigned int), ctx->stream));
+  }
+  const double px = (double)(row1 - row0) * w;
+  CK(timed(ctx, ctx->stream, mode == sharp::kStepPass1 ? 1 : 2, px, [&] {
+    return sharp::launch_band_tma(a, mode, w, h, row0, row1, in0, in1 - in0, prm, ctx->stream);
+  }));
+  ctx->last_frames = 1;
+  ctx->stats.frames = 1;
+  ctx->stats.kernels = 2;
+  return SHARP_OK;
+}
+
 }  // namespace
 
 extern "C" {
+
+int sharp_band_halo(int h, int row0, int row1, int *in0, int *in1) {
+  if (!in0 || !in1) return SHARP_EINVAL;
+  return band_halo(h, row0, row1, in0, in1);
+}
+
+int sharp_band_edge_sum(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
+                        uint64_t *d_partial) {
+  return band_impl(ctx, sharp::kStepPass1, band, w, h, row0, row1, (unsigned long long *)d_partial, nullptr,
+                   nullptr, nullptr);
+}
+
+int sharp_band_sharpen(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
+                       const uint64_t *d_total, const sharp_params *params, uint8_t *out) {
+  return band_impl(ctx, sharp::kStepPass2, band, w, h, row0, row1, nullptr,
+                   (const unsigned long long *)d_total, params, out);
+}
 
 void sharp_default_params(sharp_params *p) {
   if (!p) return;
