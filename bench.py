@@ -17,6 +17,11 @@ over the whole batch.
   cpu_baseline: the CPU oracle timed on a bounded sample (rank 0, N=1).
 
 `--impl reference` times the CPU oracle (the reference arm of this tier).
+
+`--workload bands` (not the driver's default line) times BASELINE configs[3]:
+ONE --width x --height image (default 8K) row-band sharded over the N ranks
+(bands.py: halo exchange by NCCL send/recv, one u64 all-reduce of the pEdge
+partials, sharp_band_edge_sum / sharp_band_sharpen), bands device-resident.
 """
 import argparse
 import json
@@ -164,6 +169,107 @@ def workload_config(args, world):
             "l2": "batch (2.1 GB in + out) > 126 MB L2: no flush needed between steps"}
 
 
+def run_bands_workload(args, world, rank, local):
+    """One image, row bands over the ranks (BASELINE configs[3])."""
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_icpp_fanjzac15_b200 import Sharpener, shard
+    from paper_conf_icpp_fanjzac15_b200.bands import band_rows, exchange_halos, sharpen_band
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    W, H = args.width, args.height
+    r0, r1 = band_rows(H, world, rank)
+    img = synth.image(W, H, "natural", seed=synth.BASE_SEED + 3)  # every rank generates, keeps its rows
+    h_own = torch.from_numpy(img[r0:r1].copy()).pin_memory()
+    h_out = torch.empty_like(h_own).pin_memory()
+    own = h_own.to(f"cuda:{local}")
+    out = torch.empty_like(own)
+    # Rotate over enough input copies (>= 256 MB) that no step finds its
+    # input in the 126 MB L2 left by the previous steps.
+    ncopy = max(1, -(-(256 << 20) // own.numel()))
+    owns = [own] + [own.clone() for _ in range(ncopy - 1)]
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
+    sh = Sharpener(device=local)
+
+    def step(src, dst):
+        band = exchange_halos(src, H, r0, r1)
+        sharpen_band(sh, band, W, H, r0, r1, PARAMS, out=dst)
+
+    for _ in range(args.warmup):
+        step(own, out)
+    torch.cuda.synchronize()
+    sh.set_profiling(True)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    shard.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for i in range(args.steps):
+            step(owns[i % ncopy], out)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    shard.barrier()
+    ms_step = shard.max_over_ranks(ev0.elapsed_time(ev1) / args.steps, device=f"cuda:{local}")
+    kt = sh.kernel_times()
+    sh.set_profiling(False)
+    value = W * H / (ms_step * 1e-3) / 1e6
+    # dominant kernel: the band's pass-2 launch (reads its rows + halo, writes its rows)
+    k_avg = kt.pass2_ms / max(1, kt.pass2_launches)
+    px = kt.pixels / max(1, kt.pass2_launches)
+    pk, pk_src = peaks()
+    peak = float(pk["hbm_gbs"])
+    achieved = ALG_BYTES_PER_PX * px / (k_avg * 1e-3) / 1e9
+    parity = None
+    if rank == 0 and not args.no_cpu:
+        import oracle
+        ref, _, _ = oracle.sharpen(img, *PARAMS)
+        parity = {"rows_checked": r1 - r0, "mismatched_pixels": int((out.cpu().numpy() != ref[r0:r1]).sum())}
+    # e2e: this rank's rows from pinned host memory, result back to pinned host memory
+    t_e2e = []
+    for _ in range(max(args.e2e_steps, 0)):
+        shard.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        own.copy_(h_own, non_blocking=True)
+        step(own, out)
+        h_out.copy_(out, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        t_e2e.append(e0.elapsed_time(e1))
+    e2e_ms = shard.max_over_ranks(float(np.median(t_e2e)), device=f"cuda:{local}") if t_e2e else float("nan")
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"one {W}x{H} u8 image, row bands over {world} GPU(s) (BASELINE configs[3])",
+                       "width": W, "height": H, "bands": world,
+                       "parallelism": "row bands: 4-row halo exchange (NCCL send/recv) + u64 all-reduce",
+                       "l2": f"inputs rotated over {ncopy} copies (>= 256 MB > 126 MB L2)"},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": None, "kernel": "step_kernel (band pass 2)",
+                         "peak_source": pk_src, "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px,
+                         "kernel_avg_ms": k_avg, "pass1_avg_ms": kt.pass1_ms / max(1, kt.pass1_launches)},
+            "e2e": {"value": W * H / (e2e_ms * 1e-3) / 1e6, "unit": UNIT, "h2d_bytes_per_step": W * H,
+                    "d2h_bytes_per_step": W * H, "ms_per_step": e2e_ms,
+                    "api": "bands.sharpen_band (pinned host rows -> device -> pinned host)"},
+            "gpu_launches": 4 * args.steps,  # per band: step(pass 1) + finish + arm + step(pass 2)
+            "clocks": clk.summary(),
+            "cpu_baseline": None,
+            "parity": parity,
+        }
+        print(json.dumps(line), flush=True)
+    sh.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -177,10 +283,16 @@ def main():
     ap.add_argument("--cpu-sample", type=int, default=32)
     ap.add_argument("--ref-sample", type=int, default=16)
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--workload", default="batch", choices=["batch", "bands"])
     args = ap.parse_args()
     world, rank, local = dist_setup()
+    if args.workload == "bands" and args.width == 1920 and args.height == 1080:
+        args.width, args.height = 7680, 4320  # configs[3]: 8K
     if args.impl == "reference":
         run_reference(args, world, rank)
+        return
+    if args.workload == "bands":
+        run_bands_workload(args, world, rank, local)
         return
 
     import torch
