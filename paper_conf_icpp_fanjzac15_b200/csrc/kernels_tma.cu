@@ -47,6 +47,9 @@ using namespace dev;
 constexpr int kTW = 240;     // output columns per warp tile (lanes 0..29 x 8 px)
 constexpr int kTH = 12;      // output rows per warp tile
 constexpr int kCtasPerSm = 3;  // smem ~67 KB per CTA
+#ifndef SHARP_LB_CTAS
+#define SHARP_LB_CTAS kCtasPerSm
+#endif
 constexpr int kWarpsT = 4;   // compute warps = warp tiles per CTA tile
 constexpr int kCtaCols = kTW * kWarpsT;
 constexpr int kThreadsT = 32 * (kWarpsT + 1);  // + producer warp
@@ -69,8 +72,18 @@ constexpr int kBox1 = (kPitch + kPitchB) * kRows1;
 constexpr int kSlot = (kBox2 + 127) / 128 * 128;  // per-warp smem slot (128-B aligned)
 static_assert((kPitch * kRows1) % 128 == 0 && (kPitch * kRows2) % 128 == 0, "region B alignment");
 constexpr int kLutBytes = kLutSize * 8;
-constexpr int kStage = kWarpsT * kSlot + kLutBytes;
-constexpr int kSmem = 2 * kStage + 64;
+// A pass-2 task is kSub vertically adjacent CTA tiles ("sub-tiles") of one
+// frame: each sub-tile fills one stage, the frame's LUT is copied once per
+// task into one of two LUT buffers (task parity), and the warps carry their
+// row window, D rows and interpolation state from one sub-tile to the next.
+#ifndef SHARP_P2_SUB
+#define SHARP_P2_SUB 3
+#endif
+constexpr int kSub = SHARP_P2_SUB;
+constexpr int kStage = kWarpsT * kSlot;       // one stage: the 4 warp slots
+constexpr int kLutOff = 2 * kStage;           // two LUT buffers after the two stages
+constexpr int kBarOff = kLutOff + 2 * kLutBytes;
+constexpr int kSmem = kBarOff + 64;
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
 static_assert(kTH1 % 3 == 0 && kBox1 <= kSlot, "pass-1 tiles");
@@ -97,13 +110,13 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
-// Plain polling wait (no suspend-time hint).
+// Polling wait that never suspends the warp (test_wait is non-blocking).
 __device__ __forceinline__ void mbar_wait_spin(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n"
       ".reg .pred p;\n"
       "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%0], %1;\n"
       "@!p bra WAIT_%=;\n"
       "}\n" ::"r"(bar),
       "r"(parity)
@@ -459,10 +472,35 @@ __device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y)
                      __fmul_rn(2.0f, __fsub_rn(x.z, y.z)), __fmul_rn(2.0f, __fsub_rn(x.w, y.w)));
 }
 
-// out: first row of the output rows [row_lo, row_hi).
-__device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__restrict__ out, int W, int H,
-                                        int row_lo, int row_hi, int C0w, int R0, int lane) {
+// Stage ring shared by the producer and the consumers: stage s (a running
+// count) lives in buffer s & 1 and completes phase (s >> 1) & 1.
+struct Ring {
+  uint32_t sbase, full0, empty0;
+  __device__ __forceinline__ uint32_t stage(int s) const { return sbase + (uint32_t)((s & 1) * kStage); }
+  __device__ __forceinline__ void wait_full(int s) const {
+#ifdef SHARP_EXP_SPIN_WAIT
+    mbar_wait_spin(full0 + 8u * (s & 1), (uint32_t)((s >> 1) & 1));
+#else
+    mbar_wait(full0 + 8u * (s & 1), (uint32_t)((s >> 1) & 1));
+#endif
+  }
+  __device__ __forceinline__ void release(int s, int lane) const {  // one arrival per consumer warp
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty0 + 8u * (s & 1));
+  }
+};
+
+// Pass 2 of one warp over a task of nsub sub-tiles (stages s .. s+nsub-1,
+// the first already waited for).  out: first row of the output rows
+// [row_lo, row_hi).  Releases every stage it consumed.
+__device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint32_t lut, uint8_t *__restrict__ out,
+                                        int W, int H, int row_lo, int row_hi, int C0w, int R0, int warp,
+                                        int lane) {
 #ifdef SHARP_EXP_NO_P2  // timing experiment only
+  for (int k = 0; k < nsub; ++k) {
+    if (k) ring.wait_full(s + k);
+    ring.release(s + k, lane);
+  }
   return;
 #endif
   const int c0 = C0w + 8 * lane;
@@ -471,14 +509,14 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   // W-2,W-1 in the lane with c0 == W-8.
   const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
-  const LaneRow aw = lane_row(tile, kRows2, lane);
+  LaneRow aw = lane_row(ring.stage(s) + warp * kSlot, kRows2, lane);
   const uint64_t pol_out = policy_evict_first();  // output: written once, never re-read
-  // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (kept
-  // opaque so the compiler emits one IMAD instead of folding the constant).
-  // (a shuffle hides the value from ptxas, which would otherwise split the
-  // constant back out into one extra IADD per pixel)
+  // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (a
+  // shuffle hides the value from ptxas, which would otherwise split the
+  // constant back out into one extra IADD per pixel).
   const uint32_t lut_q = __shfl_sync(0xffffffffu, lut - (0x4B000000u << 3), 0);
-  // smem row of global row R0-4 is 0: row r -> smem row r - R0 + 4.
+  // In a sub-tile starting at row R0k, smem row of global row R0k-4 is 0:
+  // row r -> smem row r - R0k + 4.
   // Vertical interpolation (L146, R3) of D rows (i, i+1) is linear in r on
   // r = 4i+2 .. 4i+5: V(r+1) = V(r) + 2 (D_{i+1} - D_i), restarted at
   // r = 4i+2 with V = 7 D_i + D_{i+1} (all exact integers, x 128).
@@ -490,30 +528,39 @@ __device__ __forceinline__ void p2_warp(uint32_t tile, uint32_t lut, uint8_t *__
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
   uint8_t *orow = out + (size_t)(R0 - row_lo) * W + c0;
-  const int rend = min(R0 + kTH, row_hi);
-  const int rend_l = active ? rend : R0;  // this lane stores rows < rend_l
 #pragma unroll 1
-  for (int r = R0; r < rend; r += 3) {
-    // 3 rows per iteration: the window rotation has period 3, so the
-    // unrolled body needs no register moves.
-#pragma unroll
-    for (int u = 0; u < 3; ++u) {
-      const int rr = r + u;
-      const int sm = rr - R0 + 4;
-      if ((rr & 3) == 0 && rr != R0) {  // next D block row
-        D0 = D1;
-        D1 = dblock(aw, sm + 4, lane);
-      } else if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
-        V = f4fma(7.0f, D0, D1);
-        slope = f4twice_diff(D1, D0);
-      }
-      const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
-      p2_row(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
-      V = f4add(V, slope);
-      orow += W;
-      ra = rb;
-      rb = rc;
+  for (int k = 0; k < nsub; ++k) {
+    const int R0k = R0 + k * kTH;
+    if (k) {  // next sub-tile: same rows layout in the next stage; state carried
+      ring.wait_full(s + k);
+      aw = lane_row(ring.stage(s + k) + warp * kSlot, kRows2, lane);
     }
+    const int rend = min(R0k + kTH, row_hi);
+    const int rend_l = active ? rend : R0k;  // this lane stores rows < rend_l
+#pragma unroll 1
+    for (int r = R0k; r < rend; r += 3) {
+      // 3 rows per iteration: the window rotation has period 3, so the
+      // unrolled body needs no register moves.
+#pragma unroll
+      for (int u = 0; u < 3; ++u) {
+        const int rr = r + u;
+        const int sm = rr - R0k + 4;
+        if ((rr & 3) == 0 && rr != R0) {  // next D block row
+          D0 = D1;
+          D1 = dblock(aw, sm + 4, lane);
+        } else if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
+          V = f4fma(7.0f, D0, D1);
+          slope = f4twice_diff(D1, D0);
+        }
+        const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
+        p2_row(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
+        V = f4add(V, slope);
+        orow += W;
+        ra = rb;
+        rb = rc;
+      }
+    }
+    ring.release(s + k, lane);
   }
 }
 
@@ -559,23 +606,29 @@ __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int C0
   return sum;
 }
 
+#ifdef SHARP_EXP_WAITSTAT  // timing experiment: consumer full-barrier wait cycles by (previous, awaited) task type
+__device__ unsigned long long g_waitstat[40][2];
+__shared__ long long stage_t[2];  // producer: clock64 at issue
+#endif
 // ============================================================== the kernel
-__global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
+__global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     step_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
                 const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, StepParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ int4 stage_task[2];                 // {type, frame, C0, R0} (LUT tasks: {type, frame, q, 0})
+  __shared__ int2 stage_aux[2];                  // pass 2: {sub-tiles of the task, LUT buffer}
   __shared__ unsigned long long stage_sum[2];    // LUT tasks: the frame's S
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t sbase = smem_u32(smem);
-  const uint32_t full0 = sbase + 2 * kStage, empty0 = full0 + 16;
+  const Ring ring{sbase, sbase + kBarOff, sbase + kBarOff + 16};
+  const uint32_t lutbase = sbase + kLutOff;
   const Geo &g = sp.g;
 
   if (threadIdx.x == 0) {
-    mbar_init(full0, 1);
-    mbar_init(full0 + 8, 1);
-    mbar_init(empty0, kWarpsT);
-    mbar_init(empty0 + 8, kWarpsT);
+    mbar_init(ring.full0, 1);
+    mbar_init(ring.full0 + 8, 1);
+    mbar_init(ring.empty0, kWarpsT);
+    mbar_init(ring.empty0 + 8, kWarpsT);
     fence_barrier_init();
   }
   __syncthreads();
@@ -586,10 +639,9 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     const unsigned long long arrivals = (unsigned long long)(g.per_frame1 * kWarpsT) << kAccShift;
     const uint64_t pol_keep = policy_evict_last(), pol_drop = policy_evict_first();
     int t_next = (int)atomicAdd(sp.task_counter, 1u);
-    for (int i = 0;; ++i) {
-      const int b = i & 1;
+    for (int s = 0, j = 0;; ++j) {  // s: stages filled, j: tasks (LUT buffer parity)
       const int4 d = decode(sp, t_next);
-      // Resolve the task's dependency first (before waiting for the stage).
+      // Resolve the task's dependency first (before waiting for a stage).
       unsigned long long S = 0;
       if (d.x == kLut) {
         // every pass-1 warp of the frame has added its partial (the global
@@ -601,55 +653,91 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
         fence_acquire();
         fence_proxy_async_global();
       }
-      if (i >= 2) mbar_wait(empty0 + 8u * b, (uint32_t)(((i >> 1) - 1) & 1));
-      // Grab the following task now: the atomic's latency overlaps this
-      // task's loads and the next empty-wait.
-      if (d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
-      const uint32_t full = full0 + 8u * b, st = sbase + (uint32_t)(b * kStage);
+      int C0 = 0, R0 = 0, nsub = 1, nw = 0;
       if (d.x == kP1 || d.x == kP2) {
-        int C0, R0;
-        tile_xy(g, d.z, d.x == kP1 ? kTH1 : kTH, C0, R0);
-        stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
-        int nw = 0;
+        tile_xy(g, d.z, d.x == kP1 ? kTH1 : kTH * kSub, C0, R0);
+        if (d.x == kP2) nsub = min(kSub, (g.row_hi - R0 + kTH - 1) / kTH);
 #pragma unroll
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
+      }
+      for (int k = 0; k < nsub; ++k, ++s) {
+        const int b = s & 1;
+        if (s >= 2) mbar_wait(ring.empty0 + 8u * b, (uint32_t)(((s >> 1) - 1) & 1));
+        // Grab the following task now: the atomic's latency overlaps this
+        // task's loads and the next empty-wait.
+        if (k == 0 && d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
+        const uint32_t full = ring.full0 + 8u * b, st = ring.stage(s);
+#ifdef SHARP_EXP_WAITSTAT
+        stage_t[b] = clock64();
+#endif
         if (d.x == kP1) {
+          stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
           mbar_expect_tx(full, (uint32_t)(nw * kBox1));
           for (int w = 0; w < nw; ++w)
             tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1 - g.y0, kRows1, d.y, full, pol_keep);
-        } else {
-#ifdef SHARP_EXP_NO_LUT  // timing experiment only (stale LUTs)
-          mbar_expect_tx(full, (uint32_t)(nw * kBox2));
-#else
-          mbar_expect_tx(full, (uint32_t)(nw * kBox2 + kLutBytes));
-#endif
+        } else if (d.x == kP2) {
+          const int R0k = R0 + k * kTH;
+          stage_task[b] = make_int4(d.x, d.y, C0, R0k);
+          stage_aux[b] = make_int2(nsub, j & 1);
+          const uint32_t lut_bytes = k == 0 ? (uint32_t)kLutBytes : 0u;
+          mbar_expect_tx(full, (uint32_t)(nw * kBox2) + lut_bytes);
           for (int w = 0; w < nw; ++w)
-            tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0 - 4 - g.y0, kRows2, d.y, full, pol_drop);
-#ifndef SHARP_EXP_NO_LUT
-          bulk_copy(st + kWarpsT * kSlot, sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
-#endif
+            tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0k - 4 - g.y0, kRows2, d.y, full, pol_drop);
+          if (lut_bytes)
+            bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
+        } else {
+          stage_task[b] = d;
+          if (d.x == kLut) stage_sum[b] = S & ((1ull << kAccShift) - 1);
+          mbar_arrive(full);  // no data: LUT, empty or end task
         }
-      } else {
-        stage_task[b] = d;
-        if (d.x == kLut) stage_sum[b] = S & ((1ull << kAccShift) - 1);
-        mbar_arrive(full);  // no data: LUT, empty or end task
-        if (d.x == kEnd) break;
       }
+      if (d.x == kEnd) break;
     }
     return;
   }
 
   // -------------------------------------------------------------- consumers
-  for (int i = 0;; ++i) {
-    const int b = i & 1;
-#ifdef SHARP_EXP_SPIN_WAIT
-    mbar_wait_spin(full0 + 8u * b, (uint32_t)((i >> 1) & 1));
-#else
-    mbar_wait(full0 + 8u * b, (uint32_t)((i >> 1) & 1));
+#ifdef SHARP_EXP_WAITSTAT
+  int prev_type = 0;
+  const long long t_begin = clock64();
 #endif
+  for (int s = 0;;) {
+    const int b = s & 1;
+#ifdef SHARP_EXP_WAITSTAT
+    const long long tw0 = clock64();
+#endif
+    ring.wait_full(s);
     const int4 d = stage_task[b];
+#ifdef SHARP_EXP_WAITSTAT
+    if (lane == 0) {
+      const int cur = d.x < 0 ? 4 : d.x;
+      atomicAdd(&g_waitstat[prev_type * 5 + cur][0], (unsigned long long)(clock64() - tw0));
+      atomicAdd(&g_waitstat[prev_type * 5 + cur][1], 1ull);
+      prev_type = cur;
+      const long long now = clock64();
+      if (warp == 0 && now - tw0 > 200) {  // waited: the load completed ~now
+        atomicAdd(&g_waitstat[26 + cur][0], (unsigned long long)(now - stage_t[b]));
+        atomicAdd(&g_waitstat[26 + cur][1], 1ull);
+      }
+      if (d.x == kEnd) atomicAdd(&g_waitstat[25][0], (unsigned long long)(clock64() - t_begin));
+    }
+#endif
     if (d.x == kEnd) break;
-    const uint32_t st = sbase + (uint32_t)(b * kStage);
+    if (d.x == kP2) {
+      const int2 aux = stage_aux[b];
+      const int C0 = d.z, R0 = d.w, C0w = C0 + warp * kTW;
+      if (C0w < g.W) {
+        p2_warp(ring, s, aux.x, lutbase + (uint32_t)(aux.y * kLutBytes), sp.out + (size_t)d.y * g.W * g.H, g.W, g.H,
+                g.row_lo, g.row_hi, C0w, R0, warp, lane);
+      } else {  // no columns for this warp: follow the stages
+        for (int k = 0; k < aux.x; ++k) {
+          if (k) ring.wait_full(s + k);
+          ring.release(s + k, lane);
+        }
+      }
+      s += aux.x;
+      continue;
+    }
     if (d.x == kLut) {
       // LUT task: entries q*128 .. q*128+127 of frame f (R9, R11; f64, one rounding)
       const int f = d.y, p = d.z * kLutPerTask + threadIdx.x;
@@ -673,22 +761,16 @@ __global__ void __launch_bounds__(kThreadsT, kCtasPerSm)
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
-      const float acc = (C0w < g.W) ? p1_warp(st + warp * kSlot, g.W, g.rmax1, C0w, R0, lane) : 0.0f;
+      const float acc = (C0w < g.W) ? p1_warp(ring.stage(s) + warp * kSlot, g.W, g.rmax1, C0w, R0, lane) : 0.0f;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
       // atomic per warp adding (1 << 40) + partial: the frame's arrival count
       // and sum in one word, so its LUT tasks can tell when S is complete
       // without any fence.
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
       if (lane == 0) atomicAdd(&sp.acc[d.y], (1ull << kAccShift) + (unsigned long long)ws);
-    } else if (d.x == kP2) {
-      const int C0 = d.z, R0 = d.w;
-      const int C0w = C0 + warp * kTW;
-      if (C0w < g.W)
-        p2_warp(st + warp * kSlot, st + kWarpsT * kSlot, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H, g.row_lo,
-                g.row_hi, C0w, R0, lane);
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty0 + 8u * b);  // stage b may be refilled
+    ring.release(s, lane);  // stage s may be refilled
+    ++s;
   }
 }
 
@@ -729,6 +811,18 @@ int num_sms() {
 }
 
 }  // namespace
+
+#ifdef SHARP_EXP_WAITSTAT
+extern "C" int sharp_debug_waitstat(unsigned long long *out, int reset) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(out, g_waitstat, sizeof(g_waitstat));
+  if (reset) {
+    static unsigned long long z[40][2] = {};
+    cudaMemcpyToSymbol(g_waitstat, z, sizeof(z));
+  }
+  return 0;
+}
+#endif
 
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
   return (W % 16) == 0 && (((uintptr_t)imgs) & 15) == 0 && (((uintptr_t)outs) & 7) == 0 && H >= 8 &&
@@ -775,7 +869,7 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.g.rmax1 = std::min(H - 2, sg.row_hi - 1);
   const int rows = sg.row_hi - sg.row_lo;
   sp.g.tiles_x = (W + kCtaCols - 1) / kCtaCols;
-  sp.g.per_frame = sp.g.tiles_x * ((rows + kTH - 1) / kTH);
+  sp.g.per_frame = sp.g.tiles_x * ((rows + kTH * kSub - 1) / (kTH * kSub));
   sp.g.per_frame1 = sp.g.tiles_x * ((rows + kTH1 - 1) / kTH1);
   sp.mode = mode;
   sp.n = sg.n;
