@@ -166,6 +166,27 @@ __device__ __forceinline__ uint32_t sharpen_px(float adj, float osc, float E, fl
   return cvt_u8(F);
 }
 
+// Round half to even, saturate to [0, 255] and pack four values into one
+// word (bytes a, b, c, d from low to high).  cvt.rni.s32 + cvt.pack.sat.u8
+// is the same function as cvt.rni.sat.u8.f32 (R14); ptxas fuses each pair
+// into one two-source F2IP.U8 (4 pixels in 2 instructions instead of 4 F2IP
+// + 3 PRMT).
+__device__ __forceinline__ uint32_t pack4_rni_u8(float a, float b, float c, float d) {
+  uint32_t r;
+  asm("{\n"
+      ".reg .b32 t0, t1, t2, t3, lo;\n"
+      "cvt.rni.s32.f32 t2, %3;\n"
+      "cvt.rni.s32.f32 t3, %4;\n"
+      "cvt.pack.sat.u8.s32.b32 lo, t3, t2, 0;\n"
+      "cvt.rni.s32.f32 t0, %1;\n"
+      "cvt.rni.s32.f32 t1, %2;\n"
+      "cvt.pack.sat.u8.s32.b32 %0, t1, t0, lo;\n"
+      "}"
+      : "=r"(r)
+      : "f"(a), "f"(b), "f"(c), "f"(d));
+  return r;
+}
+
 // Packs 8 bytes (low byte of each word) into two words.
 __device__ __forceinline__ uint2 pack8(const uint32_t o[8]) {
   const uint32_t a = prmt(prmt(o[0], o[1], 0x0040), prmt(o[2], o[3], 0x0040), 0x5410);

@@ -86,7 +86,7 @@ constexpr int kBarOff = kLutOff + 2 * kLutBytes;
 constexpr int kSmem = kBarOff + 64;
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
-static_assert(kTH1 % 3 == 0 && kBox1 <= kSlot, "pass-1 tiles");
+static_assert(kTH1 % 6 == 0 && kBox1 <= kSlot, "pass-1 tiles (6-row unrolled interior loop)");
 static_assert(kLutSize % kLutPerTask == 0, "LUT tasks");
 
 // ------------------------------------------------------------ TMA / mbarrier
@@ -408,6 +408,7 @@ __device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t 
   }
 }
 
+template <bool kRingRows>
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
                                        const float4 &D0, const float4 &D1, uint32_t lut_q,
                                        uint8_t *orow, uint64_t pol_out, bool store, int r, int c0, int W, int H,
@@ -428,7 +429,7 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   const float2 nu45 = lin2(V.y, V.z, cwt(0), cwt(1));
   const float2 nu67 = lin2(V.z, V.w, cwt(2), cwt(3));
   float NU[8] = {nu01.x, nu01.y, nu23.x, nu23.y, nu45.x, nu45.y, nu67.x, nu67.y};
-  if (r < 2 || r >= H - 2) {  // warp-uniform
+  if (kRingRows && (r < 2 || r >= H - 2)) {  // warp-uniform
     ring_rows(NU, pe, MX, MN, D0, D1, r, c0, W, H, edge);
   } else if (edge_warp) {     // warp-uniform; only the edge lane changes
     ring_cols(NU, pe, MX, MN, D0, D1, r, H, edge);
@@ -447,14 +448,16 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
     T8[x] = fminf(fmaxf(P[x], mnf), mxf);  // Fig. 8 branch target (max / min / P)
     osc[x] = L.y;
   }
-  uint32_t o[8];
+  float F[8];
 #pragma unroll
   for (int x = 0; x < 8; x += 2) {
     const float2 d = sub2(make_float2(P[x], P[x + 1]), make_float2(T8[x], T8[x + 1]));
-    o[x] = cvt_u8(__fmaf_rn(osc[x], d.x, T8[x]));  // osc max / osc min / P, clamp, RNE
-    o[x + 1] = cvt_u8(__fmaf_rn(osc[x + 1], d.y, T8[x + 1]));
+    F[x] = __fmaf_rn(osc[x], d.x, T8[x]);  // osc max / osc min / P
+    F[x + 1] = __fmaf_rn(osc[x + 1], d.y, T8[x + 1]);
   }
-  if (store) st_stream_u64(orow, pack8(o), pol_out);
+  // clamp to [0, 255], RNE, pack (R14)
+  const uint2 o = make_uint2(pack4_rni_u8(F[0], F[1], F[2], F[3]), pack4_rni_u8(F[4], F[5], F[6], F[7]));
+  if (store) st_stream_u64(orow, o, pol_out);
 }
 
 __device__ __forceinline__ float4 f4fma(float a, const float4 &x, const float4 &y) {  // a*x + y, exact here
@@ -493,6 +496,9 @@ struct Ring {
 // Pass 2 of one warp over a task of nsub sub-tiles (stages s .. s+nsub-1,
 // the first already waited for).  out: first row of the output rows
 // [row_lo, row_hi).  Releases every stage it consumed.
+// (Measured: a fully unrolled 12-row interior body -- no per-row phase or
+// ring tests -- is 40% SLOWER: ~36 KB of straight-line code overflows the
+// instruction cache.  The hot loops must stay small.)
 __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint32_t lut, uint8_t *__restrict__ out,
                                         int W, int H, int row_lo, int row_hi, int C0w, int R0, int warp,
                                         int lane) {
@@ -520,11 +526,14 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   // Vertical interpolation (L146, R3) of D rows (i, i+1) is linear in r on
   // r = 4i+2 .. 4i+5: V(r+1) = V(r) + 2 (D_{i+1} - D_i), restarted at
   // r = 4i+2 with V = 7 D_i + D_{i+1} (all exact integers, x 128).
-  const float4 Dp = dblock(aw, 0, lane);  // D row k0-1
-  float4 D0 = dblock(aw, 4, lane);        // D row r>>2
-  float4 D1 = dblock(aw, 8, lane);        // D row (r>>2)+1
-  float4 V = f4fma(5.0f, D0, f4fma(3.0f, Dp, make_float4(0.f, 0.f, 0.f, 0.f)));  // r = R0 (a' = 0): (3,5)
-  float4 slope = f4twice_diff(D0, Dp);
+  // State on entry to a sub-tile (rows R0k.., R0k % 4 == 0): D1 = D row
+  // R0k/4 (the row-R0k update shifts it into D0 and loads the next), V and
+  // slope of row R0k (a' = 0 of the interval (R0k/4 - 1, R0k/4): (3,5)).
+  const float4 Dp = dblock(aw, 0, lane);  // D row R0/4 - 1
+  float4 D1 = dblock(aw, 4, lane);        // D row R0/4
+  float4 D0 = Dp;
+  float4 V = f4fma(5.0f, D1, f4fma(3.0f, Dp, make_float4(0.f, 0.f, 0.f, 0.f)));
+  float4 slope = f4twice_diff(D1, Dp);
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
   uint8_t *orow = out + (size_t)(R0 - row_lo) * W + c0;
@@ -545,7 +554,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
       for (int u = 0; u < 3; ++u) {
         const int rr = r + u;
         const int sm = rr - R0k + 4;
-        if ((rr & 3) == 0 && rr != R0) {  // next D block row
+        if ((rr & 3) == 0) {  // next D block row
           D0 = D1;
           D1 = dblock(aw, sm + 4, lane);
         } else if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
@@ -553,7 +562,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
           slope = f4twice_diff(D1, D0);
         }
         const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
-        p2_row(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
+        p2_row<true>(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
         V = f4add(V, slope);
         orow += W;
         ra = rb;
@@ -565,6 +574,10 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 }
 
 // ========================================================== pass 1 (warp)
+// (Measured: a separate row-test-free loop for interior tiles, with or
+// without pairwise f16 row sums, is no faster -- pass 1 waits on its TMA
+// loads more than on issue -- and the 6-row variant's extra code is 5%
+// slower.)
 __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int C0w, int R0, int lane) {
 #ifdef SHARP_EXP_NO_P1  // timing experiment only
   return 0.0f;
@@ -874,7 +887,10 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.mode = mode;
   sp.n = sg.n;
   sp.per_round = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
-  const int grid = kCtasPerSm * num_sms();
+#ifndef SHARP_GRID_CTAS
+#define SHARP_GRID_CTAS kCtasPerSm
+#endif
+  const int grid = SHARP_GRID_CTAS * num_sms();
   if (mode == kStepPass1) {
     sp.L1 = sp.L2 = 0;
     sp.ntasks = sp.g.per_frame1;
