@@ -121,6 +121,33 @@ def traffic_per_launch(px_per_launch):
         return None
 
 
+def issue_profile():
+    """Warp instructions per output pixel of the dominant kernel, from the
+    committed ncu capture (profiles/<round>/traffic.json), or None."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "traffic.json")))
+    try:
+        return float(json.load(open(files[-1]))["warp_instr_per_px"]) if files else None
+    except Exception:
+        return None
+
+
+def issue_roofline(px_per_launch, k_avg_ms, sm_mhz, n_sms):
+    """The binding resource: instruction issue.  Peak =
+    4 warp-instructions per clock per SM (one per SMSP scheduler) at the SM
+    clock measured during the timed region; achieved = the committed
+    capture's warp-instructions per pixel x pixels per launch / the live
+    launch duration."""
+    wipp = issue_profile()
+    if wipp is None or not sm_mhz:
+        return None
+    achieved = wipp * px_per_launch / (k_avg_ms * 1e-3) / 1e9
+    peak = 4.0 * n_sms * sm_mhz * 1e6 / 1e9
+    return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gwarp-instr/s", "frac": achieved / peak,
+            "warp_instr_per_px": wipp, "thread_instr_per_px": 32 * wipp,
+            "peak_source": f"4 issue slots/clk/SM x {n_sms} SMs x measured SM clock (B200_PROFILING / B300_MICROARCH)"}
+
+
 def cpu_oracle_rate(frames, threads):
     """Oracle Mpix/s on `frames` ([k,H,W]) with `threads` OpenMP threads."""
     import oracle
@@ -280,7 +307,7 @@ def main():
     ap.add_argument("--width", type=int, default=1920)
     ap.add_argument("--height", type=int, default=1080)
     ap.add_argument("--e2e-steps", type=int, default=5)
-    ap.add_argument("--cpu-sample", type=int, default=32)
+    ap.add_argument("--cpu-sample", type=int, default=128)
     ap.add_argument("--ref-sample", type=int, default=16)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--workload", default="batch", choices=["batch", "bands"])
@@ -412,6 +439,8 @@ def main():
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": total_px,
                     "d2h_bytes_per_step": total_px, "ms_per_step": e2e_ms,
                     "api": "sharp_run_batch(pinned host in, pinned host out)"},
+            "issue_roofline": issue_roofline(px_per_launch, k_avg_ms, clk.summary().get("sm_mhz"),
+                                             torch.cuda.get_device_properties(local).multi_processor_count),
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clk.summary(),
             "cpu_baseline": cpu,

@@ -17,7 +17,11 @@ KEYS = [
     "dram__bytes_write.sum",
     "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed",
     "sm__throughput.avg.pct_of_peak_sustained_elapsed",
-    "sm__inst_executed.sum",
+    "smsp__inst_executed.sum",
+    "sm__inst_executed.sum.per_cycle_elapsed",
+    "smsp__issue_active.avg.pct_of_peak_sustained_active",
+    "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+    "sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active",
     "smsp__inst_executed.avg.per_cycle_active",
     "sm__warps_active.avg.pct_of_peak_sustained_active",
     "lts__t_sector_hit_rate.pct",
@@ -71,8 +75,28 @@ def main():
         for v, k in stalls:
             lines.append(f"| {k.replace('smsp__pcsamp_warps_issue_stalled_', '')} | {int(v)} | {v / tot:.1%} |")
         lines.append("")
-        summary.append({"kernel": name, "dram_read_bytes": rd, "dram_write_bytes": wr,
-                        "pixels_per_launch": px, "dram_bytes_per_px": (rd + wr) / px})
+        ent = {"kernel": name, "dram_read_bytes": rd, "dram_write_bytes": wr,
+               "pixels_per_launch": px, "dram_bytes_per_px": (rd + wr) / px}
+        # issue-rate evidence (the kernel is instruction-issue bound)
+        for k, key in [("smsp__inst_executed.sum", "warp_instr"), ("gpu__time_duration.sum", "duration"),
+                       ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue_active_pct"),
+                       ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "fma_pipe_pct"),
+                       ("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active", "alu_pipe_pct")]:
+            if k in rec and rec[k][0]:
+                v = num(rec[k][0])
+                if key == "warp_instr":
+                    v *= {"inst": 1, "Kinst": 1e3, "Minst": 1e6, "Ginst": 1e9}.get(rec[k][1], 1)
+                    ent["warp_instr_per_px"] = v / px
+                    ent["thread_instr_per_px"] = 32 * v / px
+                elif key == "duration":
+                    v *= {"ns": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3, "msecond": 1e-3, "s": 1}.get(rec[k][1], 1e-9)
+                    ent["duration_s"] = v
+                else:
+                    ent[key] = v
+        if "warp_instr_per_px" in ent:
+            lines += [f"instructions: {ent['thread_instr_per_px']:.2f} thread-instr per output pixel "
+                      f"({ent['warp_instr_per_px']:.4f} warp-instr/px)", ""]
+        summary.append(ent)
     if len(sys.argv) > 4:
         lines += ["## launch list (ncu gpu__time_duration, cold-cache, serialised)", "", "```"]
         lines += open(sys.argv[4]).read().strip().splitlines()[-12:]
