@@ -297,6 +297,96 @@ def run_bands_workload(args, world, rank, local):
         dist.destroy_process_group()
 
 
+# Compulsory HBM bytes per output pixel of the staged base design (every
+# stage materialised): K1 1 + 1/4, K3 1/4 + 4, K4 1 + 2,
+# K5 2, K6 2 + 8, K7 1 + 4 + 8 + 1.
+STAGED_BYTES_PER_PX = {"downscale": 1.25, "border": 0.0, "center": 4.25, "sobel": 3.0, "reduction": 2.0,
+                       "strength": 10.0, "sharpness": 14.0}
+
+
+def run_ladder_workload(args, world, rank, local):
+    """The optimisation ladder (sec. V, Fig. 12 / Fig. 14) on
+    BASELINE configs[2] (4K frames, "kernel-fusion roofline study"): the
+    paper's staged base design (one kernel per stage, Fig. 13 breakdown), the
+    two-pass fused kernels and the one-launch step kernel, each timed on the
+    same device-resident batch (> L2), all bit-identical."""
+    import torch
+
+    import synth
+    from paper_conf_icpp_fanjzac15_b200 import (SHARP_PATH_STAGED, SHARP_PATH_STEP, SHARP_PATH_TWO_PASS,
+                                                Sharpener)
+
+    if world > 1:
+        if rank == 0:
+            print(json.dumps({"workload": "ladder", "skipped": "single-GPU study"}))
+        return
+    torch.cuda.set_device(local)
+    W, H, n = args.width, args.height, args.frames
+    imgs = synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 2)
+    d_in = torch.from_numpy(imgs).cuda()
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
+    pk, pk_src = peaks()
+    peak = float(pk["hbm_gbs"])
+    rungs, outs = [], {}
+    for name, path in [("staged (paper base: 7 kernels, all stages in HBM)", SHARP_PATH_STAGED),
+                       ("two-pass fused (edge_sum + sharpen per chunk)", SHARP_PATH_TWO_PASS),
+                       ("step kernel (one persistent TMA launch)", SHARP_PATH_STEP)]:
+        sh = Sharpener(device=local)
+        sh.set_stream(stream)
+        sh.set_path(path)
+        d_out = torch.empty_like(d_in)
+        for _ in range(args.warmup):
+            sh.enqueue_batch(d_in, d_out, PARAMS)
+        torch.cuda.synchronize()
+        sh.set_profiling(True)
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for _ in range(args.steps):
+            sh.enqueue_batch(d_in, d_out, PARAMS)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        ms = ev0.elapsed_time(ev1) / args.steps
+        rung = {"path": name, "ms_per_step": ms, "mpix_s": n * W * H / (ms * 1e-3) / 1e6,
+                "launches_per_step": sh.stats().kernels}
+        if path == SHARP_PATH_STAGED:
+            st = sh.stage_times()
+            tot = sum(st.values()) or 1.0
+            rung["stages"] = {k: {"ms_per_frame": v / (args.steps * n), "share": v / tot,
+                                  "alg_bytes_per_px": STAGED_BYTES_PER_PX[k],
+                                  "achieved_gbs": (STAGED_BYTES_PER_PX[k] * W * H / (v / (args.steps * n) * 1e-3)
+                                                   / 1e9) if v > 0 and STAGED_BYTES_PER_PX[k] else None}
+                              for k, v in st.items()}
+            rung["alg_bytes_per_px"] = sum(STAGED_BYTES_PER_PX.values())
+        else:
+            kt = sh.kernel_times()
+            if path == SHARP_PATH_TWO_PASS:
+                rung["pass1_share"] = kt.pass1_ms / max(1e-9, kt.pass1_ms + kt.pass2_ms)
+            rung["alg_bytes_per_px"] = 3.0 if path == SHARP_PATH_TWO_PASS else ALG_BYTES_PER_PX
+        rung["hbm_frac_alg2"] = ALG_BYTES_PER_PX * n * W * H / (ms * 1e-3) / 1e9 / peak
+        sh.set_profiling(False)
+        outs[path] = d_out
+        rungs.append(rung)
+        sh.close()
+    identical = bool(torch.equal(outs[SHARP_PATH_STAGED], outs[SHARP_PATH_STEP]) and
+                     torch.equal(outs[SHARP_PATH_TWO_PASS], outs[SHARP_PATH_STEP]))
+    parity = None
+    if not args.no_cpu:
+        import oracle
+        ref, _ = oracle.sharpen_batch(imgs[:1], *PARAMS)
+        parity = {"frames_checked": 1, "mismatched_pixels": int((outs[SHARP_PATH_STEP][:1].cpu().numpy() != ref).sum())}
+    base = rungs[0]["ms_per_step"]
+    for r in rungs:
+        r["speedup_vs_staged"] = base / r["ms_per_step"]
+    line = {"metric": METRIC, "workload": "ladder", "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{n} x {W}x{H} u8 frames (BASELINE configs[2]: kernel-fusion roofline study)",
+                       "l2": f"batch {2 * n * W * H / 1e6:.0f} MB in + out > 126 MB L2"},
+            "hbm_peak_gbs": peak, "peak_source": pk_src, "ladder": rungs, "paths_identical": identical,
+            "parity": parity}
+    print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -310,7 +400,7 @@ def main():
     ap.add_argument("--cpu-sample", type=int, default=128)
     ap.add_argument("--ref-sample", type=int, default=16)
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--workload", default="batch", choices=["batch", "bands"])
+    ap.add_argument("--workload", default="batch", choices=["batch", "bands", "ladder"])
     args = ap.parse_args()
     world, rank, local = dist_setup()
     if args.workload == "bands" and args.width == 1920 and args.height == 1080:
@@ -320,6 +410,13 @@ def main():
         return
     if args.workload == "bands":
         run_bands_workload(args, world, rank, local)
+        return
+    if args.workload == "ladder":
+        if args.width == 1920 and args.height == 1080:
+            args.width, args.height = 3840, 2160  # configs[2]: 4K
+        if args.frames == 1024:
+            args.frames = 32
+        run_ladder_workload(args, world, rank, local)
         return
 
     import torch

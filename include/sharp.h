@@ -165,6 +165,39 @@ int sharp_set_profiling(sharp_ctx *ctx, int enable);
 /* Waits for the launch stream, then returns the accumulated times. */
 int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
 
+/* ---- Kernel paths: the optimisation ladder of PAPER.md sec. V (Fig. 12,
+ * Fig. 14), every rung bit-identical to the oracle.
+ *   SHARP_PATH_AUTO     the step kernel where it applies, else the two-pass path (default)
+ *   SHARP_PATH_STEP     one persistent TMA-staged launch per batch (kernels_tma.cu): pass 1,
+ *                       per-frame LUT and pass 2 as dynamically scheduled tasks with
+ *                       in-kernel dependencies; needs w % 16 == 0, 16-byte aligned input,
+ *                       8-byte aligned output, w*h <= 2^29, else SHARP_EUNSUPPORTED
+ *   SHARP_PATH_TWO_PASS two fused kernels per chunk of frames (kernels.cu): Sobel +
+ *                       reduction + LUT, then everything else; any w % 4 == 0
+ *   SHARP_PATH_STAGED   the paper's BASE GPU design (sec. IV): one kernel per
+ *                       stage, every intermediate matrix in HBM (kernels_staged.cu,
+ *                       7 launches per frame); the per-stage breakdown of Fig. 13
+ * Takes effect at the next call.  Row-band calls need AUTO or STEP.  Environment
+ * SHARP_FORCE_GENERIC=1 at sharp_create selects SHARP_PATH_TWO_PASS. */
+enum { SHARP_PATH_AUTO = 0, SHARP_PATH_STEP = 1, SHARP_PATH_TWO_PASS = 2, SHARP_PATH_STAGED = 3 };
+int sharp_set_path(sharp_ctx *ctx, int path);
+int sharp_get_path(const sharp_ctx *ctx);
+
+/* Staged path + profiling: device ms per stage (CUDA events around each
+ * launch, summed since sharp_set_profiling(ctx, 1)); ms[SHARP_NUM_STAGES]
+ * in the order below (sec. III / Fig. 13).  Waits for the events. */
+enum {
+  SHARP_STAGE_DOWNSCALE = 0, /* K1  O -> D (L130)                         */
+  SHARP_STAGE_BORDER,        /* K2  D -> U ring, steps i-vii (L140-L142)  */
+  SHARP_STAGE_CENTER,        /* K3  D -> U body (L146)                    */
+  SHARP_STAGE_SOBEL,         /* K4  O -> pEdge (L158-L172)                */
+  SHARP_STAGE_REDUCE,        /* K5  pEdge -> S (L174)                     */
+  SHARP_STAGE_STRENGTH,      /* K6  pEdge, S -> adj, osc per pixel (L178) */
+  SHARP_STAGE_SHARPEN,       /* K7  O, U, adj, osc -> out (L178-L212)     */
+  SHARP_NUM_STAGES
+};
+int sharp_get_stage_times(sharp_ctx *ctx, float *ms, int n);
+
 /* Static strings. */
 const char *sharp_strerror(int code);
 const char *sharp_last_error(const sharp_ctx *ctx);

@@ -42,4 +42,12 @@ from .binding import (  # noqa: F401
     sharp_band_halo,
     sharp_band_edge_sum,
     sharp_band_sharpen,
+    sharp_set_path,
+    sharp_get_path,
+    sharp_get_stage_times,
+    SHARP_PATH_AUTO,
+    SHARP_PATH_STEP,
+    SHARP_PATH_TWO_PASS,
+    SHARP_PATH_STAGED,
+    STAGE_NAMES,
 )

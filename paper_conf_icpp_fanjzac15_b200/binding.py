@@ -18,6 +18,13 @@ SHARP_ENCCL = -4
 SHARP_EUNSUPPORTED = -5
 SHARP_ESTATE = -6
 LUT_SIZE = 1536
+# kernel paths (sharp_set_path) and stages (sharp_get_stage_times), include/sharp.h
+SHARP_PATH_AUTO = 0
+SHARP_PATH_STEP = 1
+SHARP_PATH_TWO_PASS = 2
+SHARP_PATH_STAGED = 3
+STAGE_NAMES = ("downscale", "border", "center", "sobel", "reduction", "strength", "sharpness")
+SHARP_NUM_STAGES = len(STAGE_NAMES)
 
 
 class SharpParams(ctypes.Structure):
@@ -63,6 +70,9 @@ _SIGS = {
     "sharp_band_halo": ([_I, _I, _I, ctypes.POINTER(_I), ctypes.POINTER(_I)], _I),
     "sharp_band_edge_sum": ([_P, _P, _I, _I, _I, _I, _P], _I),
     "sharp_band_sharpen": ([_P, _P, _I, _I, _I, _I, _P, ctypes.POINTER(SharpParams), _P], _I),
+    "sharp_set_path": ([_P, _I], _I),
+    "sharp_get_path": ([_P], _I),
+    "sharp_get_stage_times": ([_P, ctypes.POINTER(ctypes.c_float), _I], _I),
 }
 
 _lib = None
@@ -202,6 +212,21 @@ def sharp_get_kernel_times(ctx):
     return t
 
 
+def sharp_set_path(ctx, path):
+    return _check(lib().sharp_set_path(ctx, int(path)), ctx)
+
+
+def sharp_get_path(ctx):
+    return lib().sharp_get_path(ctx)
+
+
+def sharp_get_stage_times(ctx):
+    """-> dict stage name -> summed device ms (staged path, profiling on)."""
+    arr = (ctypes.c_float * SHARP_NUM_STAGES)()
+    _check(lib().sharp_get_stage_times(ctx, arr, SHARP_NUM_STAGES), ctx)
+    return dict(zip(STAGE_NAMES, list(arr)))
+
+
 def sharp_strerror(code):
     return lib().sharp_strerror(code).decode()
 
@@ -273,6 +298,12 @@ class Sharpener:
 
     def set_stream(self, stream):
         sharp_set_stream(self.ctx, stream)
+
+    def set_path(self, path):
+        sharp_set_path(self.ctx, path)
+
+    def stage_times(self):
+        return sharp_get_stage_times(self.ctx)
 
     def run(self, img, params=None, out=None):
         H, W = self._shape(img)

@@ -57,6 +57,30 @@ enum StepMode { kStepAll = 0, kStepPass1 = 1, kStepPass2 = 2 };
 cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int row_lo, int row_hi, int y0, int rows_in,
                             const Params &p, cudaStream_t stream);
 
+// The paper's base design (kernels_staged.cu): one kernel per stage, every
+// intermediate in HBM (the "base GPU" of sec. IV; first rung of the ladder).
+enum Stage {
+  kStageDownscale = 0, kStageBorder, kStageCenter, kStageSobel, kStageReduce, kStageStrength, kStageSharpen,
+  kNumStages
+};
+// Optional per-stage event hook (profiling): begin(stage) / end(stage).
+struct StageTimer {
+  void *ctx = nullptr;
+  void (*rec)(void *ctx, int stage, int begin, cudaStream_t st) = nullptr;
+  void begin(int s, cudaStream_t st) const {
+    if (rec) rec(ctx, s, 1, st);
+  }
+  void end(int s, cudaStream_t st) const {
+    if (rec) rec(ctx, s, 0, st);
+  }
+};
+size_t staged_scratch_bytes(int W, int H);
+// One frame through K1..K7; *sum (u64) and *mean receive S and S / (W H).
+cudaError_t launch_staged(const uint8_t *in, int W, int H, const Params &p, void *scratch,
+                          unsigned long long *sum, double *mean, uint8_t *out, cudaStream_t st,
+                          const StageTimer &timer);
+constexpr int kStagedLaunches = 7;
+
 // Kernel launches issued per (pass-1, pass-2) chunk.
 constexpr int kLaunchesPerChunk = 2;
 

@@ -42,7 +42,10 @@ struct sharp_ctx {
   cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
   int nslots = 3;
   int chunk_cfg = 0;
-  bool use_tma = true;  // SHARP_FORCE_GENERIC=1 at sharp_create selects the LDG kernels
+  int path = SHARP_PATH_AUTO;  // SHARP_FORCE_GENERIC=1 at sharp_create selects SHARP_PATH_TWO_PASS
+  void *staged = nullptr;      // SHARP_PATH_STAGED scratch (D, U, pEdge, strength of one frame)
+  size_t staged_cap = 0;
+  cudaEvent_t stage_open[sharp::kNumStages] = {};
   Slot slots[kMaxSlots];
   size_t slot_chunk_frames = 0, slot_stage_bytes = 0;  // capacity of the slot buffers
   unsigned long long *sums = nullptr;
@@ -55,7 +58,8 @@ struct sharp_ctx {
   float2 *luts = nullptr;             // per frame lookup tables (batch kernel)
   int last_frames = 0;
   sharp_stats stats{};
-  // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2)
+  // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2,
+  // 3 = step kernel, 10 + s = stage s of the staged path)
   bool profiling = false;
   struct Rec { cudaEvent_t a, b; int kind; double px; };
   std::vector<Rec> recs;
@@ -249,6 +253,36 @@ cudaError_t timed(sharp_ctx *ctx, cudaStream_t st, int kind, double px, F launch
   return e;
 }
 
+// Staged-path scratch for one w x h frame (grown on demand).
+int rc_staged(sharp_ctx *ctx, int w, int h) {
+  const size_t need = sharp::staged_scratch_bytes(w, h);
+  if (need <= ctx->staged_cap) return SHARP_OK;
+  cudaStreamSynchronize(ctx->stream);
+  cudaFree(ctx->staged);
+  ctx->staged = nullptr;
+  ctx->staged_cap = 0;
+  if (cudaMalloc(&ctx->staged, need) != cudaSuccess) {
+    cudaGetLastError();
+    return SHARP_ENOMEM;
+  }
+  ctx->staged_cap = need;
+  return SHARP_OK;
+}
+
+// StageTimer hook: an event pair per stage launch (profiling only).
+void stage_rec(void *vctx, int stage, int begin, cudaStream_t st) {
+  sharp_ctx *ctx = static_cast<sharp_ctx *>(vctx);
+  cudaEvent_t e = pool_event(ctx);
+  if (!e) return;
+  cudaEventRecord(e, st);
+  if (begin) {
+    ctx->stage_open[stage] = e;
+  } else if (ctx->stage_open[stage]) {
+    ctx->recs.push_back({ctx->stage_open[stage], e, 10 + stage, 0.0});
+    ctx->stage_open[stage] = nullptr;
+  }
+}
+
 // Device-resident batch on one stream, in chunks of frames.
 //  * TMA path: launch c = pass 1 of chunk c + pass 2 of chunk c-1 (one
 //    dynamically scheduled step kernel); chunk c's input is still in L2 when
@@ -260,7 +294,25 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
                    unsigned int *tc) {
   const size_t fb = (size_t)w * h;
   const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
-  const bool tma = ctx->use_tma && sharp::tma_supported(din, dout, w, h);
+  if (ctx->path == SHARP_PATH_STAGED) {  // the paper's base design: K1..K7 per frame
+    if ((rc_staged(ctx, w, h))) return SHARP_ENOMEM;
+    sharp::StageTimer tm;
+    if (ctx->profiling) {
+      tm.ctx = ctx;
+      tm.rec = stage_rec;
+    }
+    for (int f = 0; f < n; ++f) {
+      CK(sharp::launch_staged(din + (size_t)f * fb, w, h, prm, ctx->staged, ctx->sums + frame_base + f,
+                              ctx->means + frame_base + f, dout + (size_t)f * fb, st, tm));
+      *launches += sharp::kStagedLaunches;
+    }
+    return SHARP_OK;
+  }
+  const bool tma_ok = sharp::tma_supported(din, dout, w, h);
+  if (ctx->path == SHARP_PATH_STEP && !tma_ok)
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
+                   "SHARP_PATH_STEP needs w % 16 == 0, 16-byte aligned input, 8-byte aligned output, w*h <= 2^29");
+  const bool tma = (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) && tma_ok;
   if (tma) {  // the whole batch in one persistent launch
     sharp::BatchLaunch a;
     a.in = din;
@@ -420,7 +472,8 @@ int band_impl(sharp_ctx *ctx, int mode, const uint8_t *band, int w, int h, int r
     const size_t na = (size_t)(in1 - in0) * w, nb = (size_t)(row1 - row0) * w;
     if (a < b + nb && b < a + na) return set_err(ctx, SHARP_EINVAL, "%s", "input and output overlap");
   }
-  if (!ctx->use_tma || !sharp::tma_supported(band, mode == sharp::kStepPass2 ? out : (uint8_t *)band, w, h))
+  if (!(ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) ||
+      !sharp::tma_supported(band, mode == sharp::kStepPass2 ? out : (uint8_t *)band, w, h))
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
                    "row bands need the TMA path (w % 16 == 0, 16-byte aligned band, 8-byte aligned out)");
   sharp_params p;
@@ -507,7 +560,7 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
   ctx->device = dev;
   {
     const char *g = getenv("SHARP_FORCE_GENERIC");
-    ctx->use_tma = !(g && g[0] == '1');
+    ctx->path = (g && g[0] == '1') ? SHARP_PATH_TWO_PASS : SHARP_PATH_AUTO;
   }
   ctx->nslots = c.streams ? c.streams : 3;
   ctx->chunk_cfg = c.chunk_frames;
@@ -555,6 +608,7 @@ void sharp_destroy(sharp_ctx *ctx) {
   cudaFree(ctx->acc);
   cudaFree(ctx->luts);
   cudaFree(ctx->tcounters);
+  cudaFree(ctx->staged);
   for (auto &r : ctx->recs) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -632,7 +686,7 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t) {
       t->pass2_ms += ms;
       t->pass2_launches++;
       t->pixels += r.px;
-    } else {
+    } else if (r.kind == 3) {
       t->step_ms += ms;
       t->step_launches++;
       t->pixels += r.px;
@@ -640,6 +694,29 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t) {
   }
   return SHARP_OK;
 }
+
+int sharp_get_stage_times(sharp_ctx *ctx, float *ms, int n) {
+  if (!ctx || !ms || n < SHARP_NUM_STAGES) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  for (int i = 0; i < SHARP_NUM_STAGES; ++i) ms[i] = 0.0f;
+  for (auto &r : ctx->recs) {
+    if (r.kind < 10 || r.kind >= 10 + SHARP_NUM_STAGES) continue;
+    CK(cudaEventSynchronize(r.b));
+    float t = 0.0f;
+    CK(cudaEventElapsedTime(&t, r.a, r.b));
+    ms[r.kind - 10] += t;
+  }
+  return SHARP_OK;
+}
+
+int sharp_set_path(sharp_ctx *ctx, int path) {
+  if (!ctx || path < SHARP_PATH_AUTO || path > SHARP_PATH_STAGED) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  ctx->path = path;
+  return SHARP_OK;
+}
+
+int sharp_get_path(const sharp_ctx *ctx) { return ctx ? ctx->path : SHARP_EINVAL; }
 
 const char *sharp_strerror(int code) {
   switch (code) {

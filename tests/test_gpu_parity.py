@@ -10,7 +10,8 @@ import torch
 
 import oracle
 import synth
-from paper_conf_icpp_fanjzac15_b200 import SHARP_EINVAL, SharpError, Sharpener
+from paper_conf_icpp_fanjzac15_b200 import (SHARP_EINVAL, SHARP_EUNSUPPORTED, SHARP_PATH_STAGED, SHARP_PATH_STEP,
+                                            SHARP_PATH_TWO_PASS, STAGE_NAMES, SharpError, Sharpener)
 
 pytestmark = pytest.mark.gpu
 
@@ -26,15 +27,18 @@ PARAMS = [
 ]
 
 
-@pytest.fixture(scope="module", params=["auto", "generic"])
+@pytest.fixture(scope="module", params=["auto", "generic", "staged"])
 def sh(request):
     """A context on the automatic kernel path (TMA-staged persistent kernels
-    when W % 16 == 0) and one forced onto the generic LDG kernels."""
+    when W % 16 == 0), one forced onto the generic two-pass LDG kernels, and
+    one on the paper's staged base design (one kernel per stage)."""
     assert torch.cuda.is_available(), "GPU tests need a CUDA device"
     import os
     old = os.environ.get("SHARP_FORCE_GENERIC")
     os.environ["SHARP_FORCE_GENERIC"] = "1" if request.param == "generic" else "0"
     s = Sharpener()
+    if request.param == "staged":
+        s.set_path(SHARP_PATH_STAGED)
     if old is None:
         del os.environ["SHARP_FORCE_GENERIC"]
     else:
@@ -211,3 +215,34 @@ def test_invalid_params_and_overlap_rejected(sh):
     with pytest.raises(SharpError) as e:
         sh.run(big[0], DEFAULT, big[0])  # in place
     assert e.value.code == SHARP_EINVAL
+
+
+def test_ladder_paths_identical_and_stage_times():
+    """The optimisation ladder (staged base -> two-pass fused -> step kernel)
+    gives the same bytes; the staged path reports a time for every stage."""
+    imgs = synth.frames(2, 3840, 2160, "natural", seed=synth.BASE_SEED + 2)
+    ref, ref_sums = oracle.sharpen_batch(imgs, *DEFAULT)
+    d = torch.from_numpy(imgs).cuda()
+    for path in [SHARP_PATH_STAGED, SHARP_PATH_TWO_PASS, SHARP_PATH_STEP]:
+        with Sharpener() as s:
+            s.set_path(path)
+            s.set_profiling(True)
+            o = torch.empty_like(d)
+            s.run_batch(d, DEFAULT, o)
+            np.testing.assert_array_equal(o.cpu().numpy(), ref)
+            assert s.batch_sums(2) == [int(x) for x in ref_sums]
+            if path == SHARP_PATH_STAGED:
+                t = s.stage_times()
+                assert list(t) == list(STAGE_NAMES)
+                assert all(v > 0 for v in t.values()), t
+                assert s.stats().kernels == 2 * 7
+
+
+def test_step_path_rejects_unsupported_geometry():
+    with Sharpener() as s:
+        s.set_path(SHARP_PATH_STEP)
+        d = torch.zeros((16, 20), dtype=torch.uint8, device="cuda")  # W % 16 != 0
+        o = torch.empty_like(d)
+        with pytest.raises(SharpError) as e:
+            s.run(d, DEFAULT, o)
+        assert e.value.code == SHARP_EUNSUPPORTED
