@@ -222,10 +222,23 @@ def run_bands_workload(args, world, rank, local):
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
     sh = Sharpener(device=local)
+    sh.set_stream(stream)
+    if args.exchange == "p2p":
+        # fused peer-memory exchange: halos and the u64 partials stored
+        # straight into the neighbours' / all ranks' windows (CUDA IPC over
+        # NVLink), epoch-flagged; no NCCL on the data path
+        from paper_conf_icpp_fanjzac15_b200.bands import P2PBand
+        p2p = P2PBand(sh, W, H)
+        epoch = [0]
 
-    def step(src, dst):
-        band = exchange_halos(src, H, r0, r1)
-        sharpen_band(sh, band, W, H, r0, r1, PARAMS, out=dst)
+        def step(src, dst):
+            p2p.own.copy_(src)  # this image's rows into the window (the NCCL path copies them too)
+            epoch[0] += 1
+            p2p.step(epoch[0], dst, PARAMS)
+    else:
+        def step(src, dst):
+            band = exchange_halos(src, H, r0, r1)
+            sharpen_band(sh, band, W, H, r0, r1, PARAMS, out=dst)
 
     for _ in range(args.warmup):
         step(own, out)
@@ -276,8 +289,11 @@ def run_bands_workload(args, world, rank, local):
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": f"one {W}x{H} u8 image, row bands over {world} GPU(s) (BASELINE configs[3])",
-                       "width": W, "height": H, "bands": world,
-                       "parallelism": "row bands: 4-row halo exchange (NCCL send/recv) + u64 all-reduce",
+                       "width": W, "height": H, "bands": world, "exchange": args.exchange,
+                       "parallelism": ("row bands: 4-row halo exchange (NCCL send/recv) + u64 all-reduce"
+                                       if args.exchange == "nccl" else
+                                       "row bands: halo rows + u64 partials stored into peer windows "
+                                       "(CUDA IPC / NVLink, epoch flags), no NCCL on the data path"),
                        "l2": f"inputs rotated over {ncopy} copies (>= 256 MB > 126 MB L2)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": None, "kernel": "step_kernel (band pass 2)",
@@ -286,7 +302,8 @@ def run_bands_workload(args, world, rank, local):
             "e2e": {"value": W * H / (e2e_ms * 1e-3) / 1e6, "unit": UNIT, "h2d_bytes_per_step": W * H,
                     "d2h_bytes_per_step": W * H, "ms_per_step": e2e_ms,
                     "api": "bands.sharpen_band (pinned host rows -> device -> pinned host)"},
-            "gpu_launches": 4 * args.steps,  # per band: step(pass 1) + finish + arm + step(pass 2)
+            # per band: [halo] + step(pass 1) + finish + [all-reduce] + arm + step(pass 2)
+            "gpu_launches": (6 if args.exchange == "p2p" else 4) * args.steps,
             "clocks": clk.summary(),
             "cpu_baseline": None,
             "parity": parity,
@@ -401,6 +418,8 @@ def main():
     ap.add_argument("--ref-sample", type=int, default=16)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--workload", default="batch", choices=["batch", "bands", "ladder"])
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
+                    help="bands workload: NCCL send/recv + all-reduce, or the fused peer-memory exchange")
     args = ap.parse_args()
     world, rank, local = dist_setup()
     if args.workload == "bands" and args.width == 1920 and args.height == 1080:

@@ -149,6 +149,51 @@ int sharp_band_edge_sum(sharp_ctx *ctx, const uint8_t *band, int w, int h, int r
 int sharp_band_sharpen(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
                        const uint64_t *d_total, const sharp_params *params, uint8_t *out);
 
+/* ---- Fused peer-memory band exchange (
+ * DESIGN.md sec. 9): the same two couplings as above -- 4 halo rows per side
+ * and the 64-bit pEdge sum -- moved by direct stores into the neighbours' /
+ * every rank's memory (NVLink peer mappings from CUDA IPC) with epoch flags,
+ * instead of NCCL: one single-CTA kernel per exchange, no host round trip.
+ *
+ * Each rank owns a zero-initialised device "window" of
+ * sharp_p2p_window_bytes(w, rows_own) bytes (16-byte aligned):
+ *   [0, SHARP_P2P_CTL_BYTES)  control words (flags, partial slots; library-owned)
+ *   then rows of pitch w: 4 halo rows | the band's rows_own own rows | 4 halo rows.
+ * The caller writes its own rows at offset SHARP_P2P_CTL_BYTES + 4*w; after
+ * sharp_band_p2p_halo the window rows [in0 - (row0 - 4), ...) are exactly the
+ * band input of sharp_band_edge_sum / sharp_band_sharpen (for the first band
+ * skip the upper halo rows, for the last the lower ones).
+ * sharp_band_p2p_halo: pushes this band's first/last 4 own rows into the
+ *   neighbours' halos (up_window / down_window: their windows as mapped on
+ *   this device, NULL at the image edges; up_rows_own: the upper band's own
+ *   rows), publishes them with `epoch`, and returns (asynchronously) when
+ *   both neighbours' rows for `epoch` have arrived in ours.
+ * sharp_band_p2p_allreduce: stores (epoch, *d_partial) into slot `rank` of
+ *   every window (windows: HOST array of the n_ranks windows as mapped on this
+ *   device, windows[rank] = ours), waits for all n_ranks slots of ours and
+ *   writes their sum to *d_total (device u64).
+ * Every rank must make the same sequence of calls with epochs 1, 2, 3, ...
+ * (one per image); w % 16 == 0, rows_own >= 4, n_ranks <= 32; both calls are
+ * asynchronous on the context's stream and wait on the device for the peers.
+ * sharp_ipc_*: thin wrappers of cudaIpcGetMemHandle / cudaIpcOpenMemHandle
+ * (lazy peer access) / cudaIpcCloseMemHandle for exchanging the windows
+ * between processes (handles are SHARP_IPC_HANDLE_BYTES opaque bytes). */
+#define SHARP_P2P_CTL_BYTES 1024
+#define SHARP_IPC_HANDLE_BYTES 64
+size_t sharp_p2p_window_bytes(int w, int rows_own); /* 0 on bad arguments */
+/* cudaMalloc + zero of one window on the current device (its own allocation,
+ * so an IPC handle of it maps exactly the window); the caller owns it and
+ * releases it with sharp_p2p_window_destroy (after closing peer mappings). */
+int sharp_p2p_window_create(int w, int rows_own, void **d_window);
+void sharp_p2p_window_destroy(void *d_window);
+int sharp_band_p2p_halo(sharp_ctx *ctx, uint8_t *self_window, int w, int rows_own, uint8_t *up_window,
+                        int up_rows_own, uint8_t *down_window, uint64_t epoch);
+int sharp_band_p2p_allreduce(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank,
+                             const uint64_t *d_partial, uint64_t epoch, uint64_t *d_total);
+int sharp_ipc_get_handle(const void *d_ptr, void *handle);
+int sharp_ipc_open_handle(const void *handle, void **d_ptr);
+int sharp_ipc_close_handle(void *d_ptr);
+
 /* Per-kernel device time accounting (CUDA events around every launch, on
  * the launch stream).  enable != 0 starts (and resets) accounting. */
 typedef struct {

@@ -43,6 +43,15 @@ from .binding import (  # noqa: F401
     sharp_band_edge_sum,
     sharp_band_sharpen,
     sharp_set_path,
+    sharp_p2p_window_bytes,
+    sharp_p2p_window_create,
+    sharp_p2p_window_destroy,
+    sharp_band_p2p_halo,
+    sharp_band_p2p_allreduce,
+    sharp_ipc_get_handle,
+    sharp_ipc_open_handle,
+    sharp_ipc_close_handle,
+    SHARP_P2P_CTL_BYTES,
     sharp_get_path,
     sharp_get_stage_times,
     SHARP_PATH_AUTO,

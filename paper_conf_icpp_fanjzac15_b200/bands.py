@@ -102,3 +102,89 @@ def sharpen_band(sharpener, band, w, h, row0, row1, params=None, out=None, group
         dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)  # the L174 reduction across bands
     sharpener.band_sharpen(band, w, h, row0, row1, s, out, params)
     return out, s
+
+
+# ---------------------------------------------------------------------------
+# Fused peer-memory exchange:
+# the halo rows and the u64 pEdge partials move by direct stores into the
+# neighbours' / every rank's window (NVLink peer mappings via CUDA IPC) with
+# epoch flags -- libsharp.so's sharp_band_p2p_halo / sharp_band_p2p_allreduce
+# -- instead of NCCL send/recv + all-reduce.  torch.distributed only carries
+# the one-time exchange of the IPC handles.
+
+def _device_view(addr, nbytes, device):
+    """A torch uint8 tensor aliasing device memory [addr, addr + nbytes)."""
+    class _Mem:
+        __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (addr, False), "version": 3}
+    return torch.as_tensor(_Mem(), device=device)
+
+
+class P2PBand:
+    """This rank's band of a w x h image and its exchange window.
+
+    Multi-process (one GPU per rank): P2PBand(sharpener, w, h, group) --
+    windows are exchanged once as CUDA IPC handles over `group`.
+    Single-process (tests, several bands on one device): pass `windows`, the
+    list of every band's window address, and `rank`.
+    Use: write this band's rows into `own` ([rows, w] uint8 view), then
+    step(epoch, out, params) with epochs 1, 2, 3, ... (the same on every rank)."""
+
+    def __init__(self, sharpener, w, h, group=None, rank=None, world=None, window=None, windows=None):
+        from . import binding as B
+        self.B, self.sh, self.w, self.h = B, sharpener, w, h
+        if world is None:
+            world, rank = _world(group)
+        self.world, self.rank = world, rank
+        self.rows = [band_rows(h, world, g) for g in range(world)]
+        self.row0, self.row1 = self.rows[rank]
+        self.rows_own = self.row1 - self.row0
+        if w % 16 or self.rows_own < HALO:
+            raise ValueError("P2P bands need w % 16 == 0 and >= 4 rows per band")
+        self.nbytes = B.sharp_p2p_window_bytes(w, self.rows_own)
+        self._owned = window is None
+        self.window = window if window is not None else B.sharp_p2p_window_create(w, self.rows_own)
+        self._opened = []
+        if windows is None:  # multi-process: exchange IPC handles once
+            if world > 1:
+                handles = [None] * world
+                dist.all_gather_object(handles, B.sharp_ipc_get_handle(self.window), group=group)
+                windows = []
+                for g, hnd in enumerate(handles):
+                    if g == rank:
+                        windows.append(self.window)
+                    else:
+                        p = B.sharp_ipc_open_handle(hnd)
+                        self._opened.append(p)
+                        windows.append(p)
+            else:
+                windows = [self.window]
+        self.windows = list(windows)
+        dev = torch.device("cuda", torch.cuda.current_device())
+        base = self.window + B.SHARP_P2P_CTL_BYTES
+        self.own = _device_view(base + HALO * w, self.rows_own * w, dev).view(self.rows_own, w)
+        in0, in1 = halo_rows(h, self.row0, self.row1)
+        first = base + (in0 - (self.row0 - HALO)) * w
+        self.band = _device_view(first, (in1 - in0) * w, dev).view(in1 - in0, w)
+        self.partial = torch.zeros(1, dtype=torch.int64, device=dev)
+        self.total = torch.zeros(1, dtype=torch.int64, device=dev)
+
+    def step(self, epoch, out, params=None):
+        """Halo push + pass 1 + peer all-reduce + pass 2 of image `epoch`, on
+        the sharpener's stream.  out: [rows, w] uint8 CUDA tensor."""
+        B, g = self.B, self.rank
+        up = self.windows[g - 1] if g > 0 else None
+        dn = self.windows[g + 1] if g < self.world - 1 else None
+        up_rows = self.rows[g - 1][1] - self.rows[g - 1][0] if g > 0 else 0
+        B.sharp_band_p2p_halo(self.sh.ctx, self.window, self.w, self.rows_own, up, up_rows, dn, epoch)
+        self.sh.band_edge_sum(self.band, self.w, self.h, self.row0, self.row1, self.partial)
+        B.sharp_band_p2p_allreduce(self.sh.ctx, self.windows, g, self.partial, epoch, self.total)
+        self.sh.band_sharpen(self.band, self.w, self.h, self.row0, self.row1, self.total, out, params)
+        return out
+
+    def close(self):
+        for p in self._opened:
+            self.B.sharp_ipc_close_handle(p)
+        self._opened = []
+        if self._owned and self.window:
+            self.B.sharp_p2p_window_destroy(self.window)
+        self.window = 0

@@ -70,6 +70,14 @@ _SIGS = {
     "sharp_band_halo": ([_I, _I, _I, ctypes.POINTER(_I), ctypes.POINTER(_I)], _I),
     "sharp_band_edge_sum": ([_P, _P, _I, _I, _I, _I, _P], _I),
     "sharp_band_sharpen": ([_P, _P, _I, _I, _I, _I, _P, ctypes.POINTER(SharpParams), _P], _I),
+    "sharp_p2p_window_bytes": ([_I, _I], ctypes.c_size_t),
+    "sharp_p2p_window_create": ([_I, _I, ctypes.POINTER(_P)], _I),
+    "sharp_p2p_window_destroy": ([_P], None),
+    "sharp_band_p2p_halo": ([_P, _P, _I, _I, _P, _I, _P, ctypes.c_uint64], _I),
+    "sharp_band_p2p_allreduce": ([_P, ctypes.POINTER(_P), _I, _I, _P, ctypes.c_uint64, _P], _I),
+    "sharp_ipc_get_handle": ([_P, _P], _I),
+    "sharp_ipc_open_handle": ([_P, ctypes.POINTER(_P)], _I),
+    "sharp_ipc_close_handle": ([_P], _I),
     "sharp_set_path": ([_P, _I], _I),
     "sharp_get_path": ([_P], _I),
     "sharp_get_stage_times": ([_P, ctypes.POINTER(ctypes.c_float), _I], _I),
@@ -210,6 +218,63 @@ def sharp_get_kernel_times(ctx):
     t = SharpKernelTimes()
     _check(lib().sharp_get_kernel_times(ctx, ctypes.byref(t)), ctx)
     return t
+
+
+SHARP_P2P_CTL_BYTES = 1024
+SHARP_IPC_HANDLE_BYTES = 64
+
+
+def sharp_p2p_window_bytes(w, rows_own):
+    return int(lib().sharp_p2p_window_bytes(w, rows_own))
+
+
+def sharp_p2p_window_create(w, rows_own):
+    """-> device address (int) of a zeroed window (caller owns it)."""
+    p = _P()
+    rc = lib().sharp_p2p_window_create(w, rows_own, ctypes.byref(p))
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_p2p_window_create: {sharp_strerror(rc)}")
+    return p.value
+
+
+def sharp_p2p_window_destroy(d_window):
+    lib().sharp_p2p_window_destroy(d_window)
+
+
+def sharp_band_p2p_halo(ctx, self_window, w, rows_own, up_window, up_rows_own, down_window, epoch):
+    return _check(lib().sharp_band_p2p_halo(ctx, self_window, w, rows_own, up_window or None, up_rows_own,
+                                            down_window or None, int(epoch)), ctx)
+
+
+def sharp_band_p2p_allreduce(ctx, windows, rank, d_partial, epoch, d_total):
+    arr = (_P * len(windows))(*windows)
+    return _check(lib().sharp_band_p2p_allreduce(ctx, arr, len(windows), rank, _addr(d_partial), int(epoch),
+                                                 _addr(d_total)), ctx)
+
+
+def sharp_ipc_get_handle(d_ptr):
+    """-> bytes (SHARP_IPC_HANDLE_BYTES) naming the allocation of d_ptr."""
+    buf = ctypes.create_string_buffer(SHARP_IPC_HANDLE_BYTES)
+    rc = lib().sharp_ipc_get_handle(d_ptr, buf)
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_ipc_get_handle: {sharp_strerror(rc)}")
+    return buf.raw
+
+
+def sharp_ipc_open_handle(handle):
+    """-> device address (int) of a peer allocation mapped on this device."""
+    buf = ctypes.create_string_buffer(bytes(handle), SHARP_IPC_HANDLE_BYTES)
+    p = _P()
+    rc = lib().sharp_ipc_open_handle(buf, ctypes.byref(p))
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_ipc_open_handle: {sharp_strerror(rc)}")
+    return p.value
+
+
+def sharp_ipc_close_handle(d_ptr):
+    rc = lib().sharp_ipc_close_handle(d_ptr)
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_ipc_close_handle: {sharp_strerror(rc)}")
 
 
 def sharp_set_path(ctx, path):

@@ -332,4 +332,13 @@ cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float
   return cudaGetLastError();
 }
 
+// Forces the (lazy) module load of this file's kernels; see kernels.h.
+cudaError_t preload_two_pass() {
+  cudaFuncAttributes a;
+  cudaError_t e;
+  if ((e = cudaFuncGetAttributes(&a, edge_sum_kernel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, sharpen_kernel)) != cudaSuccess) return e;
+  return cudaSuccess;
+}
+
 }  // namespace sharp

@@ -81,6 +81,24 @@ cudaError_t launch_staged(const uint8_t *in, int W, int H, const Params &p, void
                           const StageTimer &timer);
 constexpr int kStagedLaunches = 7;
 
+// Fused peer-memory band exchange (bands_p2p.cu).
+constexpr int kP2PCtlBytes = 1024;
+constexpr int kP2PHalo = 4;
+size_t p2p_window_bytes(int w, int rows_own);
+cudaError_t launch_p2p_halo(uint8_t *self, int w, int rows_own, uint8_t *up, int up_rows_own, uint8_t *down,
+                            unsigned long long epoch, cudaStream_t st);
+cudaError_t launch_p2p_allreduce(uint8_t *const *windows, int G, int rank, const unsigned long long *partial,
+                                 unsigned long long epoch, unsigned long long *total, cudaStream_t st);
+
+// Under CUDA lazy module loading a kernel's module is loaded at its first
+// launch, and that load can wait for the device to go idle -- a deadlock when
+// an already running kernel spins on work the host has not launched yet (the
+// peer-memory band exchange).  sharp_create loads every kernel up front.
+cudaError_t preload_two_pass();
+cudaError_t preload_staged();
+cudaError_t preload_step();
+cudaError_t preload_p2p();
+
 // Kernel launches issued per (pass-1, pass-2) chunk.
 constexpr int kLaunchesPerChunk = 2;
 

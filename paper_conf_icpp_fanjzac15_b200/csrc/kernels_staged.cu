@@ -222,4 +222,18 @@ cudaError_t launch_staged(const uint8_t *in, int W, int H, const Params &p, void
   return cudaGetLastError();
 }
 
+// Forces the (lazy) module load of this file's kernels; see kernels.h.
+cudaError_t preload_staged() {
+  cudaFuncAttributes a;
+  cudaError_t e;
+  if ((e = cudaFuncGetAttributes(&a, st_downscale)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, st_border)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, st_center)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, st_sobel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, st_reduce)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, st_strength)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, st_sharpen)) != cudaSuccess) return e;
+  return cudaSuccess;
+}
+
 }  // namespace sharp

@@ -86,7 +86,7 @@ constexpr int kBarOff = kLutOff + 2 * kLutBytes;
 constexpr int kSmem = kBarOff + 64;
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
-static_assert(kTH1 % 6 == 0 && kBox1 <= kSlot, "pass-1 tiles (6-row unrolled interior loop)");
+static_assert(kTH1 % 3 == 0 && kBox1 <= kSlot, "pass-1 tiles (3-row loop)");
 static_assert(kLutSize % kLutPerTask == 0, "LUT tasks");
 
 // ------------------------------------------------------------ TMA / mbarrier
@@ -213,8 +213,10 @@ __device__ __forceinline__ float2 sub2(float2 a, float2 b) {
 struct Geo {
   int W, H;        // the whole image (ring rows, Sobel frame, mean denominator)
   int tiles_x;     // CTA tiles per row band (ceil(W / 960))
-  int per_frame;   // pass-2 CTA tiles per frame (kTH rows)
-  int per_frame1;  // pass-1 CTA tiles per frame (kTH1 rows)
+  int per_frame;   // pass-2 tasks per frame (sub sub-tiles of kTH rows each)
+  int sub;         // sub-tiles per pass-2 task (kSub; 1 when a launch has too few tasks to fill the GPU)
+  int per_frame1;  // pass-1 CTA tiles per frame (th1 rows)
+  int th1;         // pass-1 rows per tile: kTH1, or 9 / 6 / 3 when a launch has too few tiles
   // Rows processed: [row_lo, row_hi) of the image (the whole image, or one
   // row band, sec. 8(e)); the tensor map's row 0 is image row y0 (a band's
   // buffer starts with its upper halo); rmax1 = min(H-2, row_hi-1) is the
@@ -578,7 +580,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 // without pairwise f16 row sums, is no faster -- pass 1 waits on its TMA
 // loads more than on issue -- and the 6-row variant's extra code is 5%
 // slower.)
-__device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int C0w, int R0, int lane) {
+__device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int th1, int C0w, int R0, int lane) {
 #ifdef SHARP_EXP_NO_P1  // timing experiment only
   return 0.0f;
 #endif
@@ -597,7 +599,7 @@ __device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int C0
   // per-lane branches.
   float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 #pragma unroll 1
-  for (int m = 0; m < kTH1; m += 3) {
+  for (int m = 0; m < th1; m += 3) {
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
       const int r = R0 + m + a;
@@ -668,8 +670,8 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       }
       int C0 = 0, R0 = 0, nsub = 1, nw = 0;
       if (d.x == kP1 || d.x == kP2) {
-        tile_xy(g, d.z, d.x == kP1 ? kTH1 : kTH * kSub, C0, R0);
-        if (d.x == kP2) nsub = min(kSub, (g.row_hi - R0 + kTH - 1) / kTH);
+        tile_xy(g, d.z, d.x == kP1 ? g.th1 : kTH * g.sub, C0, R0);
+        if (d.x == kP2) nsub = min(g.sub, (g.row_hi - R0 + kTH - 1) / kTH);
 #pragma unroll
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
       }
@@ -774,7 +776,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
-      const float acc = (C0w < g.W) ? p1_warp(ring.stage(s) + warp * kSlot, g.W, g.rmax1, C0w, R0, lane) : 0.0f;
+      const float acc = (C0w < g.W) ? p1_warp(ring.stage(s) + warp * kSlot, g.W, g.rmax1, g.th1, C0w, R0, lane) : 0.0f;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
       // atomic per warp adding (1 << 40) + partial: the frame's arrival count
       // and sum in one word, so its LUT tasks can tell when S is complete
@@ -882,8 +884,18 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.g.rmax1 = std::min(H - 2, sg.row_hi - 1);
   const int rows = sg.row_hi - sg.row_lo;
   sp.g.tiles_x = (W + kCtaCols - 1) / kCtaCols;
-  sp.g.per_frame = sp.g.tiles_x * ((rows + kTH * kSub - 1) / (kTH * kSub));
-  sp.g.per_frame1 = sp.g.tiles_x * ((rows + kTH1 - 1) / kTH1);
+  const int grid_ctas = kCtasPerSm * num_sms();
+  // Latency: a launch with fewer kSub-row-group tasks than CTAs (one image,
+  // a short batch, a small band) runs its pass 2 as single sub-tiles, 3x the
+  // parallelism; big launches keep kSub (one LUT copy per kSub sub-tiles).
+  const int per_frame_sub = sp.g.tiles_x * ((rows + kTH * kSub - 1) / (kTH * kSub));
+  sp.g.sub = ((long long)sg.n * per_frame_sub < grid_ctas) ? 1 : kSub;
+  sp.g.per_frame = sp.g.tiles_x * ((rows + kTH * sp.g.sub - 1) / (kTH * sp.g.sub));
+  // pass-1 tiles: as tall as kTH1 while the launch has >= one tile per CTA
+  sp.g.th1 = kTH1;
+  while (sp.g.th1 > 3 && (long long)sg.n * sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1) < grid_ctas)
+    sp.g.th1 = sp.g.th1 == kTH1 ? 9 : sp.g.th1 - 3;
+  sp.g.per_frame1 = sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1);
   sp.mode = mode;
   sp.n = sg.n;
   sp.per_round = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
@@ -944,6 +956,16 @@ cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int ro
                             const Params &p, cudaStream_t stream) {
   if (mode != kStepPass1 && mode != kStepPass2) return cudaErrorInvalidValue;
   return launch_step(a, StepGeometry{1, rows_in, row_lo, row_hi, y0}, mode, W, H, p, stream);
+}
+
+// Forces the (lazy) module load of this file's kernels; see kernels.h.
+cudaError_t preload_step() {
+  cudaFuncAttributes a;
+  cudaError_t e;
+  if ((e = cudaFuncGetAttributes(&a, step_kernel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, band_prep_kernel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, band_finish_kernel)) != cudaSuccess) return e;
+  return cudaSuccess;
 }
 
 }  // namespace sharp

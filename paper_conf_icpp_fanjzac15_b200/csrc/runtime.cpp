@@ -576,6 +576,10 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
       if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->slots[i].done, cudaEventDisableTiming);
     }
     if (e != cudaSuccess) break;
+    // load every kernel now (lazy module loading can deadlock spinning kernels, kernels.h)
+    if ((e = sharp::preload_step()) != cudaSuccess || (e = sharp::preload_two_pass()) != cudaSuccess ||
+        (e = sharp::preload_staged()) != cudaSuccess || (e = sharp::preload_p2p()) != cudaSuccess)
+      break;
     if (c.max_frames > 0 && (rc = ensure_frames(ctx, (size_t)c.max_frames))) break;
     if (c.max_width > 0 && c.max_height > 0) {
       const size_t fb = (size_t)c.max_width * c.max_height;
@@ -705,6 +709,93 @@ int sharp_get_stage_times(sharp_ctx *ctx, float *ms, int n) {
     float t = 0.0f;
     CK(cudaEventElapsedTime(&t, r.a, r.b));
     ms[r.kind - 10] += t;
+  }
+  return SHARP_OK;
+}
+
+// ---- fused peer-memory band exchange (bands_p2p.cu)
+size_t sharp_p2p_window_bytes(int w, int rows_own) {
+  if (w < 16 || (w & 15) || rows_own < 4) return 0;
+  return sharp::p2p_window_bytes(w, rows_own);
+}
+
+int sharp_p2p_window_create(int w, int rows_own, void **d_window) {
+  if (!d_window) return SHARP_EINVAL;
+  *d_window = nullptr;
+  const size_t bytes = sharp_p2p_window_bytes(w, rows_own);
+  if (!bytes) return SHARP_EINVAL;
+  if (cudaMalloc(d_window, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    *d_window = nullptr;
+    return SHARP_ENOMEM;
+  }
+  if (cudaMemset(*d_window, 0, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    cudaFree(*d_window);
+    *d_window = nullptr;
+    return SHARP_ECUDA;
+  }
+  return SHARP_OK;
+}
+
+void sharp_p2p_window_destroy(void *d_window) {
+  if (d_window) cudaFree(d_window);
+}
+
+int sharp_band_p2p_halo(sharp_ctx *ctx, uint8_t *self_window, int w, int rows_own, uint8_t *up_window,
+                        int up_rows_own, uint8_t *down_window, uint64_t epoch) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  if (!self_window || w < 16 || (w & 15) || rows_own < 4 || epoch == 0 || (up_window && up_rows_own < 4) ||
+      (((uintptr_t)self_window | (uintptr_t)up_window | (uintptr_t)down_window) & 15))
+    return set_err(ctx, SHARP_EINVAL, "%s", "bad p2p halo request (w % 16, rows >= 4, 16-byte windows, epoch > 0)");
+  CK(sharp::launch_p2p_halo(self_window, w, rows_own, up_window, up_rows_own, down_window, epoch, ctx->stream));
+  return SHARP_OK;
+}
+
+int sharp_band_p2p_allreduce(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank,
+                             const uint64_t *d_partial, uint64_t epoch, uint64_t *d_total) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  if (!windows || !d_partial || !d_total || n_ranks < 1 || n_ranks > 32 || rank < 0 || rank >= n_ranks ||
+      epoch == 0)
+    return set_err(ctx, SHARP_EINVAL, "%s", "bad p2p all-reduce request (1 <= n_ranks <= 32, epoch > 0)");
+  for (int g = 0; g < n_ranks; ++g)
+    if (!windows[g] || ((uintptr_t)windows[g] & 15)) return set_err(ctx, SHARP_EINVAL, "%s", "bad window pointer");
+  CK(sharp::launch_p2p_allreduce(windows, n_ranks, rank, reinterpret_cast<const unsigned long long *>(d_partial),
+                                 epoch, reinterpret_cast<unsigned long long *>(d_total), ctx->stream));
+  return SHARP_OK;
+}
+
+int sharp_ipc_get_handle(const void *d_ptr, void *handle) {
+  if (!d_ptr || !handle) return SHARP_EINVAL;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, const_cast<void *>(d_ptr)) != cudaSuccess) {
+    cudaGetLastError();
+    return SHARP_ECUDA;
+  }
+  static_assert(sizeof(h) == SHARP_IPC_HANDLE_BYTES, "IPC handle size");
+  memcpy(handle, &h, sizeof(h));
+  return SHARP_OK;
+}
+
+int sharp_ipc_open_handle(const void *handle, void **d_ptr) {
+  if (!handle || !d_ptr) return SHARP_EINVAL;
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, sizeof(h));
+  if (cudaIpcOpenMemHandle(d_ptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+    cudaGetLastError();
+    *d_ptr = nullptr;
+    return SHARP_ECUDA;
+  }
+  return SHARP_OK;
+}
+
+int sharp_ipc_close_handle(void *d_ptr) {
+  if (!d_ptr) return SHARP_EINVAL;
+  if (cudaIpcCloseMemHandle(d_ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return SHARP_ECUDA;
   }
   return SHARP_OK;
 }
