@@ -441,8 +441,15 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   for (int x = 0; x < 8; ++x) {
     const int p = pair_of(x);
     const bool hi = half_of(x);
+#ifdef SHARP_EXP_LUT_MAD8
     const uint32_t qb = __float_as_uint(add_f32_f16(hi ? hi16(pe[p]) : lo16(pe[p]), 8388608.0f));  // 2^23 + pEdge
     const float2 L = lds_f2(mad8(qb, lut_q));                                                      // {adj, osc}
+#else
+    // f32 bits of 2^20 + pEdge = 0x49800000 + 8 pEdge: the byte offset of the
+    // entry, scaled by the exponent (ulp 1/8) -- one FHADD, no IMAD.
+    const uint32_t q8 = __float_as_uint(add_f32_f16(hi ? hi16(pe[p]) : lo16(pe[p]), 1048576.0f));
+    const float2 L = lds_f2(q8 + lut_q);  // {adj, osc}
+#endif
     const float E = add_f32_f16(hi ? hi16(rb.c[p]) : lo16(rb.c[p]), NU[x]);                       // O - U (L148)
     P[x] = __fmaf_rn(L.x, E, -NU[x]);                                                              // L178
     const float mxf = add_f32_f16(hi ? hi16(MX[p]) : lo16(MX[p]), 0.0f);
@@ -501,7 +508,8 @@ struct Ring {
 // (Measured: a fully unrolled 12-row interior body -- no per-row phase or
 // ring tests -- is 40% SLOWER: ~36 KB of straight-line code overflows the
 // instruction cache.  The hot loops must stay small.)
-__device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint32_t lut, uint8_t *__restrict__ out,
+__device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint32_t lut0, int lut_odd,
+                                        uint8_t *__restrict__ out,
                                         int W, int H, int row_lo, int row_hi, int C0w, int R0, int warp,
                                         int lane) {
 #ifdef SHARP_EXP_NO_P2  // timing experiment only
@@ -522,7 +530,14 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (a
   // shuffle hides the value from ptxas, which would otherwise split the
   // constant back out into one extra IADD per pixel).
-  const uint32_t lut_q = __shfl_sync(0xffffffffu, lut - (0x4B000000u << 3), 0);
+#ifdef SHARP_EXP_LUT_MAD8
+  const uint32_t lut_q = __shfl_sync(0xffffffffu, lut0 + (lut_odd ? kLutBytes : 0) - (0x4B000000u << 3), 0);
+#else
+  // (The vote makes the buffer choice -- and so the base -- provably
+  // warp-uniform: ptxas keeps it in a uniform register and folds it into the
+  // LDS address, [R + UR].)
+  const uint32_t lut_q = lut0 + (__any_sync(0xffffffffu, lut_odd) ? (uint32_t)kLutBytes : 0u) - 0x49800000u;
+#endif
   // In a sub-tile starting at row R0k, smem row of global row R0k-4 is 0:
   // row r -> smem row r - R0k + 4.
   // Vertical interpolation (L146, R3) of D rows (i, i+1) is linear in r on
@@ -742,7 +757,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       const int2 aux = stage_aux[b];
       const int C0 = d.z, R0 = d.w, C0w = C0 + warp * kTW;
       if (C0w < g.W) {
-        p2_warp(ring, s, aux.x, lutbase + (uint32_t)(aux.y * kLutBytes), sp.out + (size_t)d.y * g.W * g.H, g.W, g.H,
+        p2_warp(ring, s, aux.x, lutbase, aux.y, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H,
                 g.row_lo, g.row_hi, C0w, R0, warp, lane);
       } else {  // no columns for this warp: follow the stages
         for (int k = 0; k < aux.x; ++k) {
