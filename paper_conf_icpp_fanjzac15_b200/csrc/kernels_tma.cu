@@ -54,7 +54,11 @@ constexpr int kWarpsT = 4;   // compute warps = warp tiles per CTA tile
 constexpr int kCtaCols = kTW * kWarpsT;
 constexpr int kThreadsT = 32 * (kWarpsT + 1);  // + producer warp
 constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task
-constexpr int kLutTasks = kLutSize / kLutPerTask;
+// pEdge = |Gx| + |Gy| is always even (Gx and Gy both have the parity of the
+// sum of the four window corners), so the step kernel's tables hold the even
+// entries only: entry k = pEdge / 2, k < kLut2 (766 used).
+constexpr int kLut2 = 768;
+constexpr int kLutTasks = kLut2 / kLutPerTask;
 // A warp tile needs columns C0w-8 .. C0w+247.  TMA box starts must be
 // 16-byte aligned in the innermost dimension and a box dimension is at most
 // 256, so each warp tile is fetched as two boxes of the [n][H][W] frames:
@@ -71,7 +75,7 @@ constexpr int kBox2 = (kPitch + kPitchB) * kRows2;
 constexpr int kBox1 = (kPitch + kPitchB) * kRows1;
 constexpr int kSlot = (kBox2 + 127) / 128 * 128;  // per-warp smem slot (128-B aligned)
 static_assert((kPitch * kRows1) % 128 == 0 && (kPitch * kRows2) % 128 == 0, "region B alignment");
-constexpr int kLutBytes = kLutSize * 8;
+constexpr int kLutBytes = kLut2 * 8;
 // A pass-2 task is kSub vertically adjacent CTA tiles ("sub-tiles") of one
 // frame: each sub-tile fills one stage, the frame's LUT is copied once per
 // task into one of two LUT buffers (task parity), and the warps carry their
@@ -87,7 +91,7 @@ constexpr int kSmem = kBarOff + 64;
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
 static_assert(kTH1 % 3 == 0 && kBox1 <= kSlot, "pass-1 tiles (3-row loop)");
-static_assert(kLutSize % kLutPerTask == 0, "LUT tasks");
+static_assert(kLut2 % kLutPerTask == 0 && kLut2 <= kLutSize && 2 * (kLut2 - 1) >= 1530, "LUT tasks");
 
 // ------------------------------------------------------------ TMA / mbarrier
 __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
@@ -177,13 +181,6 @@ __device__ __forceinline__ unsigned int ld_acquire(const unsigned int *p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-// LDS address q*8 + base in one integer op.
-__device__ __forceinline__ uint32_t mad8(uint32_t q, uint32_t base) {
-  uint32_t r;
-  asm("mad.lo.u32 %0, %1, 8, %2;" : "=r"(r) : "r"(q), "r"(base));
-  return r;
-}
-
 // ----------------------------------------------------------- packed f32x2
 __device__ __forceinline__ unsigned long long f2pack(float a, float b) {
   unsigned long long r;
@@ -441,15 +438,12 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   for (int x = 0; x < 8; ++x) {
     const int p = pair_of(x);
     const bool hi = half_of(x);
-#ifdef SHARP_EXP_LUT_MAD8
-    const uint32_t qb = __float_as_uint(add_f32_f16(hi ? hi16(pe[p]) : lo16(pe[p]), 8388608.0f));  // 2^23 + pEdge
-    const float2 L = lds_f2(mad8(qb, lut_q));                                                      // {adj, osc}
-#else
-    // f32 bits of 2^20 + pEdge = 0x49800000 + 8 pEdge: the byte offset of the
-    // entry, scaled by the exponent (ulp 1/8) -- one FHADD, no IMAD.
-    const uint32_t q8 = __float_as_uint(add_f32_f16(hi ? hi16(pe[p]) : lo16(pe[p]), 1048576.0f));
+    // f32 bits of 2^21 + pEdge = 0x4A000000 + 4 pEdge = 0x4A000000 + 8 k (ulp
+    // 1/4; pEdge = 2k is even): the byte offset of entry k, scaled by the
+    // exponent -- one FHADD, no IMAD.  (Even-only entries also spread the
+    // lookups over all 32 banks.)
+    const uint32_t q8 = __float_as_uint(add_f32_f16(hi ? hi16(pe[p]) : lo16(pe[p]), 2097152.0f));
     const float2 L = lds_f2(q8 + lut_q);  // {adj, osc}
-#endif
     const float E = add_f32_f16(hi ? hi16(rb.c[p]) : lo16(rb.c[p]), NU[x]);                       // O - U (L148)
     P[x] = __fmaf_rn(L.x, E, -NU[x]);                                                              // L178
     const float mxf = add_f32_f16(hi ? hi16(MX[p]) : lo16(MX[p]), 0.0f);
@@ -527,17 +521,11 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
   LaneRow aw = lane_row(ring.stage(s) + warp * kSlot, kRows2, lane);
   const uint64_t pol_out = policy_evict_first();  // output: written once, never re-read
-  // LDS address of entry p from the bits of (2^23 + p): q*8 + lut_q (a
-  // shuffle hides the value from ptxas, which would otherwise split the
-  // constant back out into one extra IADD per pixel).
-#ifdef SHARP_EXP_LUT_MAD8
-  const uint32_t lut_q = __shfl_sync(0xffffffffu, lut0 + (lut_odd ? kLutBytes : 0) - (0x4B000000u << 3), 0);
-#else
-  // (The vote makes the buffer choice -- and so the base -- provably
+  // LDS address of entry k = pEdge/2: the f32 bits of (2^21 + pEdge) plus
+  // lut_q.  The vote makes the LUT-buffer choice -- and so lut_q -- provably
   // warp-uniform: ptxas keeps it in a uniform register and folds it into the
-  // LDS address, [R + UR].)
-  const uint32_t lut_q = lut0 + (__any_sync(0xffffffffu, lut_odd) ? (uint32_t)kLutBytes : 0u) - 0x49800000u;
-#endif
+  // load, LDS [R + UR] (one FHADD + one LDS per pixel).
+  const uint32_t lut_q = lut0 + (__any_sync(0xffffffffu, lut_odd) ? (uint32_t)kLutBytes : 0u) - 0x4A000000u;
   // In a sub-tile starting at row R0k, smem row of global row R0k-4 is 0:
   // row r -> smem row r - R0k + 4.
   // Vertical interpolation (L146, R3) of D rows (i, i+1) is linear in r on
@@ -769,8 +757,9 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       continue;
     }
     if (d.x == kLut) {
-      // LUT task: entries q*128 .. q*128+127 of frame f (R9, R11; f64, one rounding)
-      const int f = d.y, p = d.z * kLutPerTask + threadIdx.x;
+      // LUT task: entries k = q*128 .. q*128+127 (pEdge p = 2k) of frame f
+      // (R9, R11; f64, one rounding)
+      const int f = d.y, k = d.z * kLutPerTask + threadIdx.x, p = 2 * k;
       // L174: mean of pEdge over all W*H elements (R8), from the exact sum.
       const unsigned long long S = stage_sum[b];
       const double mean = (double)S / ((double)g.W * (double)g.H);
@@ -784,7 +773,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         adj = (float)((double)sp.prm.amount * pow((double)p / m, (double)sp.prm.gamma));
         osc = (float)fmin(fmax((double)sp.prm.osc_gain * exp(-(double)p / ((double)sp.prm.osc_scale * m)), 0.0), 1.0);
       }
-      sp.luts[(size_t)f * kLutSize + p] = make_float2(adj, osc);
+      sp.luts[(size_t)f * kLutSize + k] = make_float2(adj, osc);
       __threadfence();
       __syncwarp();
       if (lane == 0) atomicAdd(&sp.lut_done[f], 1u);
