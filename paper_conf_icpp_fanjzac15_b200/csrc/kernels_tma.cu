@@ -61,20 +61,21 @@ constexpr int kLut2 = 768;
 constexpr int kLutTasks = kLut2 / kLutPerTask;
 // A warp tile needs columns C0w-8 .. C0w+247.  TMA box starts must be
 // 16-byte aligned in the innermost dimension and a box dimension is at most
-// 256, so each warp tile is fetched as two boxes of the [n][H][W] frames:
-//   region A: 256 columns C0w-16 .. C0w+239  (smem pitch 256)
-//   region B:  16 columns C0w+240 .. C0w+255 (smem pitch 16; only lane 30,
-//             the right halo, reads it)
+// 256, so a warp tile is fetched as one 256-column box of the [n][H][W]
+// frames, region A = columns C0w-16 .. C0w+239 (smem pitch 256).  Its right
+// halo C0w+240.. is the first own column of the next warp's region A (offset
+// kCol0 there); only the CTA tile's last warp needs one more box, region B =
+// 16 columns C0w+240 .. C0w+255 (smem pitch 16) after the four slots.  (When
+// the next warp has no columns, the halo lies beyond the image and only feeds
+// pixels that are either not stored or on the overridden frame column W-1.)
 constexpr int kPitch = 256;           // region A pitch
 constexpr int kPitchB = 16;           // region B pitch
 constexpr int kCol0 = 16;             // region-A column of C0w
 constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+kTH+3
 constexpr int kTH1 = 18;              // pass-1 output rows per warp tile (fits the same slot)
 constexpr int kRows1 = kTH1 + 2;      // pass-1 box rows: R0-1 .. R0+kTH1
-constexpr int kBox2 = (kPitch + kPitchB) * kRows2;
-constexpr int kBox1 = (kPitch + kPitchB) * kRows1;
-constexpr int kSlot = (kBox2 + 127) / 128 * 128;  // per-warp smem slot (128-B aligned)
-static_assert((kPitch * kRows1) % 128 == 0 && (kPitch * kRows2) % 128 == 0, "region B alignment");
+constexpr int kSlot = kPitch * kRows2;  // per-warp smem slot: region A (128-B aligned)
+static_assert(kRows1 <= kRows2 && kSlot % 128 == 0, "pass-1 tiles fit the slots");
 constexpr int kLutBytes = kLut2 * 8;
 // A pass-2 task is kSub vertically adjacent CTA tiles ("sub-tiles") of one
 // frame: each sub-tile fills one stage, the frame's LUT is copied once per
@@ -84,13 +85,18 @@ constexpr int kLutBytes = kLut2 * 8;
 #define SHARP_P2_SUB 3
 #endif
 constexpr int kSub = SHARP_P2_SUB;
-constexpr int kStage = kWarpsT * kSlot;       // one stage: the 4 warp slots
-constexpr int kLutOff = 2 * kStage;           // two LUT buffers after the two stages
+#ifndef SHARP_STAGES
+#define SHARP_STAGES 2  // measured: 3 stages +0.3%, 2 stages (this layout) +0.6% vs the old layout
+#endif
+constexpr int kStages = SHARP_STAGES;          // smem ring depth
+constexpr int kRegB = kWarpsT * kSlot;         // region B of the last warp
+constexpr int kStage = (kRegB + kPitchB * kRows2 + 127) / 128 * 128;  // one stage
+constexpr int kLutOff = kStages * kStage;      // two LUT buffers after the stages
 constexpr int kBarOff = kLutOff + 2 * kLutBytes;
-constexpr int kSmem = kBarOff + 64;
+constexpr int kSmem = kBarOff + 16 * kStages;  // full + empty barrier per stage
 static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
-static_assert(kTH1 % 3 == 0 && kBox1 <= kSlot, "pass-1 tiles (3-row loop)");
+static_assert(kTH1 % 3 == 0, "pass-1 tiles (3-row loop)");
 static_assert(kLut2 % kLutPerTask == 0 && kLut2 <= kLutSize && 2 * (kLut2 - 1) >= 1530, "LUT tasks");
 
 // ------------------------------------------------------------ TMA / mbarrier
@@ -152,11 +158,15 @@ __device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, in
       "l"(map), "r"(x), "r"(r), "r"(f), "r"(bar), "l"(policy)
       : "memory");
 }
-// Both boxes of a warp tile (region A then region B at dst + kPitch*rows).
-__device__ __forceinline__ void tma_tile(uint32_t dst, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0w,
-                                         int r, int rows, int f, uint32_t bar, uint64_t policy) {
-  tma_box(dst, mapA, C0w - kCol0, r, f, bar, policy);
-  tma_box(dst + (uint32_t)(kPitch * rows), mapB, C0w + 256 - kCol0, r, f, bar, policy);
+// The boxes of a CTA tile of nw warp tiles into stage st: region A per warp,
+// and region B (the last warp's right halo) when all kWarpsT warps have columns.
+__device__ __forceinline__ uint32_t tile_bytes(int nw, int rows) {
+  return (uint32_t)((nw * kPitch + (nw == kWarpsT ? kPitchB : 0)) * rows);
+}
+__device__ __forceinline__ void tma_tiles(uint32_t st, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0, int nw,
+                                          int r, int f, uint32_t bar, uint64_t policy) {
+  for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, mapA, C0 + w * kTW - kCol0, r, f, bar, policy);
+  if (nw == kWarpsT) tma_box(st + kRegB, mapB, C0 + kWarpsT * kTW, r, f, bar, policy);
 }
 // Output store.  (Measured: an L2::cache_hint store costs ~5% of the step
 // through extra issue; plain STG.64 it is -- SHARP_EXP_HINT_STORE to compare.)
@@ -285,20 +295,18 @@ __device__ __forceinline__ void fence_acquire() { asm volatile("fence.acq_rel.gp
 // ------------------------------------------------------------- row window
 // Lane words of smem row s: lanes 0..29 own columns C0w+8l..+7 (region A);
 // lane 31 the left halo C0w-8..C0w-1 (region A); lane 30 the right halo
-// C0w+240..247 (region B, pitch 16).
+// C0w+240..247 (the next warp's region A, or region B for the last warp).
 struct LaneRow {
   uint32_t base, pitch;
 };
-__device__ __forceinline__ LaneRow lane_row(uint32_t tile, int rows, int lane) {
-  if (lane == 30) return LaneRow{tile + (uint32_t)(kPitch * rows), (uint32_t)kPitchB};
-  return LaneRow{tile + (uint32_t)(kCol0 + 8 * (lane < 31 ? lane : -1)), (uint32_t)kPitch};
+__device__ __forceinline__ LaneRow lane_row(uint32_t stage, int warp, int lane) {
+  if (lane == 30) {
+    if (warp == kWarpsT - 1) return LaneRow{stage + (uint32_t)kRegB, (uint32_t)kPitchB};
+    return LaneRow{stage + (uint32_t)((warp + 1) * kSlot + kCol0), (uint32_t)kPitch};
+  }
+  return LaneRow{stage + (uint32_t)(warp * kSlot + kCol0 + 8 * (lane < 31 ? lane : -1)), (uint32_t)kPitch};
 }
 __device__ __forceinline__ uint2 row_words(const LaneRow &a, int s) { return lds_u64(a.base + (uint32_t)s * a.pitch); }
-// smem address of (tile row s, column C0w - kCol0 + rel), either region.
-__device__ __forceinline__ uint32_t tile_addr(uint32_t tile, int rows, int s, int rel) {
-  return rel < kPitch ? tile + (uint32_t)(s * kPitch + rel)
-                      : tile + (uint32_t)(kPitch * rows + s * kPitchB + (rel - kPitch));
-}
 
 // Converts a row of words into the window data.  Neighbour pairs come from
 // the adjacent lanes (shuffle), so each lane loads only its own 8 bytes.
@@ -479,20 +487,22 @@ __device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y)
 }
 
 // Stage ring shared by the producer and the consumers: stage s (a running
-// count) lives in buffer s & 1 and completes phase (s >> 1) & 1.
+// count) lives in buffer s % kStages and completes phase (s / kStages) & 1.
 struct Ring {
   uint32_t sbase, full0, empty0;
-  __device__ __forceinline__ uint32_t stage(int s) const { return sbase + (uint32_t)((s & 1) * kStage); }
+  __device__ __forceinline__ static int buf(int s) { return (unsigned)s % kStages; }
+  __device__ __forceinline__ static uint32_t phase(int s) { return ((unsigned)s / kStages) & 1u; }
+  __device__ __forceinline__ uint32_t stage(int s) const { return sbase + (uint32_t)(buf(s) * kStage); }
   __device__ __forceinline__ void wait_full(int s) const {
 #ifdef SHARP_EXP_SPIN_WAIT
-    mbar_wait_spin(full0 + 8u * (s & 1), (uint32_t)((s >> 1) & 1));
+    mbar_wait_spin(full0 + 8u * buf(s), phase(s));
 #else
-    mbar_wait(full0 + 8u * (s & 1), (uint32_t)((s >> 1) & 1));
+    mbar_wait(full0 + 8u * buf(s), phase(s));
 #endif
   }
   __device__ __forceinline__ void release(int s, int lane) const {  // one arrival per consumer warp
     __syncwarp();
-    if (lane == 0) mbar_arrive(empty0 + 8u * (s & 1));
+    if (lane == 0) mbar_arrive(empty0 + 8u * buf(s));
   }
 };
 
@@ -519,7 +529,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   // W-2,W-1 in the lane with c0 == W-8.
   const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
-  LaneRow aw = lane_row(ring.stage(s) + warp * kSlot, kRows2, lane);
+  LaneRow aw = lane_row(ring.stage(s), warp, lane);
   const uint64_t pol_out = policy_evict_first();  // output: written once, never re-read
   // LDS address of entry k = pEdge/2: the f32 bits of (2^21 + pEdge) plus
   // lut_q.  The vote makes the LUT-buffer choice -- and so lut_q -- provably
@@ -547,7 +557,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
     const int R0k = R0 + k * kTH;
     if (k) {  // next sub-tile: same rows layout in the next stage; state carried
       ring.wait_full(s + k);
-      aw = lane_row(ring.stage(s + k) + warp * kSlot, kRows2, lane);
+      aw = lane_row(ring.stage(s + k), warp, lane);
     }
     const int rend = min(R0k + kTH, row_hi);
     const int rend_l = active ? rend : R0k;  // this lane stores rows < rend_l
@@ -583,12 +593,13 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 // without pairwise f16 row sums, is no faster -- pass 1 waits on its TMA
 // loads more than on issue -- and the 6-row variant's extra code is 5%
 // slower.)
-__device__ __forceinline__ float p1_warp(uint32_t tile, int W, int rmax1, int th1, int C0w, int R0, int lane) {
+__device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rmax1, int th1, int C0w, int R0,
+                                        int lane) {
 #ifdef SHARP_EXP_NO_P1  // timing experiment only
   return 0.0f;
 #endif
   const int c0 = C0w + 8 * lane;
-  const LaneRow aw = lane_row(tile, kRows1, lane);
+  const LaneRow aw = lane_row(stage, warp, lane);
   // Sobel-body pixels of this lane (not frame columns, not beyond the image).
   uint32_t vmask = 0;
 #pragma unroll
@@ -633,20 +644,20 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     step_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
                 const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, StepParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ int4 stage_task[2];                 // {type, frame, C0, R0} (LUT tasks: {type, frame, q, 0})
-  __shared__ int2 stage_aux[2];                  // pass 2: {sub-tiles of the task, LUT buffer}
-  __shared__ unsigned long long stage_sum[2];    // LUT tasks: the frame's S
+  __shared__ int4 stage_task[kStages];               // {type, frame, C0, R0} (LUT tasks: {type, frame, q, 0})
+  __shared__ int2 stage_aux[kStages];                // pass 2: {sub-tiles of the task, LUT buffer}
+  __shared__ unsigned long long stage_sum[kStages];  // LUT tasks: the frame's S
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t sbase = smem_u32(smem);
-  const Ring ring{sbase, sbase + kBarOff, sbase + kBarOff + 16};
+  const Ring ring{sbase, sbase + kBarOff, sbase + kBarOff + 8 * kStages};
   const uint32_t lutbase = sbase + kLutOff;
   const Geo &g = sp.g;
 
   if (threadIdx.x == 0) {
-    mbar_init(ring.full0, 1);
-    mbar_init(ring.full0 + 8, 1);
-    mbar_init(ring.empty0, kWarpsT);
-    mbar_init(ring.empty0 + 8, kWarpsT);
+    for (int i = 0; i < kStages; ++i) {
+      mbar_init(ring.full0 + 8 * i, 1);
+      mbar_init(ring.empty0 + 8 * i, kWarpsT);
+    }
     fence_barrier_init();
   }
   __syncthreads();
@@ -657,7 +668,10 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     const unsigned long long arrivals = (unsigned long long)(g.per_frame1 * kWarpsT) << kAccShift;
     const uint64_t pol_keep = policy_evict_last(), pol_drop = policy_evict_first();
     int t_next = (int)atomicAdd(sp.task_counter, 1u);
-    for (int s = 0, j = 0;; ++j) {  // s: stages filled, j: tasks (LUT buffer parity)
+    // s: stages filled; j: pass-2 tasks (LUT buffer j & 1); lut_last[b]: the
+    // last stage of the pass-2 task that used LUT buffer b.
+    int lut_last[2] = {-kStages, -kStages};
+    for (int s = 0, j = 0;;) {
       const int4 d = decode(sp, t_next);
       // Resolve the task's dependency first (before waiting for a stage).
       unsigned long long S = 0;
@@ -679,8 +693,8 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
       }
       for (int k = 0; k < nsub; ++k, ++s) {
-        const int b = s & 1;
-        if (s >= 2) mbar_wait(ring.empty0 + 8u * b, (uint32_t)(((s >> 1) - 1) & 1));
+        const int b = Ring::buf(s);
+        if (s >= kStages) mbar_wait(ring.empty0 + 8u * b, Ring::phase(s) ^ 1u);
         // Grab the following task now: the atomic's latency overlaps this
         // task's loads and the next empty-wait.
         if (k == 0 && d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
@@ -690,17 +704,20 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
 #endif
         if (d.x == kP1) {
           stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
-          mbar_expect_tx(full, (uint32_t)(nw * kBox1));
-          for (int w = 0; w < nw; ++w)
-            tma_tile(st + w * kSlot, &map1A, &map1B, C0 + w * kTW, R0 - 1 - g.y0, kRows1, d.y, full, pol_keep);
+          mbar_expect_tx(full, tile_bytes(nw, kRows1));
+          tma_tiles(st, &map1A, &map1B, C0, nw, R0 - 1 - g.y0, d.y, full, pol_keep);
         } else if (d.x == kP2) {
           const int R0k = R0 + k * kTH;
           stage_task[b] = make_int4(d.x, d.y, C0, R0k);
           stage_aux[b] = make_int2(nsub, j & 1);
           const uint32_t lut_bytes = k == 0 ? (uint32_t)kLutBytes : 0u;
-          mbar_expect_tx(full, (uint32_t)(nw * kBox2) + lut_bytes);
-          for (int w = 0; w < nw; ++w)
-            tma_tile(st + w * kSlot, &map2A, &map2B, C0 + w * kTW, R0k - 4 - g.y0, kRows2, d.y, full, pol_drop);
+          // LUT buffer j & 1 is free once the stages of pass-2 task j-2 are
+          // released: stages <= s - kStages are (the empty wait above); a
+          // later one only after single-stage pass-2 tasks.
+          const int tl = lut_last[j & 1];
+          if (k == 0 && tl > s - kStages) mbar_wait(ring.empty0 + 8u * Ring::buf(tl), Ring::phase(tl));
+          mbar_expect_tx(full, tile_bytes(nw, kRows2) + lut_bytes);
+          tma_tiles(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
           if (lut_bytes)
             bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
         } else {
@@ -709,6 +726,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           mbar_arrive(full);  // no data: LUT, empty or end task
         }
       }
+      if (d.x == kP2) lut_last[j++ & 1] = s - 1;
       if (d.x == kEnd) break;
     }
     return;
@@ -720,7 +738,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
   const long long t_begin = clock64();
 #endif
   for (int s = 0;;) {
-    const int b = s & 1;
+    const int b = Ring::buf(s);
 #ifdef SHARP_EXP_WAITSTAT
     const long long tw0 = clock64();
 #endif
@@ -780,7 +798,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
-      const float acc = (C0w < g.W) ? p1_warp(ring.stage(s) + warp * kSlot, g.W, g.rmax1, g.th1, C0w, R0, lane) : 0.0f;
+      const float acc = (C0w < g.W) ? p1_warp(ring.stage(s), warp, g.W, g.rmax1, g.th1, C0w, R0, lane) : 0.0f;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
       // atomic per warp adding (1 << 40) + partial: the frame's arrival count
       // and sum in one word, so its LUT tasks can tell when S is complete
@@ -906,7 +924,13 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
 #ifndef SHARP_GRID_CTAS
 #define SHARP_GRID_CTAS kCtasPerSm
 #endif
-  const int grid = SHARP_GRID_CTAS * num_sms();
+  static int resident = 0;  // CTAs per SM that actually fit (registers, smem)
+  if (!resident) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, step_kernel, kThreadsT, kSmem) != cudaSuccess ||
+        resident < 1)
+      resident = 1;
+  }
+  const int grid = std::min(SHARP_GRID_CTAS, resident) * num_sms();
   if (mode == kStepPass1) {
     sp.L1 = sp.L2 = 0;
     sp.ntasks = sp.g.per_frame1;
