@@ -27,14 +27,18 @@ int oracle_check_geometry(int W, int H) {
  * downscaled matrix is the mean value of the elements in the corresponding
  * 4 x 4 submatrix".  R2: exact mean (sum/16 is exact in float).
  * ------------------------------------------------------------------------- */
-void oracle_downscale(const uint8_t *O, int W, int H, float *D) {
+void oracle_downscale(const uint8_t *O, int W, int H, float *D) { oracle_downscale_ex(O, W, H, 0, D); }
+
+/* flags & ORACLE_READ_INT_DOWNSCALE (R2 alternative, "shifts replace
+ * division", L374): D = floor(sum / 16), the integer shift sum >> 4. */
+void oracle_downscale_ex(const uint8_t *O, int W, int H, int flags, float *D) {
   const int w = W / 4, h = H / 4;
   for (int i = 0; i < h; ++i)
     for (int j = 0; j < w; ++j) {
       unsigned sum = 0;
       for (int a = 0; a < 4; ++a)
         for (int b = 0; b < 4; ++b) sum += O[(size_t)(4 * i + a) * W + (4 * j + b)];
-      D[(size_t)i * w + j] = (float)sum / 16.0f;
+      D[(size_t)i * w + j] = (flags & ORACLE_READ_INT_DOWNSCALE) ? (float)(sum >> 4) : (float)sum / 16.0f;
     }
 }
 
@@ -61,12 +65,26 @@ static void line(const float *v, int vs, int n, float *out, int os) {
   out[(size_t)(n - 3) * os] = out[(size_t)(n - 4) * os]; /* third last <- fourth last */
 }
 
-void oracle_upscale(const float *D, int W, int H, float *U) {
-  oracle_upscale_steps(D, W, H, U, 8);
-}
+void oracle_upscale(const float *D, int W, int H, float *U) { oracle_upscale_steps_ex(D, W, H, U, 8, 0); }
 
 void oracle_upscale_steps(const float *D, int W, int H, float *U, int last_step) {
+  oracle_upscale_steps_ex(D, W, H, U, last_step, 0);
+}
+
+void oracle_upscale_ex(const float *D, int W, int H, int flags, float *U) {
+  oracle_upscale_steps_ex(D, W, H, U, 8, flags);
+}
+
+/* Default order: steps (i)..(vii) as L140-L142 list them (R5).  With
+ * flags & ORACLE_READ_COLUMN_WINS (the R5 alternative) the row work comes
+ * first -- (i), (iii), (v) -- and the column work after it -- (ii), (iv),
+ * (vi) -- so in the top-left 2x2 the column line and the column copy are the
+ * last writers; (vii) stays last.  last_step counts steps in the order run. */
+void oracle_upscale_steps_ex(const float *D, int W, int H, float *U, int last_step, int flags) {
   const int w = W / 4, h = H / 4;
+  static const int order_default[7] = {1, 2, 3, 4, 5, 6, 7};
+  static const int order_colwins[7] = {1, 3, 5, 2, 4, 6, 7};
+  const int *order = (flags & ORACLE_READ_COLUMN_WINS) ? order_colwins : order_default;
   /* Fill with NaN so a pixel that no step writes is visible (the pins check
    * that none is left). */
   for (size_t p = 0; p < (size_t)W * H; ++p) U[p] = NAN;
@@ -74,41 +92,44 @@ void oracle_upscale_steps(const float *D, int W, int H, float *U, int last_step)
 #define D_(i, j) D[(size_t)(i) * w + (j)]
 
   /* 1) Upscale the border (L140-L142). */
-  /* (i)  first row of D -> first row of U, columns 0..W-3 */
-  line(&D_(0, 0), 1, W, &U_(0, 0), 1);
-  if (last_step < 2) return;
-  /* (ii) first column of D -> first column of U, rows 0..H-3 */
-  line(&D_(0, 0), w, H, &U_(0, 0), W);
-  if (last_step < 3) return;
-  /* (iii) "the penultimate row ... based on the last row" of D */
-  line(&D_(h - 1, 0), 1, W, &U_(H - 2, 0), 1);
-  if (last_step < 4) return;
-  /* (iv) "the penultimate ... column ... based on the last ... column" of D */
-  line(&D_(0, w - 1), w, H, &U_(0, W - 2), W);
-  if (last_step < 5) return;
-  /* (v) "copied directly to the second row" / "copied to the last row"
-   *     (over the columns the row passes computed, 0..W-3) */
-  for (int c = 0; c <= W - 3; ++c) {
-    U_(1, c) = U_(0, c);
-    U_(H - 1, c) = U_(H - 2, c);
-  }
-  if (last_step < 6) return;
-  /* (vi) "... and column respectively" / "... and the last column"
-   *      (over the rows the column passes computed, 0..H-3) */
-  for (int r = 0; r <= H - 3; ++r) {
-    U_(r, 1) = U_(r, 0);
-    U_(r, W - 1) = U_(r, W - 2);
-  }
-  if (last_step < 7) return;
-  /* (vii) "the four elements of the bottom right corner are still missing.
-   *       The third last value of the last column will be copied to those
-   *       elements" */
-  {
-    const float v = U_(H - 3, W - 1);
-    U_(H - 2, W - 2) = v;
-    U_(H - 2, W - 1) = v;
-    U_(H - 1, W - 2) = v;
-    U_(H - 1, W - 1) = v;
+  for (int k = 0; k < 7 && k < last_step; ++k) {
+    switch (order[k]) {
+      case 1: /* (i)  first row of D -> first row of U, columns 0..W-3 */
+        line(&D_(0, 0), 1, W, &U_(0, 0), 1);
+        break;
+      case 2: /* (ii) first column of D -> first column of U, rows 0..H-3 */
+        line(&D_(0, 0), w, H, &U_(0, 0), W);
+        break;
+      case 3: /* (iii) "the penultimate row ... based on the last row" of D */
+        line(&D_(h - 1, 0), 1, W, &U_(H - 2, 0), 1);
+        break;
+      case 4: /* (iv) "the penultimate ... column ... based on the last ... column" of D */
+        line(&D_(0, w - 1), w, H, &U_(0, W - 2), W);
+        break;
+      case 5: /* (v) "copied directly to the second row" / "copied to the last row"
+               *     (over the columns the row passes computed, 0..W-3) */
+        for (int c = 0; c <= W - 3; ++c) {
+          U_(1, c) = U_(0, c);
+          U_(H - 1, c) = U_(H - 2, c);
+        }
+        break;
+      case 6: /* (vi) "... and column respectively" / "... and the last column"
+               *      (over the rows the column passes computed, 0..H-3) */
+        for (int r = 0; r <= H - 3; ++r) {
+          U_(r, 1) = U_(r, 0);
+          U_(r, W - 1) = U_(r, W - 2);
+        }
+        break;
+      default: { /* (vii) "the four elements of the bottom right corner are still
+                  * missing.  The third last value of the last column will be
+                  * copied to those elements" */
+        const float v = U_(H - 3, W - 1);
+        U_(H - 2, W - 2) = v;
+        U_(H - 2, W - 1) = v;
+        U_(H - 1, W - 2) = v;
+        U_(H - 1, W - 1) = v;
+      }
+    }
   }
 
   if (last_step < 8) return;
@@ -174,10 +195,19 @@ void oracle_sobel(const uint8_t *O, int W, int H, int32_t *pE) {
  * included); exact u64 sum; mean in double.
  * ------------------------------------------------------------------------- */
 void oracle_reduce(const int32_t *pE, int W, int H, uint64_t *S, double *mean) {
+  oracle_reduce_ex(pE, W, H, 0, S, mean);
+}
+
+/* flags & ORACLE_READ_INTERIOR_MEAN (R8 alternative): the mean over the
+ * (W-2)(H-2) body elements only (the frame is 0 either way, so S is equal). */
+void oracle_reduce_ex(const int32_t *pE, int W, int H, int flags, uint64_t *S, double *mean) {
   uint64_t s = 0;
   for (size_t p = 0; p < (size_t)W * H; ++p) s += (uint64_t)pE[p];
   *S = s;
-  *mean = (double)s / ((double)W * (double)H);
+  if (flags & ORACLE_READ_INTERIOR_MEAN)
+    *mean = (double)s / ((double)(W - 2) * (double)(H - 2));
+  else
+    *mean = (double)s / ((double)W * (double)H);
 }
 
 /* ---------------------------------------------------------------------------
@@ -189,9 +219,20 @@ void oracle_reduce(const int32_t *pE, int W, int H, uint64_t *S, double *mean) {
  * ------------------------------------------------------------------------- */
 void oracle_strength(const int32_t *pE, int n, double mean, float A, float gamma,
                      float *adj) {
+  oracle_strength_ex(pE, n, mean, A, gamma, 1.0f, 0, adj);
+}
+
+/* flags & ORACLE_READ_STRENGTH_EXP (R9 alternative, a saturating curve):
+ * adj = A * (1 - exp(-pE / (K*m))), K = the osc_scale parameter. */
+void oracle_strength_ex(const int32_t *pE, int n, double mean, float A, float gamma, float K,
+                        int flags, float *adj) {
   const double m = mean > 1.0 ? mean : 1.0;
-  for (int p = 0; p < n; ++p)
-    adj[p] = (float)((double)A * pow((double)pE[p] / m, (double)gamma));
+  for (int p = 0; p < n; ++p) {
+    if (flags & ORACLE_READ_STRENGTH_EXP)
+      adj[p] = (float)((double)A * (1.0 - exp(-(double)pE[p] / ((double)K * m))));
+    else
+      adj[p] = (float)((double)A * pow((double)pE[p] / m, (double)gamma));
+  }
 }
 
 /* ---------------------------------------------------------------------------
@@ -221,6 +262,13 @@ void oracle_preliminary(const float *adj, const float *E, const float *U, int n,
  * ------------------------------------------------------------------------- */
 void oracle_overshoot(const uint8_t *O, const float *P, const int32_t *pE, int W,
                       int H, double mean, float G, float K, float *F) {
+  oracle_overshoot_ex(O, P, pE, W, H, mean, G, K, 0, F);
+}
+
+/* flags & ORACLE_READ_OSC_CONST (R11 alternative): oscStrength = G for every
+ * element (no dependence on pEdge). */
+void oracle_overshoot_ex(const uint8_t *O, const float *P, const int32_t *pE, int W,
+                         int H, double mean, float G, float K, int flags, float *F) {
   const double m = mean > 1.0 ? mean : 1.0;
   for (int r = 0; r < H; ++r)
     for (int c = 0; c < W; ++c) {
@@ -239,7 +287,9 @@ void oracle_overshoot(const uint8_t *O, const float *P, const int32_t *pE, int W
         }
       const float fmx = (float)mx, fmn = (float)mn;
       const float osc =
-          (float)fmin(fmax((double)G * exp(-(double)pE[p] / ((double)K * m)), 0.0), 1.0);
+          (flags & ORACLE_READ_OSC_CONST)
+              ? G
+              : (float)fmin(fmax((double)G * exp(-(double)pE[p] / ((double)K * m)), 0.0), 1.0);
       if (pre > fmx) {
         const float osc_max = fmaf(osc, pre - fmx, fmx);
         F[p] = fminf(osc_max, 255.0f);
@@ -253,8 +303,13 @@ void oracle_overshoot(const uint8_t *O, const float *P, const int32_t *pE, int W
 }
 
 /* R14: round half to even (default FP environment) to 8 bits. */
-void oracle_output(const float *F, int n, uint8_t *out) {
-  for (int p = 0; p < n; ++p) out[p] = (uint8_t)nearbyintf(F[p]);
+void oracle_output(const float *F, int n, uint8_t *out) { oracle_output_ex(F, n, 0, out); }
+
+/* flags & ORACLE_READ_TRUNCATE (R14 alternative): the C cast, truncation
+ * toward zero (F is already in [0, 255]). */
+void oracle_output_ex(const float *F, int n, int flags, uint8_t *out) {
+  for (int p = 0; p < n; ++p)
+    out[p] = (flags & ORACLE_READ_TRUNCATE) ? (uint8_t)truncf(F[p]) : (uint8_t)nearbyintf(F[p]);
 }
 
 static int params_ok(float A, float gamma, float G, float K) {
@@ -266,9 +321,10 @@ static int params_ok(float A, float gamma, float G, float K) {
   return 1;
 }
 
-int oracle_sharpen(const uint8_t *O, int W, int H, float A, float gamma, float G,
-                   float K, uint8_t *out, uint64_t *S_out, double *mean_out) {
-  if (oracle_check_geometry(W, H) != 0 || !params_ok(A, gamma, G, K)) return -1;
+/* The pipeline on a W x H image with W, H multiples of 4 (R1), stages in the
+ * order of Fig. 1, each with the reading switches of `flags`. */
+static int sharpen_core(const uint8_t *O, int W, int H, float A, float gamma, float G, float K, int flags,
+                        uint8_t *out, uint64_t *S_out, double *mean_out) {
   const size_t n = (size_t)W * H;
   float *D = (float *)malloc(sizeof(float) * (n / 16));
   float *U = (float *)malloc(sizeof(float) * n);
@@ -281,20 +337,53 @@ int oracle_sharpen(const uint8_t *O, int W, int H, float A, float gamma, float G
   if (D && U && E && pE && adj && P && F) {
     uint64_t S;
     double mean;
-    oracle_downscale(O, W, H, D);              /* Fig. 1: downscale()  */
-    oracle_upscale(D, W, H, U);                /* Fig. 1: upscale()    */
+    oracle_downscale_ex(O, W, H, flags, D);    /* Fig. 1: downscale()  */
+    oracle_upscale_ex(D, W, H, flags, U);      /* Fig. 1: upscale()    */
     oracle_perror(O, U, (int)n, E);            /* Fig. 1: pError()     */
     oracle_sobel(O, W, H, pE);                 /* Fig. 1: Sharpness(): */
-    oracle_reduce(pE, W, H, &S, &mean);        /*   Sobel, reduction,  */
-    oracle_strength(pE, (int)n, mean, A, gamma, adj); /* strength,     */
-    oracle_preliminary(adj, E, U, (int)n, P);  /*   preliminary,       */
-    oracle_overshoot(O, P, pE, W, H, mean, G, K, F); /* overshoot      */
-    oracle_output(F, (int)n, out);
+    oracle_reduce_ex(pE, W, H, flags, &S, &mean);                 /* Sobel, reduction, */
+    oracle_strength_ex(pE, (int)n, mean, A, gamma, K, flags, adj); /* strength,         */
+    oracle_preliminary(adj, E, U, (int)n, P);                     /* preliminary,      */
+    oracle_overshoot_ex(O, P, pE, W, H, mean, G, K, flags, F);    /* overshoot         */
+    oracle_output_ex(F, (int)n, flags, out);
     if (S_out) *S_out = S;
     if (mean_out) *mean_out = mean;
     rc = 0;
   }
   free(D); free(U); free(E); free(pE); free(adj); free(P); free(F);
+  return rc;
+}
+
+int oracle_sharpen(const uint8_t *O, int W, int H, float A, float gamma, float G,
+                   float K, uint8_t *out, uint64_t *S_out, double *mean_out) {
+  if (oracle_check_geometry(W, H) != 0 || !params_ok(A, gamma, G, K)) return -1;
+  return sharpen_core(O, W, H, A, gamma, G, K, 0, out, S_out, mean_out);
+}
+
+/* General geometry (reading R1' in DESIGN.md):
+ * any W, H >= 5.  The image is extended to W4 x H4 (the next multiples of 4)
+ * by replicating its last column and last row, the pipeline runs on the
+ * extended image (so S and the mean are those of the extended image), and the
+ * output is its top-left W x H.  For W, H multiples of 4 this is exactly
+ * oracle_sharpen.  Rows are read / written with the given pitches (bytes). */
+int oracle_sharpen_ex(const uint8_t *O, int W, int H, int in_pitch, float A, float gamma, float G, float K,
+                      int flags, uint8_t *out, int out_pitch, uint64_t *S_out, double *mean_out) {
+  if (W < 5 || H < 5 || in_pitch < W || out_pitch < W || !params_ok(A, gamma, G, K)) return -1;
+  if (flags & ~ORACLE_READ_ALL) return -1;
+  const int W4 = (W + 3) / 4 * 4, H4 = (H + 3) / 4 * 4;
+  uint8_t *X = (uint8_t *)malloc((size_t)W4 * H4);
+  uint8_t *Y = (uint8_t *)malloc((size_t)W4 * H4);
+  int rc = -1;
+  if (X && Y) {
+    for (int r = 0; r < H4; ++r)
+      for (int c = 0; c < W4; ++c)
+        X[(size_t)r * W4 + c] = O[(size_t)(r < H ? r : H - 1) * in_pitch + (c < W ? c : W - 1)];
+    rc = sharpen_core(X, W4, H4, A, gamma, G, K, flags, Y, S_out, mean_out);
+    if (rc == 0)
+      for (int r = 0; r < H; ++r) memcpy(out + (size_t)r * out_pitch, Y + (size_t)r * W4, (size_t)W);
+  }
+  free(X);
+  free(Y);
   return rc;
 }
 

@@ -84,6 +84,34 @@ void oracle_output(const float *F, int n, uint8_t *out);
 int oracle_sharpen(const uint8_t *O, int W, int H, float A, float gamma, float G,
                    float K, uint8_t *out, uint64_t *S, double *mean);
 
+/* ---- Reading switches: the
+ * alternative readings of places where the paper is silent, as flags of the
+ * _ex functions (0 = the default readings above). */
+#define ORACLE_READ_INT_DOWNSCALE 1  /* R2:  D = floor(block sum / 16) (integer shift, L374)   */
+#define ORACLE_READ_COLUMN_WINS 2    /* R5:  border steps (i),(iii),(v),(ii),(iv),(vi),(vii)    */
+#define ORACLE_READ_INTERIOR_MEAN 4  /* R8:  mean = S / ((W-2)(H-2))                            */
+#define ORACLE_READ_STRENGTH_EXP 8   /* R9:  adj = A (1 - exp(-pE / (K m)))                     */
+#define ORACLE_READ_OSC_CONST 16     /* R11: oscStrength = G                                    */
+#define ORACLE_READ_TRUNCATE 32      /* R14: out = trunc(F)                                     */
+#define ORACLE_READ_ALL 63
+void oracle_downscale_ex(const uint8_t *O, int W, int H, int flags, float *D);
+void oracle_upscale_ex(const float *D, int W, int H, int flags, float *U);
+void oracle_upscale_steps_ex(const float *D, int W, int H, float *U, int last_step, int flags);
+void oracle_reduce_ex(const int32_t *pE, int W, int H, int flags, uint64_t *S, double *mean);
+void oracle_strength_ex(const int32_t *pE, int n, double mean, float A, float gamma, float K,
+                        int flags, float *adj);
+void oracle_overshoot_ex(const uint8_t *O, const float *P, const int32_t *pE, int W,
+                         int H, double mean, float G, float K, int flags, float *F);
+void oracle_output_ex(const float *F, int n, int flags, uint8_t *out);
+
+/* General geometry (reading R1'): any W, H >= 5,
+ * rows at in_pitch / out_pitch bytes.  The image is extended to the next
+ * multiples of 4 by replicating the last column and row, sharpened (with the
+ * reading switches `flags`), and cropped back to W x H; S / mean are those of
+ * the extended image.  Returns 0, or -1 on bad arguments. */
+int oracle_sharpen_ex(const uint8_t *O, int W, int H, int in_pitch, float A, float gamma, float G, float K,
+                      int flags, uint8_t *out, int out_pitch, uint64_t *S, double *mean);
+
 /* n frames [n][H][W], each exactly oracle_sharpen; frames split over
  * `threads` OpenMP threads (<=0: all).  sums may be NULL. */
 int oracle_sharpen_batch(const uint8_t *imgs, int n, int W, int H, float A,
