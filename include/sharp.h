@@ -16,6 +16,8 @@
  *    ("4096 x 4096 bytes").  A batch is dense [n][h][w].
  *  - Width and height must be multiples of 4 and >= 8 (R1: the downscaled
  *    matrix is width/4 x height/4, L130); otherwise SHARP_EINVAL.
+ *    (sharp_run_ex takes any size >= 5, strided / pitched / interleaved
+ *    layouts, in-place calls and the reading switches.)
  *  - Pointers may be device pointers (on the context's device), pinned host
  *    or pageable host memory; the library classifies them
  *    (cudaPointerGetAttributes).  Host pointers go through pinned staging with
@@ -114,6 +116,66 @@ int sharp_run_batch(sharp_ctx *ctx, const uint8_t *imgs, int n, int w, int h,
  * is not updated).  Used for graph capture / device-resident benchmarking. */
 int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int h,
                         const sharp_params *params, uint8_t *d_outs);
+
+/* ---- General geometry, layouts and reading switches (SURVEY.md sec. 8(f)
+ * NEXT 3 and 4; DESIGN.md sec. 3 R1' and the R2/R5/R8/R9/R11/R14 switches).
+ *
+ * sharp_layout describes where the pixels of a batch live (all in bytes):
+ * pixel (f, c, r, x) -- frame f, channel c, row r, column x -- is at
+ *   base + f * frame_stride + c + r * pitch + x * elem_stride.
+ * Zero fields take the dense defaults: elem_stride 1, pitch w * elem_stride,
+ * frame_stride pitch * h.  A NULL layout is all defaults.  Requirements:
+ * pitch >= w * elem_stride, frame_stride >= pitch * h, channels <= elem_stride.
+ * So an ROI of a bigger image is {pitch = the big image's pitch}, an
+ * interleaved C-channel image is {elem_stride = C} with channels = C, and a
+ * planar one is C frames.
+ *
+ * sharp_run_ex sharpens the n * channels single-channel images ("units")
+ * independently (each with its own pEdge mean: the method is
+ * defined on one 8-bit matrix, so colour is handled per channel) and writes
+ * them with out_layout.  Any w, h >= 5: when w or h is not a multiple of 4
+ * (R1: the downscaled matrix is w/4 x h/4, L130) the unit is extended to the
+ * next multiples of 4 by replicating its last column and last row, sharpened,
+ * and cropped back (reading R1'; sharp_get_batch_sums then reports S of the
+ * extended units).  In-place is allowed when imgs == outs with the same
+ * layout; any other overlap is SHARP_EINVAL.  Pixels outside the w x h crops
+ * (gaps between rows, other channels) are never modified.
+ *
+ * flags: reading switches, 0 = the default readings (bit-identical to
+ * sharp_run_batch).  Each selects the alternative reading of a place where the
+ * paper is silent; the CPU oracle implements the same switches.
+ *   SHARP_READ_INT_DOWNSCALE  R2:  D = floor(block sum / 16) (the shift of L374)
+ *   SHARP_READ_COLUMN_WINS    R5:  border column lines / copies after the row
+ *                                  copies (top-left 2x2 from the column line)
+ *   SHARP_READ_INTERIOR_MEAN  R8:  mean of pEdge over the (w-2)(h-2) body
+ *   SHARP_READ_STRENGTH_EXP   R9:  adj(p) = amount * (1 - exp(-p / (osc_scale * m)))
+ *   SHARP_READ_OSC_CONST      R11: oscStrength = osc_gain for every element
+ *   SHARP_READ_TRUNCATE       R14: truncate instead of round-half-even
+ * R8 / R9 / R11 only change the per-frame tables and run on every path; R2,
+ * R5 and R14 change per-pixel arithmetic and run on the two-pass and staged
+ * paths (SHARP_PATH_AUTO picks two-pass; SHARP_PATH_STEP returns
+ * SHARP_EUNSUPPORTED).  Unknown bits -> SHARP_EINVAL.
+ *
+ * Dense single-channel inputs with w, h multiples of 4 take exactly the
+ * sharp_run_batch path (host buffers pipelined, device buffers in one launch);
+ * everything else is gathered into dense scratch on the device (host buffers:
+ * their byte range is copied up first), run, and scattered back, one chunk of
+ * frames at a time.  Synchronous. */
+typedef struct {
+  size_t pitch;        /* bytes from one row to the next          (0 -> w * elem_stride) */
+  size_t frame_stride; /* bytes from one frame to the next        (0 -> pitch * h)       */
+  int elem_stride;     /* bytes from one pixel to the next in a row (0 -> 1)             */
+} sharp_layout;
+enum {
+  SHARP_READ_INT_DOWNSCALE = 1,
+  SHARP_READ_COLUMN_WINS = 2,
+  SHARP_READ_INTERIOR_MEAN = 4,
+  SHARP_READ_STRENGTH_EXP = 8,
+  SHARP_READ_OSC_CONST = 16,
+  SHARP_READ_TRUNCATE = 32
+};
+int sharp_run_ex(sharp_ctx *ctx, const uint8_t *imgs, const sharp_layout *in_layout, int n, int channels, int w,
+                 int h, const sharp_params *params, int flags, uint8_t *outs, const sharp_layout *out_layout);
 
 /* Statistics of the last completed call. */
 int sharp_get_stats(const sharp_ctx *ctx, sharp_stats *s);

@@ -43,6 +43,20 @@ class SharpStats(ctypes.Structure):
                 ("frames", ctypes.c_int), ("kernels", ctypes.c_int)]
 
 
+class SharpLayout(ctypes.Structure):
+    """Byte strides of a batch (include/sharp.h sharp_layout); 0 = dense default."""
+    _fields_ = [("pitch", ctypes.c_size_t), ("frame_stride", ctypes.c_size_t), ("elem_stride", ctypes.c_int)]
+
+
+# reading switches (include/sharp.h SHARP_READ_*; DESIGN.md sec. 3)
+SHARP_READ_INT_DOWNSCALE = 1   # R2
+SHARP_READ_COLUMN_WINS = 2     # R5
+SHARP_READ_INTERIOR_MEAN = 4   # R8
+SHARP_READ_STRENGTH_EXP = 8    # R9
+SHARP_READ_OSC_CONST = 16      # R11
+SHARP_READ_TRUNCATE = 32       # R14
+
+
 class SharpKernelTimes(ctypes.Structure):
     _fields_ = [("pass1_ms", ctypes.c_float), ("pass2_ms", ctypes.c_float),
                 ("pass1_launches", ctypes.c_int), ("pass2_launches", ctypes.c_int),
@@ -81,6 +95,8 @@ _SIGS = {
     "sharp_set_path": ([_P, _I], _I),
     "sharp_get_path": ([_P], _I),
     "sharp_get_stage_times": ([_P, ctypes.POINTER(ctypes.c_float), _I], _I),
+    "sharp_run_ex": ([_P, _P, ctypes.POINTER(SharpLayout), _I, _I, _I, _I, ctypes.POINTER(SharpParams), _I, _P,
+                      ctypes.POINTER(SharpLayout)], _I),
 }
 
 _lib = None
@@ -192,6 +208,57 @@ def sharp_run(ctx, img, w, h, params, out):
 
 def sharp_run_batch(ctx, imgs, n, w, h, params, outs):
     return _check(lib().sharp_run_batch(ctx, _addr(imgs), n, w, h, _pp(params), _addr(outs)), ctx)
+
+
+def _raw_addr(buf):
+    """Address of a (possibly strided) torch tensor / numpy array / int."""
+    if isinstance(buf, int):
+        return buf
+    if hasattr(buf, "data_ptr"):
+        return buf.data_ptr()
+    if hasattr(buf, "ctypes"):
+        return buf.ctypes.data
+    raise TypeError(f"unsupported buffer type {type(buf)}")
+
+
+def _layout(l):
+    if l is None or isinstance(l, SharpLayout):
+        return l
+    if isinstance(l, dict):
+        return SharpLayout(**l)
+    return SharpLayout(*l)
+
+
+def sharp_run_ex(ctx, imgs, in_layout, n, channels, w, h, params, flags, outs, out_layout):
+    """imgs / outs: base addresses (tensors or arrays: their first element);
+    layouts: SharpLayout, dict, tuple (pitch, frame_stride, elem_stride) or None."""
+    li, lo = _layout(in_layout), _layout(out_layout)
+    return _check(lib().sharp_run_ex(ctx, _raw_addr(imgs), ctypes.byref(li) if li is not None else None, n, channels,
+                                     w, h, _pp(params), int(flags), _raw_addr(outs),
+                                     ctypes.byref(lo) if lo is not None else None), ctx)
+
+
+def layout_of(t, channels_last=False):
+    """(n, channels, h, w, SharpLayout) of a uint8 tensor / array view:
+    [H, W], [N, H, W], or with channels_last=True [H, W, C] / [N, H, W, C]."""
+    shape = tuple(t.shape)
+    st = tuple(t.stride()) if hasattr(t, "stride") and callable(t.stride) else tuple(t.strides)
+    if channels_last:
+        if len(shape) == 3:
+            shape, st = (1,) + shape, (0,) + st
+        n, h, w, c = shape
+        fs, pitch, es, cs = st
+        if c > 1 and cs != 1:
+            raise ValueError("channels must be adjacent bytes (channel stride 1)")
+    else:
+        if len(shape) == 2:
+            shape, st = (1,) + shape, (0,) + st
+        n, h, w = shape
+        fs, pitch, es = st
+        c = 1
+    if n == 1:
+        fs = 0
+    return n, c, h, w, SharpLayout(pitch=pitch, frame_stride=fs, elem_stride=es)
 
 
 def sharp_enqueue_batch(ctx, d_imgs, n, w, h, params, d_outs):
@@ -382,6 +449,18 @@ class Sharpener:
         if out is None:
             out = self._like(imgs)
         sharp_run_batch(self.ctx, imgs, N, W, H, params, out)
+        return out
+
+    def run_ex(self, imgs, params=None, out=None, flags=0, channels_last=False):
+        """Any size >= 5, any strides (ROI views, interleaved channels with
+        channels_last=True), in-place (out=imgs), reading switches `flags`."""
+        n, c, h, w, li = layout_of(imgs, channels_last)
+        if out is None:
+            out = self._like(imgs)
+        n2, c2, h2, w2, lo = layout_of(out, channels_last)
+        if (n2, c2, h2, w2) != (n, c, h, w):
+            raise ValueError("out must have the shape of imgs")
+        sharp_run_ex(self.ctx, imgs, li, n, c, w, h, params, flags, out, lo)
         return out
 
     def enqueue_batch(self, d_imgs, d_outs, params=None):

@@ -5,6 +5,8 @@
 #include <cuda_fp16.h>
 #include <stdint.h>
 
+#include "kernels.h"
+
 namespace sharp {
 namespace dev {
 
@@ -185,6 +187,36 @@ __device__ __forceinline__ uint32_t pack4_rni_u8(float a, float b, float c, floa
       : "=r"(r)
       : "f"(a), "f"(b), "f"(c), "f"(d));
   return r;
+}
+
+// Truncate toward zero and saturate to [0, 255] (the R14 alternative).
+__device__ __forceinline__ uint32_t cvt_u8_rz(float a) {
+  uint32_t r;
+  asm("cvt.rzi.sat.u8.f32 %0, %1;" : "=r"(r) : "f"(a));
+  return r;
+}
+
+// ---------------------------------------------------------- per-frame tables
+// L174: the mean of pEdge over the W*H elements (R8), or over the (W-2)(H-2)
+// body (the R8 alternative); S is exact.
+__device__ __forceinline__ double frame_mean(unsigned long long S, int W, int H, int flags) {
+  return (flags & kReadInteriorMean) ? (double)S / ((double)(W - 2) * (double)(H - 2))
+                                     : (double)S / ((double)W * (double)H);
+}
+// {adj(p), osc(p)} for pEdge value p (f64, rounded once to f32; R9, R11, R15):
+//   adj = A (p / m)^gamma        (R9)   or A (1 - exp(-p / (K m)))   (R9 alternative)
+//   osc = clamp(G exp(-p / (K m)), 0, 1)   (R11)   or G               (R11 alternative)
+// with m = max(mean, 1).
+__device__ __forceinline__ float2 lut_entry(int p, double mean, const Params &prm) {
+  const double m = mean > 1.0 ? mean : 1.0;
+  const float adj = (prm.flags & kReadStrengthExp)
+                        ? (float)((double)prm.amount * (1.0 - exp(-(double)p / ((double)prm.osc_scale * m))))
+                        : (float)((double)prm.amount * pow((double)p / m, (double)prm.gamma));
+  const float osc = (prm.flags & kReadOscConst)
+                        ? prm.osc_gain
+                        : (float)fmin(fmax((double)prm.osc_gain * exp(-(double)p / ((double)prm.osc_scale * m)), 0.0),
+                                      1.0);
+  return make_float2(adj, osc);
 }
 
 // Packs 8 bytes (low byte of each word) into two words.

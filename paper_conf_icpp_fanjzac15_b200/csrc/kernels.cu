@@ -64,21 +64,26 @@ struct Block {  // 4 rows of words + the four D sums (16*D) of columns j0-1..j0+
   float S[4];
 };
 
+// S = 16 * D; with the R2 alternative (integer downscale) D = floor(sum / 16),
+// i.e. S = sum with its low 4 bits cleared.
 __device__ __forceinline__ void load_block(Block &B, const uint8_t *__restrict__ img, int W, int H, int k,
-                                           int c0, int lane) {
+                                           int c0, int lane, uint32_t smask) {
 #pragma unroll
   for (int a = 0; a < 4; ++a) B.r[a] = load_row(img, W, H, 4 * k + a, c0, lane);
-  B.S[0] = (float)blk4(B.r[0].pw, B.r[1].pw, B.r[2].pw, B.r[3].pw);
-  B.S[1] = (float)blk4(B.r[0].w0, B.r[1].w0, B.r[2].w0, B.r[3].w0);
-  B.S[2] = (float)blk4(B.r[0].w1, B.r[1].w1, B.r[2].w1, B.r[3].w1);
-  B.S[3] = (float)blk4(B.r[0].nw, B.r[1].nw, B.r[2].nw, B.r[3].nw);
+  B.S[0] = (float)(blk4(B.r[0].pw, B.r[1].pw, B.r[2].pw, B.r[3].pw) & smask);
+  B.S[1] = (float)(blk4(B.r[0].w0, B.r[1].w0, B.r[2].w0, B.r[3].w0) & smask);
+  B.S[2] = (float)(blk4(B.r[0].w1, B.r[1].w1, B.r[2].w1, B.r[3].w1) & smask);
+  B.S[3] = (float)(blk4(B.r[0].nw, B.r[1].nw, B.r[2].nw, B.r[3].nw) & smask);
 }
 
 // ------------------------------------------------------- upscale border (R4, R5)
 // Final value of U at a pixel of the 2-pixel ring (last writer of steps
 // i..vii of L140-L142).  Sc = 16*D of the current D row block (row k) for
 // columns j0-1..j0+2, Sn = the next D row (k+1); j0 = c0/4; r = 4k + a'.
-__device__ __forceinline__ float ring_u(int r, int c, int W, int H, int j0, const float (&Sc)[4], const float (&Sn)[4]) {
+// col_wins: the R5 alternative (column work after the row work: the top-left
+// 2x2 keeps the column line's values instead of D[0][0]).
+__device__ __forceinline__ float ring_u(int r, int c, int W, int H, int j0, const float (&Sc)[4], const float (&Sn)[4],
+                                        bool col_wins) {
   const int w = W >> 2, h = H >> 2;
   auto col = [&](int j) { return j - j0 + 1; };  // index into Sc/Sn
   if (r >= H - 2 && c >= W - 2) {                 // (vii): third last of last column = D[h-1][w-1]
@@ -86,7 +91,7 @@ __device__ __forceinline__ float ring_u(int r, int c, int W, int H, int j0, cons
   }
   if ((c <= 1 || c >= W - 2) && r <= H - 3) {     // (vi)/(ii)/(iv): column lines
     const int j = (c <= 1) ? 0 : w - 1;
-    if (c <= 1 && r <= 1) return __fmul_rn(Sc[col(0)], 1.0f / 16.0f);  // (v) then (vi): D[0][0]
+    if (c <= 1 && r <= 1 && !col_wins) return __fmul_rn(Sc[col(0)], 1.0f / 16.0f);  // (v) then (vi): D[0][0]
     const int rr = (r == H - 3) ? H - 4 : r;   // third last <- fourth last
     const int k = rr & 3;                      // rr>>2 == current D row (rr in the block of r)
     return line_val(Sc[col(j)], Sn[col(j)], k);
@@ -165,16 +170,9 @@ __global__ void __launch_bounds__(kThreads) edge_sum_kernel(const uint8_t *__res
   // Stage 2 (last-block-done): mean and the per-frame lookup tables.
   __threadfence();
   const unsigned long long S = atomicAdd(&sums[f], 0ull);
-  const double mean = (double)S / ((double)W * (double)H);
-  const double m = mean > 1.0 ? mean : 1.0;
-  for (int p = threadIdx.x; p < kLutSize; p += kThreads) {
-    float adj = 0.0f, osc = 0.0f;
-    if (p <= 1530) {
-      adj = (float)((double)prm.amount * pow((double)p / m, (double)prm.gamma));
-      osc = (float)fmin(fmax((double)prm.osc_gain * exp(-(double)p / ((double)prm.osc_scale * m)), 0.0), 1.0);
-    }
-    luts[(size_t)f * kLutSize + p] = make_float2(adj, osc);
-  }
+  const double mean = frame_mean(S, W, H, prm.flags);
+  for (int p = threadIdx.x; p < kLutSize; p += kThreads)
+    luts[(size_t)f * kLutSize + p] = p <= 1530 ? lut_entry(p, mean, prm) : make_float2(0.0f, 0.0f);
   if (threadIdx.x == 0) {
     means[f] = mean;
     counters[f] = 0u;  // re-arm for the next launch
@@ -187,7 +185,7 @@ __global__ void __launch_bounds__(kThreads) edge_sum_kernel(const uint8_t *__res
 __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__restrict__ imgs, int W, int H,
                                                            int tiles_x, int tiles_y,
                                                            const float2 *__restrict__ luts,
-                                                           uint8_t *__restrict__ outs) {
+                                                           uint8_t *__restrict__ outs, int flags) {
   __shared__ float2 lut[kLutSize];
   const int f = blockIdx.y;
   for (int i = threadIdx.x; i < kLutSize; i += kThreads) lut[i] = luts[(size_t)f * kLutSize + i];
@@ -207,14 +205,16 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
   uint8_t *out = outs + (size_t)f * W * H;
   const bool ring_cols = (c0 < 2) || (c0 + kPx > W - 2);
 
+  const uint32_t smask = (flags & kReadIntDownscale) ? ~15u : ~0u;
+  const bool col_wins = (flags & kReadColumnWins) != 0, trunc = (flags & kReadTruncate) != 0;
   Block prev, cur, next;
-  load_block(prev, img, W, H, (R0 >> 2) - 1, c0, lane);
-  load_block(cur, img, W, H, R0 >> 2, c0, lane);
+  load_block(prev, img, W, H, (R0 >> 2) - 1, c0, lane, smask);
+  load_block(cur, img, W, H, R0 >> 2, c0, lane, smask);
   RowD ra = derive<true>(prev.r[3]);
   RowD rb = derive<true>(cur.r[0]);
 
   for (int k = R0 >> 2; 4 * k < R1; ++k) {
-    load_block(next, img, W, H, k + 1, c0, lane);
+    load_block(next, img, W, H, k + 1, c0, lane, smask);
 #pragma unroll
     for (int a = 0; a < 4; ++a) {
       const int r = 4 * k + a;
@@ -272,7 +272,7 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
 #pragma unroll
           for (int x = 0; x < 8; ++x) {
             const int c = c0 + x;
-            if (c < W && (r < 2 || r >= H - 2 || c < 2 || c >= W - 2)) NU[x] = -ring_u(r, c, W, H, j0, Sc, Sn);
+            if (c < W && (r < 2 || r >= H - 2 || c < 2 || c >= W - 2)) NU[x] = -ring_u(r, c, W, H, j0, Sc, Sn, col_wins);
           }
         }
         uint32_t o[8];
@@ -291,7 +291,7 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
           const float mxf = add_f32_f16(mx_h, 0.0f), mnf = add_f32_f16(mn_h, 0.0f);
           const float t = fminf(fmaxf(P, mnf), mxf);                         // Fig. 8 branch target
           const float F = __fmaf_rn(L.y, __fsub_rn(P, t), t);                // osc max / osc min / P
-          o[x] = cvt_u8(F);                                                  // clamp [0,255], RNE
+          o[x] = trunc ? cvt_u8_rz(F) : cvt_u8(F);                           // clamp [0,255], RNE (R14)
         }
         const uint32_t o0 = prmt(prmt(o[0], o[1], 0x0040), prmt(o[2], o[3], 0x0040), 0x5410);
         const uint32_t o1 = prmt(prmt(o[4], o[5], 0x0040), prmt(o[6], o[7], 0x0040), 0x5410);
@@ -324,11 +324,11 @@ cudaError_t launch_edge_sum(const uint8_t *imgs, int n, int W, int H, const Para
   return cudaGetLastError();
 }
 
-cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts, uint8_t *outs,
+cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts, uint8_t *outs, int flags,
                            cudaStream_t stream) {
   int tx, ty, ctas;
   geometry(W, H, tx, ty, ctas);
-  sharpen_kernel<<<dim3(ctas, n), kThreads, 0, stream>>>(imgs, W, H, tx, ty, luts, outs);
+  sharpen_kernel<<<dim3(ctas, n), kThreads, 0, stream>>>(imgs, W, H, tx, ty, luts, outs, flags);
   return cudaGetLastError();
 }
 

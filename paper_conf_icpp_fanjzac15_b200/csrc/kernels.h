@@ -11,7 +11,19 @@ constexpr int kLutSize = 1536;
 
 struct Params {
   float amount, gamma, osc_gain, osc_scale;
+  int flags = 0;  // reading switches, include/sharp.h SHARP_READ_*
 };
+// Reading switches (values of include/sharp.h SHARP_READ_*).
+constexpr int kReadIntDownscale = 1;   // R2:  D = floor(block sum / 16)
+constexpr int kReadColumnWins = 2;     // R5:  border column work after the row work
+constexpr int kReadInteriorMean = 4;   // R8:  mean over the (W-2)(H-2) body
+constexpr int kReadStrengthExp = 8;    // R9:  adj = A (1 - exp(-p / (K m)))
+constexpr int kReadOscConst = 16;      // R11: oscStrength = G
+constexpr int kReadTruncate = 32;      // R14: truncating output conversion
+constexpr int kReadAll = 63;
+// Switches that change per-pixel arithmetic (only the two-pass and staged
+// paths implement them; the step kernel handles the LUT-only ones).
+constexpr int kReadPerPixel = kReadIntDownscale | kReadColumnWins | kReadTruncate;
 
 // Pass 1 (Sobel + reduction + LUT): for frames [0, n) of `imgs` (dense
 // [n][H][W]) accumulates S into sums[frame_base + f] (must be zero on entry),
@@ -24,7 +36,16 @@ cudaError_t launch_edge_sum(const uint8_t *imgs, int n, int W, int H, const Para
 // Pass 2 (fused downscale/upscale/pError/Sobel/min-max/strength/preliminary/
 // overshoot/output): frames [0, n) with the per-frame LUTs of pass 1.
 cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float2 *luts,
-                           uint8_t *outs, cudaStream_t stream);
+                           uint8_t *outs, int flags, cudaStream_t stream);
+
+// General layouts (layout.cu): units u = f * C + c
+// (frame f, channel c) of a strided source -> dense [units][H4][W4] with the
+// last column / row replicated (R1'), and back (top-left w x h only).
+cudaError_t launch_gather(const uint8_t *src, size_t frame_stride, size_t pitch, int elem_stride, int C, int w,
+                          int h, int W4, int H4, int units, uint8_t *dst, cudaStream_t st);
+cudaError_t launch_scatter(const uint8_t *src, int W4, int H4, int units, int w, int h, uint8_t *dst,
+                           size_t frame_stride, size_t pitch, int elem_stride, int C, cudaStream_t st);
+cudaError_t preload_layout();
 
 // TMA-staged, persistent, dynamically scheduled kernel (kernels_tma.cu) for a
 // whole batch in ONE launch (pass 1, per-frame LUT build and pass 2 as tasks

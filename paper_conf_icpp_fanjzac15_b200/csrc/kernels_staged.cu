@@ -16,13 +16,14 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include "device_common.cuh"
 #include "kernels.h"
 
 namespace sharp {
 namespace {
 
 // ---------------------------------------------------------------- K1
-__global__ void st_downscale(const uint8_t *__restrict__ O, int W, int h, int w, float *__restrict__ D) {
+__global__ void st_downscale(const uint8_t *__restrict__ O, int W, int h, int w, int flags, float *__restrict__ D) {
   const int j = blockIdx.x * blockDim.x + threadIdx.x, i = blockIdx.y;
   if (j >= w || i >= h) return;
   unsigned s = 0;
@@ -30,7 +31,8 @@ __global__ void st_downscale(const uint8_t *__restrict__ O, int W, int h, int w,
     const uint32_t v = *reinterpret_cast<const uint32_t *>(O + (size_t)(4 * i + a) * W + 4 * j);
     s += (v & 0xff) + ((v >> 8) & 0xff) + ((v >> 16) & 0xff) + (v >> 24);
   }
-  D[(size_t)i * w + j] = __fmul_rn((float)s, 1.0f / 16.0f);  // mean of the 4x4 block (R2, exact)
+  // mean of the 4x4 block (R2, exact), or the integer shift s >> 4 (the R2 alternative, L374)
+  D[(size_t)i * w + j] = (flags & kReadIntDownscale) ? (float)(s >> 4) : __fmul_rn((float)s, 1.0f / 16.0f);
 }
 
 // ---------------------------------------------------------------- K2
@@ -46,27 +48,34 @@ __device__ __forceinline__ float line_at(const float *v, size_t stride, int n, i
   return k == 0 ? v[(size_t)j * stride] : lerp4(v[(size_t)j * stride], v[(size_t)(j + 1) * stride], k);
 }
 // One CTA walks the steps (i)..(vii) of L140-L142 in order (the border is
-// 4(W+H) elements; __syncthreads orders the overlapping steps).
-__global__ void st_border(const float *__restrict__ D, int W, int H, int w, int h, float *__restrict__ U) {
+// 4(W+H) elements; __syncthreads orders the overlapping steps).  With the R5
+// alternative the row copies (v) run before the column lines (ii), (iv).
+__global__ void st_border(const float *__restrict__ D, int W, int H, int w, int h, int flags,
+                          float *__restrict__ U) {
   const int t = threadIdx.x, nt = blockDim.x;
+  const bool col_wins = (flags & kReadColumnWins) != 0;
   // (i) row 0 and (iii) row H-2: lines of D rows 0 and h-1 over columns 0..W-3
   for (int c = t; c <= W - 3; c += nt) {
     U[c] = line_at(D, 1, W, c);
     U[(size_t)(H - 2) * W + c] = line_at(D + (size_t)(h - 1) * w, 1, W, c);
   }
   __syncthreads();
-  // (ii) column 0 and (iv) column W-2: lines of D columns 0 and w-1 over rows 0..H-3
-  for (int r = t; r <= H - 3; r += nt) {
-    U[(size_t)r * W] = line_at(D, (size_t)w, H, r);
-    U[(size_t)r * W + W - 2] = line_at(D + (w - 1), (size_t)w, H, r);
+  for (int pass = 0; pass < 2; ++pass) {
+    if ((pass == 0) != col_wins) {
+      // (ii) column 0 and (iv) column W-2: lines of D columns 0 and w-1 over rows 0..H-3
+      for (int r = t; r <= H - 3; r += nt) {
+        U[(size_t)r * W] = line_at(D, (size_t)w, H, r);
+        U[(size_t)r * W + W - 2] = line_at(D + (w - 1), (size_t)w, H, r);
+      }
+    } else {
+      // (v) copy row 0 -> 1 and row H-2 -> H-1 over columns 0..W-3
+      for (int c = t; c <= W - 3; c += nt) {
+        U[(size_t)W + c] = U[c];
+        U[(size_t)(H - 1) * W + c] = U[(size_t)(H - 2) * W + c];
+      }
+    }
+    __syncthreads();
   }
-  __syncthreads();
-  // (v) copy row 0 -> 1 and row H-2 -> H-1 over columns 0..W-3
-  for (int c = t; c <= W - 3; c += nt) {
-    U[(size_t)W + c] = U[c];
-    U[(size_t)(H - 1) * W + c] = U[(size_t)(H - 2) * W + c];
-  }
-  __syncthreads();
   // (vi) copy column 0 -> 1 and column W-2 -> W-1 over rows 0..H-3
   for (int r = t; r <= H - 3; r += nt) {
     U[(size_t)r * W + 1] = U[(size_t)r * W];
@@ -133,24 +142,20 @@ __global__ void st_reduce(const uint16_t *__restrict__ pE, size_t n, unsigned lo
 // Per-pixel brightness strength (the "many exponentiations" of L232):
 // adj = A (p / m)^gamma, osc = clamp(G exp(-p / (K m)), 0, 1), f64 rounded
 // once to f32 (R9, R11, R15); thread (0,0) also stores the mean (L174, R8).
-__global__ void st_strength(const uint16_t *__restrict__ pE, size_t n, const unsigned long long *S, double npx,
+__global__ void st_strength(const uint16_t *__restrict__ pE, size_t n, const unsigned long long *S, int W, int H,
                             Params prm, float2 *__restrict__ ao, double *mean_out) {
-  const double mean = (double)*S / npx;
-  const double m = mean > 1.0 ? mean : 1.0;
+  const double mean = dev::frame_mean(*S, W, H, prm.flags);
   const size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
   if (k == 0) *mean_out = mean;
   if (k >= n) return;
-  const double p = (double)pE[k];
-  const float adj = (float)((double)prm.amount * pow(p / m, (double)prm.gamma));
-  const float osc = (float)fmin(fmax((double)prm.osc_gain * exp(-p / ((double)prm.osc_scale * m)), 0.0), 1.0);
-  ao[k] = make_float2(adj, osc);
+  ao[k] = dev::lut_entry(pE[k], mean, prm);
 }
 
 // ---------------------------------------------------------------- K7
 // pError E = O - U (L148, R6), preliminary P = fma(adj, E, U) (L178, R10),
 // overshoot control of Fig. 8 (L180-L212, R11-R13), RNE to 8 bits (R14).
 __global__ void st_sharpen(const uint8_t *__restrict__ O, const float *__restrict__ U,
-                           const float2 *__restrict__ ao, int W, int H, uint8_t *__restrict__ out) {
+                           const float2 *__restrict__ ao, int W, int H, int flags, uint8_t *__restrict__ out) {
   const int c = blockIdx.x * blockDim.x + threadIdx.x, r = blockIdx.y;
   if (c >= W || r >= H) return;
   const size_t k = (size_t)r * W + c;
@@ -174,7 +179,7 @@ __global__ void st_sharpen(const uint8_t *__restrict__ O, const float *__restric
     else if (P < mnf) F = fmaxf(__fmaf_rn(s.y, __fsub_rn(P, mnf), mnf), 0.0f);   // osc min
     else F = fminf(fmaxf(P, 0.0f), 255.0f);
   }
-  out[k] = (uint8_t)__float2int_rn(F);
+  out[k] = (uint8_t)((flags & kReadTruncate) ? __float2int_rz(F) : __float2int_rn(F));  // R14
 }
 
 }  // namespace
@@ -198,10 +203,10 @@ cudaError_t launch_staged(const uint8_t *in, int W, int H, const Params &p, void
   const int tb = 256;
   cudaError_t e;
   timer.begin(kStageDownscale, st);
-  st_downscale<<<dim3((w + tb - 1) / tb, h), tb, 0, st>>>(in, W, h, w, D);
+  st_downscale<<<dim3((w + tb - 1) / tb, h), tb, 0, st>>>(in, W, h, w, p.flags, D);
   timer.end(kStageDownscale, st);
   timer.begin(kStageBorder, st);
-  st_border<<<1, 1024, 0, st>>>(D, W, H, w, h, U);
+  st_border<<<1, 1024, 0, st>>>(D, W, H, w, h, p.flags, U);
   timer.end(kStageBorder, st);
   timer.begin(kStageCenter, st);
   st_center<<<dim3((W - 4 + tb - 1) / tb, H - 4), tb, 0, st>>>(D, W, H, w, U);
@@ -214,10 +219,10 @@ cudaError_t launch_staged(const uint8_t *in, int W, int H, const Params &p, void
   st_reduce<<<148 * 8, 256, 0, st>>>(pE, px, sum);
   timer.end(kStageReduce, st);
   timer.begin(kStageStrength, st);
-  st_strength<<<(unsigned)((px + tb - 1) / tb), tb, 0, st>>>(pE, px, sum, (double)W * (double)H, p, ao, mean);
+  st_strength<<<(unsigned)((px + tb - 1) / tb), tb, 0, st>>>(pE, px, sum, W, H, p, ao, mean);
   timer.end(kStageStrength, st);
   timer.begin(kStageSharpen, st);
-  st_sharpen<<<dim3((W + tb - 1) / tb, H), tb, 0, st>>>(in, U, ao, W, H, out);
+  st_sharpen<<<dim3((W + tb - 1) / tb, H), tb, 0, st>>>(in, U, ao, W, H, p.flags, out);
   timer.end(kStageSharpen, st);
   return cudaGetLastError();
 }

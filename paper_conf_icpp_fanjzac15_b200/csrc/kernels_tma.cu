@@ -778,20 +778,14 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       // LUT task: entries k = q*128 .. q*128+127 (pEdge p = 2k) of frame f
       // (R9, R11; f64, one rounding)
       const int f = d.y, k = d.z * kLutPerTask + threadIdx.x, p = 2 * k;
-      // L174: mean of pEdge over all W*H elements (R8), from the exact sum.
+      // L174: mean of pEdge (R8), from the exact sum.
       const unsigned long long S = stage_sum[b];
-      const double mean = (double)S / ((double)g.W * (double)g.H);
+      const double mean = frame_mean(S, g.W, g.H, sp.prm.flags);
       if (p == 0) {
         sp.sums[f] = S;
         sp.means[f] = mean;
       }
-      const double m = mean > 1.0 ? mean : 1.0;
-      float adj = 0.0f, osc = 0.0f;
-      if (p <= 1530) {
-        adj = (float)((double)sp.prm.amount * pow((double)p / m, (double)sp.prm.gamma));
-        osc = (float)fmin(fmax((double)sp.prm.osc_gain * exp(-(double)p / ((double)sp.prm.osc_scale * m)), 0.0), 1.0);
-      }
-      sp.luts[(size_t)f * kLutSize + k] = make_float2(adj, osc);
+      sp.luts[(size_t)f * kLutSize + k] = p <= 1530 ? lut_entry(p, mean, sp.prm) : make_float2(0.0f, 0.0f);
       __threadfence();
       __syncwarp();
       if (lane == 0) atomicAdd(&sp.lut_done[f], 1u);

@@ -56,6 +56,9 @@ struct sharp_ctx {
   unsigned int *lut_done = nullptr;   // per frame: finished LUT-task warps (batch kernel)
   unsigned long long *acc = nullptr;  // per frame: pass-1 arrivals << 40 | partial sum (batch kernel)
   float2 *luts = nullptr;             // per frame lookup tables (batch kernel)
+  // general layouts (sharp_run_ex): dense padded in / out, device copies of host byte ranges
+  uint8_t *gx_in = nullptr, *gx_out = nullptr, *gx_src = nullptr, *gx_dst = nullptr;
+  size_t gx_cap = 0, gx_out_cap = 0, gx_src_cap = 0, gx_dst_cap = 0;
   int last_frames = 0;
   sharp_stats stats{};
   // profiling: event pairs around launches (kind 1 = pass 1, 2 = pass 2,
@@ -308,10 +311,13 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
     }
     return SHARP_OK;
   }
-  const bool tma_ok = sharp::tma_supported(din, dout, w, h);
+  // The step kernel implements the LUT-only reading switches; R2 / R5 / R14
+  // change per-pixel arithmetic and run on the two-pass path.
+  const bool tma_ok = sharp::tma_supported(din, dout, w, h) && !(prm.flags & sharp::kReadPerPixel);
   if (ctx->path == SHARP_PATH_STEP && !tma_ok)
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
-                   "SHARP_PATH_STEP needs w % 16 == 0, 16-byte aligned input, 8-byte aligned output, w*h <= 2^29");
+                   "SHARP_PATH_STEP needs w % 16 == 0, 16-byte aligned input, 8-byte aligned output, w*h <= 2^29 "
+                   "and no per-pixel reading switch (R2, R5, R14)");
   const bool tma = (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) && tma_ok;
   if (tma) {  // the whole batch in one persistent launch
     sharp::BatchLaunch a;
@@ -338,20 +344,20 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
       return sharp::launch_edge_sum(ci, cn, w, h, prm, ctx->sums + frame_base + f0, slot.counters, slot.luts,
                                     ctx->means + frame_base + f0, st);
     }));
-    CK(timed(ctx, st, 2, px, [&] { return sharp::launch_sharpen(ci, cn, w, h, slot.luts, co, st); }));
+    CK(timed(ctx, st, 2, px, [&] { return sharp::launch_sharpen(ci, cn, w, h, slot.luts, co, prm.flags, st); }));
     *launches += sharp::kLaunchesPerChunk;
   }
   return SHARP_OK;
 }
 
 int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp_params *pp, uint8_t *out,
-             bool async) {
+             bool async, int flags = 0) {
   int rc = validate(ctx, in, out, n, w, h, pp);
   if (rc) return rc;
   sharp_params p;
   if (pp) p = *pp;
   else sharp_default_params(&p);
-  const sharp::Params prm{p.amount, p.gamma, p.osc_gain, p.osc_scale};
+  const sharp::Params prm{p.amount, p.gamma, p.osc_gain, p.osc_scale, flags};
   Kind kin, kout;
   if ((rc = classify(ctx, in, &kin)) || (rc = classify(ctx, out, &kout))) return rc;
   if (async && (kin != kDevice || kout != kDevice))
@@ -439,6 +445,144 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   ctx->stats.total_ms =
       std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return SHARP_OK;
+}
+
+
+// ---- General layouts (R1').
+struct Layout {
+  size_t pitch, fs;
+  int es;
+};
+
+bool layout_of(const sharp_layout *l, int w, int h, Layout *o) {
+  o->es = (l && l->elem_stride > 0) ? l->elem_stride : 1;
+  o->pitch = (l && l->pitch) ? l->pitch : (size_t)w * o->es;
+  o->fs = (l && l->frame_stride) ? l->frame_stride : o->pitch * h;
+  return o->pitch >= (size_t)w * o->es && o->fs >= o->pitch * (size_t)h;
+}
+
+// Bytes from the first to one past the last byte a layout touches.
+size_t layout_span(const Layout &L, int n, int C, int w, int h) {
+  return (size_t)(n - 1) * L.fs + (size_t)(h - 1) * L.pitch + (size_t)(w - 1) * L.es + (size_t)C;
+}
+
+int grow(sharp_ctx *ctx, uint8_t **buf, size_t *cap, size_t need) {
+  if (need <= *cap) return SHARP_OK;
+  CK(cudaStreamSynchronize(ctx->stream));
+  cudaFree(*buf);
+  *buf = nullptr;
+  *cap = 0;
+  CK(cudaMalloc(buf, need));
+  *cap = need;
+  return SHARP_OK;
+}
+
+constexpr size_t kGeneralChunkBytes = 256u << 20;  // dense padded bytes per chunk (each of in / out)
+
+int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int C, int w, int h,
+                const sharp::Params &prm, uint8_t *out, const Layout &Lo, Kind kin, Kind kout) {
+  const int W4 = (w + 3) & ~3, H4 = (h + 3) & ~3;
+  const size_t ub = (size_t)W4 * H4;
+  const int fpc = (int)std::max<size_t>(1, std::min<size_t>((size_t)n, kGeneralChunkBytes / (ub * C)));
+  const size_t units_all = (size_t)n * C;
+  int rc;
+  if ((rc = ensure_frames(ctx, units_all))) return rc;
+  const size_t cu_max = (size_t)fpc * C;
+  const size_t chunk = chunk_frames(ctx, ub, (int)cu_max);
+  if ((rc = ensure_slots(ctx, chunk, ub, false))) return rc;
+  if ((rc = ensure_task_counters(ctx, 2))) return rc;
+  if ((rc = grow(ctx, &ctx->gx_in, &ctx->gx_cap, cu_max * ub))) return rc;
+  if ((rc = grow(ctx, &ctx->gx_out, &ctx->gx_out_cap, cu_max * ub))) return rc;
+  int launches = 0;
+  CK(cudaEventRecord(ctx->ev_start, ctx->stream));
+  for (int f0 = 0; f0 < n; f0 += fpc) {
+    const int fn = std::min(fpc, n - f0), units = fn * C;
+    const size_t u0 = (size_t)f0 * C;
+    // source bytes of frames [f0, f0 + fn) on the device
+    const uint8_t *src = in + (size_t)f0 * Li.fs;
+    if (kin != kDevice) {
+      const size_t span = layout_span(Li, fn, C, w, h);
+      if ((rc = grow(ctx, &ctx->gx_src, &ctx->gx_src_cap, span))) return rc;
+      CK(cudaMemcpyAsync(ctx->gx_src, src, span, cudaMemcpyHostToDevice, ctx->stream));
+      src = ctx->gx_src;
+    }
+    CK(sharp::launch_gather(src, Li.fs, Li.pitch, Li.es, C, w, h, W4, H4, units, ctx->gx_in, ctx->stream));
+    CK(cudaMemsetAsync(ctx->sums + u0, 0, units * sizeof(unsigned long long), ctx->stream));
+    CK(cudaMemsetAsync(ctx->lut_done + u0, 0, units * sizeof(unsigned int), ctx->stream));
+    CK(cudaMemsetAsync(ctx->acc + u0, 0, units * sizeof(unsigned long long), ctx->stream));
+    CK(cudaMemsetAsync(ctx->tcounters, 0, sizeof(unsigned int), ctx->stream));
+    if ((rc = enqueue_device(ctx, ctx->gx_in, units, W4, H4, prm, ctx->gx_out, ctx->stream, ctx->slots[0],
+                             std::min(chunk, (size_t)units), u0, &launches, ctx->tcounters)))
+      return rc;
+    // the w x h crops into the caller's layout (a host destination goes
+    // through a device copy of its byte range, so bytes between the pixels
+    // keep their values)
+    uint8_t *dst = out + (size_t)f0 * Lo.fs;
+    if (kout == kDevice) {
+      CK(sharp::launch_scatter(ctx->gx_out, W4, H4, units, w, h, dst, Lo.fs, Lo.pitch, Lo.es, C, ctx->stream));
+    } else {
+      const size_t span = layout_span(Lo, fn, C, w, h);
+      if ((rc = grow(ctx, &ctx->gx_dst, &ctx->gx_dst_cap, span))) return rc;
+      CK(cudaMemcpyAsync(ctx->gx_dst, dst, span, cudaMemcpyHostToDevice, ctx->stream));
+      CK(sharp::launch_scatter(ctx->gx_out, W4, H4, units, w, h, ctx->gx_dst, Lo.fs, Lo.pitch, Lo.es, C,
+                               ctx->stream));
+      CK(cudaMemcpyAsync(dst, ctx->gx_dst, span, cudaMemcpyDeviceToHost, ctx->stream));
+    }
+    launches += 2;
+    CK(cudaStreamSynchronize(ctx->stream));  // host ranges / scratch are reused by the next chunk
+  }
+  CK(cudaEventRecord(ctx->ev_stop, ctx->stream));
+  CK(cudaEventSynchronize(ctx->ev_stop));
+  float ms = 0.0f;
+  CK(cudaEventElapsedTime(&ms, ctx->ev_start, ctx->ev_stop));
+  unsigned long long s0 = 0;
+  double m0 = 0.0;
+  CK(cudaMemcpy(&s0, ctx->sums, sizeof(s0), cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(&m0, ctx->means, sizeof(m0), cudaMemcpyDeviceToHost));
+  ctx->last_frames = (int)units_all;
+  ctx->stats.frames = (int)units_all;
+  ctx->stats.kernels = launches;
+  ctx->stats.edge_sum = s0;
+  ctx->stats.edge_mean = m0;
+  ctx->stats.device_ms = ms;
+  ctx->stats.total_ms = ms;
+  return SHARP_OK;
+}
+
+int run_ex_impl(sharp_ctx *ctx, const uint8_t *in, const sharp_layout *lin, int n, int C, int w, int h,
+                const sharp_params *pp, int flags, uint8_t *out, const sharp_layout *lout) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  if (!in || !out) return set_err(ctx, SHARP_EINVAL, "%s", "NULL image pointer");
+  if (n < 1 || C < 1) return set_err(ctx, SHARP_EINVAL, "%s", "n < 1 or channels < 1");
+  if (w < 5 || h < 5) return set_err(ctx, SHARP_EINVAL, "%s", "width and height must be >= 5 (R1')");
+  if (w > 65532 || h > 65532 || (long long)((w + 3) & ~3) * ((h + 3) & ~3) >= (1ll << 31))
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "image larger than 2^31 pixels");
+  if (flags & ~sharp::kReadAll) return set_err(ctx, SHARP_EINVAL, "%s", "unknown reading switch");
+  if (pp && !params_ok(*pp)) return set_err(ctx, SHARP_EINVAL, "%s", "parameter out of range or not finite");
+  Layout Li, Lo;
+  if (!layout_of(lin, w, h, &Li) || !layout_of(lout, w, h, &Lo))
+    return set_err(ctx, SHARP_EINVAL, "%s", "layout: pitch < w * elem_stride or frame_stride < pitch * h");
+  if (C > 1 && (C > Li.es || C > Lo.es))
+    return set_err(ctx, SHARP_EINVAL, "%s", "channels > elem_stride (interleaved channels overlap)");
+  const bool dense = C == 1 && Li.es == 1 && Lo.es == 1 && Li.pitch == (size_t)w && Lo.pitch == (size_t)w &&
+                     Li.fs == (size_t)w * h && Lo.fs == (size_t)w * h && !(w & 3) && !(h & 3) && w >= 8 && h >= 8;
+  const uintptr_t a = (uintptr_t)in, b = (uintptr_t)out;
+  const size_t sa = layout_span(Li, n, C, w, h), sb = layout_span(Lo, n, C, w, h);
+  const bool overlap = a < b + sb && b < a + sa;
+  const bool same = a == b && Li.pitch == Lo.pitch && Li.fs == Lo.fs && Li.es == Lo.es;
+  if (overlap && !same)
+    return set_err(ctx, SHARP_EINVAL, "%s", "input and output overlap without being the same layout (in-place)");
+  if (dense && !overlap) return run_impl(ctx, in, n, w, h, pp, out, false, flags);
+  sharp_params p;
+  if (pp) p = *pp;
+  else sharp_default_params(&p);
+  const sharp::Params prm{p.amount, p.gamma, p.osc_gain, p.osc_scale, flags};
+  Kind kin, kout;
+  int rc;
+  if ((rc = classify(ctx, in, &kin)) || (rc = classify(ctx, out, &kout))) return rc;
+  CK(cudaSetDevice(ctx->device));
+  return run_general(ctx, in, Li, n, C, w, h, prm, out, Lo, kin, kout);
 }
 
 // Row bands (sec. 8(e) of SURVEY.md / DESIGN.md sec. 9).
@@ -578,7 +722,8 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
     if (e != cudaSuccess) break;
     // load every kernel now (lazy module loading can deadlock spinning kernels, kernels.h)
     if ((e = sharp::preload_step()) != cudaSuccess || (e = sharp::preload_two_pass()) != cudaSuccess ||
-        (e = sharp::preload_staged()) != cudaSuccess || (e = sharp::preload_p2p()) != cudaSuccess)
+        (e = sharp::preload_staged()) != cudaSuccess || (e = sharp::preload_p2p()) != cudaSuccess ||
+        (e = sharp::preload_layout()) != cudaSuccess)
       break;
     if (c.max_frames > 0 && (rc = ensure_frames(ctx, (size_t)c.max_frames))) break;
     if (c.max_width > 0 && c.max_height > 0) {
@@ -613,6 +758,10 @@ void sharp_destroy(sharp_ctx *ctx) {
   cudaFree(ctx->luts);
   cudaFree(ctx->tcounters);
   cudaFree(ctx->staged);
+  cudaFree(ctx->gx_in);
+  cudaFree(ctx->gx_out);
+  cudaFree(ctx->gx_src);
+  cudaFree(ctx->gx_dst);
   for (auto &r : ctx->recs) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -644,6 +793,11 @@ int sharp_run_batch(sharp_ctx *ctx, const uint8_t *imgs, int n, int w, int h, co
 int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int h, const sharp_params *params,
                         uint8_t *d_outs) {
   return run_impl(ctx, d_imgs, n, w, h, params, d_outs, true);
+}
+
+int sharp_run_ex(sharp_ctx *ctx, const uint8_t *imgs, const sharp_layout *in_layout, int n, int channels, int w,
+                 int h, const sharp_params *params, int flags, uint8_t *outs, const sharp_layout *out_layout) {
+  return run_ex_impl(ctx, imgs, in_layout, n, channels, w, h, params, flags, outs, out_layout);
 }
 
 int sharp_get_stats(const sharp_ctx *ctx, sharp_stats *s) {
