@@ -22,6 +22,11 @@
 namespace {
 
 constexpr size_t kL2ChunkBudget = 24u << 20;  // input bytes per chunk kept L2-resident between passes
+// Host pipeline on the step kernel (no L2 residency needed between launches):
+// bigger chunks amortise the per-chunk copy / launch overheads (measured on
+// 1024 x 1080p pinned: 24 MB chunks 47.4 ms, 48-64 MB 45.3-46.3 ms, PCIe
+// ceiling with both directions busy 43.3 ms; tools/e2e_sweep.py).
+constexpr size_t kHostStepChunkBudget = 48u << 20;
 constexpr int kMaxSlots = 8;
 
 struct Slot {
@@ -207,8 +212,8 @@ int ensure_slots(sharp_ctx *ctx, size_t chunk, size_t frame_bytes, bool staging)
   return SHARP_OK;
 }
 
-size_t chunk_frames(const sharp_ctx *ctx, size_t frame_bytes, int n) {
-  size_t c = ctx->chunk_cfg > 0 ? (size_t)ctx->chunk_cfg : std::max<size_t>(1, kL2ChunkBudget / frame_bytes);
+size_t chunk_frames(const sharp_ctx *ctx, size_t frame_bytes, int n, size_t budget = kL2ChunkBudget) {
+  size_t c = ctx->chunk_cfg > 0 ? (size_t)ctx->chunk_cfg : std::max<size_t>(1, budget / frame_bytes);
   c = std::min<size_t>(c, 65535);
   return std::min<size_t>(c, (size_t)n);
 }
@@ -367,8 +372,13 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   CK(cudaSetDevice(ctx->device));
   const auto t0 = std::chrono::steady_clock::now();
   const size_t fb = (size_t)w * h;
-  const size_t chunk = chunk_frames(ctx, fb, n);
   const bool staged = !(kin == kDevice && kout == kDevice);
+  // host pipeline whose chunks run on the step kernel (staging buffers are
+  // cudaMalloc'd, so only the geometry, the path and the switches decide)
+  const bool step_chunks = staged && (w % 16) == 0 && (size_t)w * h <= (1u << 29) &&
+                           (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+                           !(prm.flags & sharp::kReadPerPixel);
+  const size_t chunk = chunk_frames(ctx, fb, n, step_chunks ? kHostStepChunkBudget : kL2ChunkBudget);
   if ((rc = ensure_frames(ctx, (size_t)n))) return rc;
   if ((rc = ensure_slots(ctx, chunk, fb, staged))) return rc;
   int launches = 0;
