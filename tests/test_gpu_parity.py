@@ -246,3 +246,48 @@ def test_step_path_rejects_unsupported_geometry():
         with pytest.raises(SharpError) as e:
             s.run(d, DEFAULT, o)
         assert e.value.code == SHARP_EUNSUPPORTED
+
+
+
+def oracle_rows(img, mean, r0, r1, prm=DEFAULT):
+    """Oracle output rows [r0, r1) of a big image from its stages on the row
+    window [max(r0 - 8, 0), min(r1 + 8, H)) (4-aligned r0, r1) with the WHOLE
+    image's mean: an output row reads D, U (body formula, L146), pEdge and the
+    3x3 window only within 5 rows, so rows more than 5 away
+    from a window edge that is not an image edge equal the whole-image stages."""
+    A, g, G, K = prm
+    lo, hi = max(r0 - 8, 0), min(r1 + 8, img.shape[0])
+    sub = np.ascontiguousarray(img[lo:hi])
+    Hs, Ws = sub.shape
+    U = oracle.upscale(oracle.downscale(sub), Ws, Hs)
+    pE = oracle.sobel(sub)
+    adj = oracle.strength(pE, mean, A, g)
+    P = oracle.preliminary(adj, oracle.perror(sub, U), U)
+    return oracle.output(oracle.overshoot(sub, P, pE, mean, G, K))[r0 - lo:r1 - lo]
+
+
+def test_oracle_rows_helper_matches_whole_image():
+    img = synth.image(512, 256, "natural", seed=5)
+    ref, S, mean = oracle.sharpen(img)
+    for r0 in (0, 8, 100, 192):
+        np.testing.assert_array_equal(oracle_rows(img, mean, r0, r0 + 64), ref[r0:r0 + 64])
+
+
+def test_full_size_16384_sampled_rows():
+    """BASELINE configs[3] C4b (16384^2, 268 Mpx) on one GPU: S exact against
+    the oracle's full-image Sobel + reduction, and 64-row bands at the top
+    (ring rows), middle and bottom (ring rows) bit-exact."""
+    W = H = 16384
+    img = synth.image(W, H, "natural", seed=synth.BASE_SEED + 4)
+    s = Sharpener()
+    d = torch.from_numpy(img).cuda()
+    o = torch.empty_like(d)
+    s.run(d, DEFAULT, o)
+    torch.cuda.synchronize()
+    st = s.stats()
+    S_ref, mean_ref = oracle.reduce(oracle.sobel(img))
+    assert st.edge_sum == S_ref and st.edge_mean == mean_ref
+    out = o.cpu().numpy()
+    for r0 in (0, 8192 - 32, H - 64):
+        np.testing.assert_array_equal(out[r0:r0 + 64], oracle_rows(img, mean_ref, r0, r0 + 64))
+    s.close()
