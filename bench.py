@@ -1,11 +1,15 @@
 #!/usr/bin/env python
 """Benchmark of the B200 sharpness pipeline (one JSON line on rank 0).
 
-Workload (BASELINE.json configs[4], frame = configs[1]): a batch of 1024
-synthetic 1920x1080 8-bit frames split across the N GPUs (one process per
-GPU).  A step = the whole hot path (pass 1: Sobel + reduction + LUTs; pass 2:
-fused downscale/upscale/pError/Sobel/min-max/strength/preliminary/overshoot)
-over the whole batch.
+Workload (BASELINE.json configs[4], frame = configs[1]): batches of 1024
+synthetic 1920x1080 8-bit frames, one process per GPU.  The frames are
+independent units (each has its own pEdge mean), so the path partitions with
+no collective on the data path: by default every rank sharpens its own 1024
+frames ("scaling": "weak", the partitioned-path rule); --scaling strong
+splits one 1024-frame batch over the ranks instead.  A step = the whole hot
+path (pass 1: Sobel + reduction + LUTs; pass 2: fused downscale/upscale/
+pError/Sobel/min-max/strength/preliminary/overshoot) over the batch; value =
+all ranks' pixels / the slowest rank's step time.
 
   value  : Mpix/s, device-resident (inputs already in HBM), CUDA events on the
            launch stream, max over ranks.  The 2.1 GB batch is larger than the
@@ -177,7 +181,7 @@ def run_reference(args, world, rank):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(np.median(times) * 1e3),
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
         "data": "synthetic", "config": workload_config(args, world),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": f"{len(idx)} of {args.frames} frames per step (every "
@@ -188,11 +192,19 @@ def run_reference(args, world, rank):
 
 
 def workload_config(args, world):
-    return {"workload": f"{args.frames} x {args.width}x{args.height} u8 frames (BASELINE configs[4]; "
-                        f"frame = configs[1])",
-            "frames": args.frames, "width": args.width, "height": args.height,
+    weak = getattr(args, "scaling", "weak") == "weak"
+    if weak:
+        wl = (f"{args.frames} x {args.width}x{args.height} u8 frames per GPU (BASELINE configs[4]'s batch on each "
+              f"of {world} GPU(s); frame = configs[1])")
+        par = f"independent frames, {args.frames} per GPU on {world} GPU(s), no collective on the data path"
+    else:
+        wl = f"{args.frames} x {args.width}x{args.height} u8 frames (BASELINE configs[4]; frame = configs[1])"
+        par = f"frames split over {world} GPU(s), no collective on the data path"
+    return {"workload": wl,
+            "frames": args.frames * (world if weak else 1), "frames_per_gpu": args.frames if weak else None,
+            "width": args.width, "height": args.height,
             "params": dict(zip(["amount", "gamma", "osc_gain", "osc_scale"], PARAMS)),
-            "parallelism": f"frames split over {world} GPU(s), no collective on the data path",
+            "parallelism": par,
             "l2": "batch (2.1 GB in + out) > 126 MB L2: no flush needed between steps"}
 
 
@@ -410,7 +422,11 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--frames", type=int, default=1024)
+    ap.add_argument("--frames", type=int, default=1024,
+                    help="batch size: per GPU with --scaling weak, in total with --scaling strong")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak (default): every rank sharpens its own --frames frames (independent units, the "
+                         "partitioned-path rule); strong: --frames split over the ranks")
     ap.add_argument("--width", type=int, default=1920)
     ap.add_argument("--height", type=int, default=1080)
     ap.add_argument("--e2e-steps", type=int, default=5)
@@ -449,7 +465,10 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     W, H = args.width, args.height
-    start, n = shard.frame_range(args.frames, world, rank)
+    if args.scaling == "weak":
+        start, n = rank * args.frames, args.frames
+    else:
+        start, n = shard.frame_range(args.frames, world, rank)
     fb = W * H
     # Inputs: pinned host (for e2e) and a device copy (device-resident value).
     h_in = torch.empty((n, H, W), dtype=torch.uint8).pin_memory()
@@ -488,7 +507,7 @@ def main():
     ms_step = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
     kt = sh.kernel_times()
     sh.set_profiling(False)
-    total_px = args.frames * fb
+    total_px = args.frames * fb * (world if args.scaling == "weak" else 1)  # all ranks' frames
     value = total_px / (ms_step * 1e-3) / 1e6
 
     # dominant kernel: the step kernel (TMA path: pass 1 of chunk c+1 fused
@@ -555,7 +574,7 @@ def main():
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": workload_config(args, world),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic_per_launch(px_per_launch),
