@@ -53,6 +53,8 @@ struct sharp_ctx {
   cudaEvent_t stage_open[sharp::kNumStages] = {};
   Slot slots[kMaxSlots];
   size_t slot_chunk_frames = 0, slot_stage_bytes = 0;  // capacity of the slot buffers
+  void *zero_block = nullptr;  // acc | sums | lut_done | tcounters (one memset per call)
+  size_t zero_bytes = 0;
   unsigned long long *sums = nullptr;
   double *means = nullptr;
   size_t frames_cap = 0;
@@ -135,41 +137,40 @@ int classify(sharp_ctx *ctx, const void *p, Kind *k) {
   return SHARP_OK;
 }
 
-int ensure_frames(sharp_ctx *ctx, size_t n) {
-  if (n <= ctx->frames_cap) return SHARP_OK;
+// Per-frame scratch.  acc, sums, lut_done and the task counters live in ONE
+// allocation ("zero block") so a call zeroes them with a single memset (for a
+// single image the memsets are a visible share of the latency).
+int ensure_frames(sharp_ctx *ctx, size_t n, size_t n_tc = 0) {
+  const size_t need_tc = std::max(n_tc, 2 * n + 2);
+  if (n <= ctx->frames_cap && need_tc <= ctx->tcounters_cap) return SHARP_OK;
   CK(cudaStreamSynchronize(ctx->stream));
   for (int i = 0; i < ctx->nslots; ++i) CK(cudaStreamSynchronize(ctx->slots[i].stream));
-  cudaFree(ctx->sums);
+  cudaFree(ctx->zero_block);
   cudaFree(ctx->means);
-  cudaFree(ctx->lut_done);
-  cudaFree(ctx->acc);
   cudaFree(ctx->luts);
-  ctx->sums = nullptr;
+  ctx->zero_block = nullptr;
+  ctx->sums = ctx->acc = nullptr;
+  ctx->lut_done = ctx->tcounters = nullptr;
   ctx->means = nullptr;
-  ctx->lut_done = nullptr;
-  ctx->acc = nullptr;
   ctx->luts = nullptr;
-  ctx->frames_cap = 0;
-  CK(cudaMalloc(&ctx->sums, n * sizeof(unsigned long long)));
-  CK(cudaMalloc(&ctx->means, n * sizeof(double)));
-  CK(cudaMalloc(&ctx->lut_done, n * sizeof(unsigned int)));
-  CK(cudaMalloc(&ctx->acc, n * sizeof(unsigned long long)));
-  CK(cudaMalloc(&ctx->luts, n * sharp::kLutSize * sizeof(float2)));
-  ctx->frames_cap = n;
+  ctx->frames_cap = ctx->tcounters_cap = ctx->zero_bytes = 0;
+  const size_t cap = std::max(n, ctx->frames_cap), tcap = std::max(need_tc, 2 * cap + 2);
+  const size_t b_acc = cap * 8, b_sums = cap * 8, b_done = (cap * 4 + 7) & ~(size_t)7, b_tc = tcap * 4;
+  CK(cudaMalloc(&ctx->zero_block, b_acc + b_sums + b_done + b_tc));
+  uint8_t *z = static_cast<uint8_t *>(ctx->zero_block);
+  ctx->acc = reinterpret_cast<unsigned long long *>(z);
+  ctx->sums = reinterpret_cast<unsigned long long *>(z + b_acc);
+  ctx->lut_done = reinterpret_cast<unsigned int *>(z + b_acc + b_sums);
+  ctx->tcounters = reinterpret_cast<unsigned int *>(z + b_acc + b_sums + b_done);
+  ctx->zero_bytes = b_acc + b_sums + b_done + b_tc;
+  CK(cudaMalloc(&ctx->means, cap * sizeof(double)));
+  CK(cudaMalloc(&ctx->luts, cap * sharp::kLutSize * sizeof(float2)));
+  ctx->frames_cap = cap;
+  ctx->tcounters_cap = tcap;
   return SHARP_OK;
 }
 
-int ensure_task_counters(sharp_ctx *ctx, size_t n) {
-  if (n <= ctx->tcounters_cap) return SHARP_OK;
-  CK(cudaStreamSynchronize(ctx->stream));
-  for (int i = 0; i < ctx->nslots; ++i) CK(cudaStreamSynchronize(ctx->slots[i].stream));
-  cudaFree(ctx->tcounters);
-  ctx->tcounters = nullptr;
-  ctx->tcounters_cap = 0;
-  CK(cudaMalloc(&ctx->tcounters, n * sizeof(unsigned int)));
-  ctx->tcounters_cap = n;
-  return SHARP_OK;
-}
+int ensure_task_counters(sharp_ctx *ctx, size_t n) { return ensure_frames(ctx, ctx->frames_cap, n); }
 
 void free_slot(Slot &s) {
   cudaFree(s.d_in);
@@ -384,10 +385,7 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   int launches = 0;
   const size_t nchunks_all = ((size_t)n + chunk - 1) / chunk;
   if ((rc = ensure_task_counters(ctx, 2 * nchunks_all + 2))) return rc;
-  CK(cudaMemsetAsync(ctx->sums, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
-  CK(cudaMemsetAsync(ctx->lut_done, 0, (size_t)n * sizeof(unsigned int), ctx->stream));
-  CK(cudaMemsetAsync(ctx->acc, 0, (size_t)n * sizeof(unsigned long long), ctx->stream));
-  CK(cudaMemsetAsync(ctx->tcounters, 0, (2 * nchunks_all + 2) * sizeof(unsigned int), ctx->stream));
+  CK(cudaMemsetAsync(ctx->zero_block, 0, ctx->zero_bytes, ctx->stream));  // acc, sums, lut_done, counters
   CK(cudaEventRecord(ctx->ev_start, ctx->stream));
   if (!staged) {
     if ((rc = enqueue_device(ctx, in, n, w, h, prm, out, ctx->stream, ctx->slots[0], chunk, 0, &launches,
@@ -761,12 +759,9 @@ void sharp_destroy(sharp_ctx *ctx) {
     if (s.done) cudaEventDestroy(s.done);
     if (s.stream) cudaStreamDestroy(s.stream);
   }
-  cudaFree(ctx->sums);
+  cudaFree(ctx->zero_block);
   cudaFree(ctx->means);
-  cudaFree(ctx->lut_done);
-  cudaFree(ctx->acc);
   cudaFree(ctx->luts);
-  cudaFree(ctx->tcounters);
   cudaFree(ctx->staged);
   cudaFree(ctx->gx_in);
   cudaFree(ctx->gx_out);
