@@ -491,7 +491,9 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
                 const sharp::Params &prm, uint8_t *out, const Layout &Lo, Kind kin, Kind kout) {
   const int W4 = (w + 3) & ~3, H4 = (h + 3) & ~3;
   const size_t ub = (size_t)W4 * H4;
-  const int fpc = (int)std::max<size_t>(1, std::min<size_t>((size_t)n, kGeneralChunkBytes / (ub * C)));
+  // frames per chunk: sharp_config.chunk_frames if set, else ~kGeneralChunkBytes of padded units
+  const int fpc = ctx->chunk_cfg > 0 ? std::min(ctx->chunk_cfg, n)
+                                     : (int)std::max<size_t>(1, std::min<size_t>((size_t)n, kGeneralChunkBytes / (ub * C)));
   const size_t units_all = (size_t)n * C;
   int rc;
   if ((rc = ensure_frames(ctx, units_all))) return rc;

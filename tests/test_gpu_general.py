@@ -215,3 +215,39 @@ def test_run_ex_errors():
         sharp_run_ex(s.ctx, d, (8, 0, 1), 1, 1, 16, 16, None, 0, o, None)
     assert e.value.code == SHARP_EINVAL
     s.close()
+
+
+@pytest.mark.parametrize("where", ["device", "host"])
+def test_general_path_in_chunks(where):
+    """chunk_frames = 1: the gather / run / scatter loop runs once per frame
+    (sums of every chunk kept), also in place."""
+    s = Sharpener(chunk_frames=1)
+    W, H, n = 45, 27, 4
+    imgs = synth.frames(n, 48, 32, "natural", seed=synth.BASE_SEED + 21)[:, :H, :W].copy()
+    refs, sums = ref_units(list(imgs), STRONG, 0)
+    t = torch.from_numpy(imgs.copy())
+    if where == "device":
+        t = t.cuda()
+    out = s.run_ex(t, STRONG)
+    torch.cuda.synchronize()
+    for f in range(n):
+        check(out[f].cpu().numpy(), refs[f], f"frame {f}")
+    assert s.batch_sums(n) == sums
+    s.run_ex(t, STRONG, out=t)  # in place, chunk by chunk
+    torch.cuda.synchronize()
+    for f in range(n):
+        check(t[f].cpu().numpy(), refs[f], f"in-place frame {f}")
+    s.close()
+
+
+@pytest.mark.parametrize("flags", [oracle.READ_TRUNCATE | oracle.READ_INTERIOR_MEAN, oracle.READ_STRENGTH_EXP])
+def test_reading_switches_host_pipeline(flags):
+    """Dense host buffers with switches: the pinned-staging pipeline path."""
+    s = Sharpener(chunk_frames=2)
+    imgs = synth.frames(5, 1920, 40, "natural", seed=synth.BASE_SEED + 2 * flags)
+    out = s.run_ex(torch.from_numpy(imgs), DEFAULT, flags=flags)
+    refs, sums = ref_units(list(imgs), DEFAULT, flags)
+    for f in range(5):
+        check(out[f].numpy(), refs[f], f"frame {f}")
+    assert s.batch_sums(5) == sums
+    s.close()
