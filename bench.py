@@ -102,11 +102,28 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+# Test hook: SHARP_BENCH_SHARE_GPU=1 maps every rank onto the visible GPUs
+# round-robin and uses gloo for the plumbing (NCCL refuses two ranks on one
+# GPU), so the multi-rank code path can be exercised on a one-GPU box.  Never
+# set for a measurement.
+SHARE_GPU = os.environ.get("SHARP_BENCH_SHARE_GPU") == "1"
+
+
 def dist_setup():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if SHARE_GPU:
+        import torch
+        local %= max(1, torch.cuda.device_count())
     return world, rank, local
+
+
+def init_group(torch, dist, local):
+    if SHARE_GPU:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
 
 def traffic_per_launch(px_per_launch):
@@ -219,7 +236,7 @@ def run_bands_workload(args, world, rank, local):
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        init_group(torch, dist, local)
     W, H = args.width, args.height
     r0, r1 = band_rows(H, world, rank)
     img = synth.image(W, H, "natural", seed=synth.BASE_SEED + 3)  # every rank generates, keeps its rows
@@ -463,7 +480,7 @@ def main():
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        init_group(torch, dist, local)
     W, H = args.width, args.height
     if args.scaling == "weak":
         start, n = rank * args.frames, args.frames
