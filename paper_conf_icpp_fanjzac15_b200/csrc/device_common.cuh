@@ -207,16 +207,20 @@ __device__ __forceinline__ double frame_mean(unsigned long long S, int W, int H,
 //   adj = A (p / m)^gamma        (R9)   or A (1 - exp(-p / (K m)))   (R9 alternative)
 //   osc = clamp(G exp(-p / (K m)), 0, 1)   (R11)   or G               (R11 alternative)
 // with m = max(mean, 1).
-__device__ __forceinline__ float2 lut_entry(int p, double mean, const Params &prm) {
+__device__ __forceinline__ float lut_adj(int p, double mean, const Params &prm) {
   const double m = mean > 1.0 ? mean : 1.0;
-  const float adj = (prm.flags & kReadStrengthExp)
-                        ? (float)((double)prm.amount * (1.0 - exp(-(double)p / ((double)prm.osc_scale * m))))
-                        : (float)((double)prm.amount * pow((double)p / m, (double)prm.gamma));
-  const float osc = (prm.flags & kReadOscConst)
-                        ? prm.osc_gain
-                        : (float)fmin(fmax((double)prm.osc_gain * exp(-(double)p / ((double)prm.osc_scale * m)), 0.0),
-                                      1.0);
-  return make_float2(adj, osc);
+  return (prm.flags & kReadStrengthExp)
+             ? (float)((double)prm.amount * (1.0 - exp(-(double)p / ((double)prm.osc_scale * m))))
+             : (float)((double)prm.amount * pow((double)p / m, (double)prm.gamma));
+}
+__device__ __forceinline__ float lut_osc(int p, double mean, const Params &prm) {
+  const double m = mean > 1.0 ? mean : 1.0;
+  return (prm.flags & kReadOscConst)
+             ? prm.osc_gain
+             : (float)fmin(fmax((double)prm.osc_gain * exp(-(double)p / ((double)prm.osc_scale * m)), 0.0), 1.0);
+}
+__device__ __forceinline__ float2 lut_entry(int p, double mean, const Params &prm) {
+  return make_float2(lut_adj(p, mean, prm), lut_osc(p, mean, prm));
 }
 
 // Packs 8 bytes (low byte of each word) into two words.

@@ -53,12 +53,13 @@ constexpr int kCtasPerSm = 3;  // smem ~67 KB per CTA
 constexpr int kWarpsT = 4;   // compute warps = warp tiles per CTA tile
 constexpr int kCtaCols = kTW * kWarpsT;
 constexpr int kThreadsT = 32 * (kWarpsT + 1);  // + producer warp
-constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task
+constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task (one per thread)
 // pEdge = |Gx| + |Gy| is always even (Gx and Gy both have the parity of the
 // sum of the four window corners), so the step kernel's tables hold the even
 // entries only: entry k = pEdge / 2, k < kLut2 (766 used).
 constexpr int kLut2 = 768;
 constexpr int kLutTasks = kLut2 / kLutPerTask;
+constexpr unsigned kPollNs = 100;  // dependency polling interval of the producer
 // A warp tile needs columns C0w-8 .. C0w+247.  TMA box starts must be
 // 16-byte aligned in the innermost dimension and a box dimension is at most
 // 256, so a warp tile is fetched as one 256-column box of the [n][H][W]
@@ -635,6 +636,19 @@ __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rm
   return sum;
 }
 
+#ifdef SHARP_EXP_TIMELINE  // timing experiment: globaltimer of the launch's phases (min / max over CTAs)
+__device__ unsigned long long g_tl[8];
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define TL_MIN(i) atomicMin(&g_tl[i], gtimer())
+#define TL_MAX(i) atomicMax(&g_tl[i], gtimer())
+#else
+#define TL_MIN(i)
+#define TL_MAX(i)
+#endif
 #ifdef SHARP_EXP_WAITSTAT  // timing experiment: consumer full-barrier wait cycles by (previous, awaited) task type
 __device__ unsigned long long g_waitstat[40][2];
 __shared__ long long stage_t[2];  // producer: clock64 at issue
@@ -653,6 +667,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
   const uint32_t lutbase = sbase + kLutOff;
   const Geo &g = sp.g;
 
+  if (threadIdx.x == 0) TL_MIN(0);
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       mbar_init(ring.full0 + 8 * i, 1);
@@ -678,13 +693,10 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       if (d.x == kLut) {
         // every pass-1 warp of the frame has added its partial (the global
         // barrier of L174's reduction)
-        while (((S = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(500);
-      } else if (d.x == kP2) {
-        // the frame's LUT tasks (grabbed earlier) have finished
-        while (ld_relaxed_u32(&sp.lut_done[d.y]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(500);
-        fence_acquire();
-        fence_proxy_async_global();
+        while (((S = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(kPollNs);
       }
+      // (A pass-2 task's dependency -- its frame's LUT -- is resolved after
+      // its first stage's tile loads are issued: the loads do not need it.)
       int C0 = 0, R0 = 0, nsub = 1, nw = 0;
       if (d.x == kP1 || d.x == kP2) {
         tile_xy(g, d.z, d.x == kP1 ? g.th1 : kTH * g.sub, C0, R0);
@@ -718,6 +730,12 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           if (k == 0 && tl > s - kStages) mbar_wait(ring.empty0 + 8u * Ring::buf(tl), Ring::phase(tl));
           mbar_expect_tx(full, tile_bytes(nw, kRows2) + lut_bytes);
           tma_tiles(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
+          if (lut_bytes) {
+            // the frame's LUT tasks (grabbed earlier) have finished
+            while (ld_relaxed_u32(&sp.lut_done[d.y]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(kPollNs);
+            fence_acquire();
+            fence_proxy_async_global();
+          }
           if (lut_bytes)
             bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
         } else {
@@ -758,10 +776,14 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       if (d.x == kEnd) atomicAdd(&g_waitstat[25][0], (unsigned long long)(clock64() - t_begin));
     }
 #endif
-    if (d.x == kEnd) break;
+    if (d.x == kEnd) {
+      if (lane == 0) TL_MAX(7);
+      break;
+    }
     if (d.x == kP2) {
       const int2 aux = stage_aux[b];
       const int C0 = d.z, R0 = d.w, C0w = C0 + warp * kTW;
+      if (lane == 0) TL_MIN(5);
       if (C0w < g.W) {
         p2_warp(ring, s, aux.x, lutbase, aux.y, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H,
                 g.row_lo, g.row_hi, C0w, R0, warp, lane);
@@ -771,12 +793,16 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           ring.release(s + k, lane);
         }
       }
+      if (lane == 0) TL_MAX(6);
       s += aux.x;
       continue;
     }
+    if (d.x == kLut && lane == 0) TL_MIN(3);
+    if (d.x == kP1 && lane == 0) TL_MIN(1);
     if (d.x == kLut) {
       // LUT task: entries k = q*128 .. q*128+127 (pEdge p = 2k) of frame f
-      // (R9, R11; f64, one rounding)
+      // (R9, R11; f64, one rounding).  (Measured: splitting adj / osc over two
+      // threads per entry does not shorten the build and costs 0.9% of the batch.)
       const int f = d.y, k = d.z * kLutPerTask + threadIdx.x, p = 2 * k;
       // L174: mean of pEdge (R8), from the exact sum.
       const unsigned long long S = stage_sum[b];
@@ -789,6 +815,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       __threadfence();
       __syncwarp();
       if (lane == 0) atomicAdd(&sp.lut_done[f], 1u);
+      if (lane == 0) TL_MAX(4);
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
@@ -799,6 +826,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       // without any fence.
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
       if (lane == 0) atomicAdd(&sp.acc[d.y], (1ull << kAccShift) + (unsigned long long)ws);
+      if (lane == 0) TL_MAX(2);
     }
     ring.release(s, lane);  // stage s may be refilled
     ++s;
@@ -843,6 +871,18 @@ int num_sms() {
 
 }  // namespace
 
+#ifdef SHARP_EXP_TIMELINE
+extern "C" int sharp_debug_timeline(unsigned long long *out, int reset) {
+  cudaDeviceSynchronize();
+  cudaMemcpyFromSymbol(out, g_tl, sizeof(g_tl));
+  if (reset) {
+    unsigned long long z[8];
+    for (int i = 0; i < 8; ++i) z[i] = (i == 0 || i == 1 || i == 3 || i == 5) ? ~0ull : 0ull;
+    cudaMemcpyToSymbol(g_tl, z, sizeof(z));
+  }
+  return 0;
+}
+#endif
 #ifdef SHARP_EXP_WAITSTAT
 extern "C" int sharp_debug_waitstat(unsigned long long *out, int reset) {
   cudaDeviceSynchronize();
