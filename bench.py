@@ -477,6 +477,7 @@ def main():
     import synth
     from paper_conf_icpp_fanjzac15_b200 import Sharpener
     from paper_conf_icpp_fanjzac15_b200 import shard
+    from paper_conf_icpp_fanjzac15_b200.binding import _params as sharp_params_of
 
     torch.cuda.set_device(local)
     if world > 1:
@@ -506,22 +507,33 @@ def main():
         return shard.max_over_ranks(x, device=f"cuda:{local}")
 
     # ---- device-resident timed region
+    prm = sharp_params_of(PARAMS)  # marshalled once: the loop times the library, not ctypes
     for _ in range(args.warmup):
-        sh.enqueue_batch(d_in, d_out, PARAMS)
+        sh.enqueue_batch(d_in, d_out, prm)
     torch.cuda.synchronize()
     launches_per_step = sh.stats().kernels
-    sh.set_profiling(True)
+    # Per-launch kernel events ride inside the timed region for batches; for a
+    # latency-sized step (a few frames, ~20 us) two extra event records per
+    # launch would be a visible part of the step, so there the kernel times
+    # come from a second, profiled pass over the same steps.
+    latency_regime = n <= 8
+    sh.set_profiling(not latency_regime)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
         ev0.record(stream)
         for _ in range(args.steps):
-            sh.enqueue_batch(d_in, d_out, PARAMS)
+            sh.enqueue_batch(d_in, d_out, prm)
         ev1.record(stream)
         torch.cuda.synchronize()
     barrier()
     ms_step = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
+    if latency_regime:
+        sh.set_profiling(True)
+        for _ in range(args.steps):
+            sh.enqueue_batch(d_in, d_out, prm)
+        torch.cuda.synchronize()
     kt = sh.kernel_times()
     sh.set_profiling(False)
     total_px = args.frames * fb * (world if args.scaling == "weak" else 1)  # all ranks' frames
@@ -598,7 +610,9 @@ def main():
                          "kernel": kname, "peak_source": pk_src,
                          "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px_per_launch,
                          "kernel_avg_ms": k_avg_ms, "kernel_launches": k_launches,
-                         "kernel_share_of_step": k_share, "step_frac": step_achieved / peak},
+                         "kernel_share_of_step": k_share, "step_frac": step_achieved / peak,
+                         "kernel_events": ("a second, profiled pass over the same steps (latency regime)"
+                                           if latency_regime else "per launch, inside the timed region")},
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": total_px,
                     "d2h_bytes_per_step": total_px, "ms_per_step": e2e_ms,
                     "api": "sharp_run_batch(pinned host in, pinned host out)"},

@@ -45,6 +45,7 @@ struct sharp_ctx {
   cudaStream_t own_stream = nullptr;
   cudaStream_t stream = nullptr;  // launch stream (own or caller's)
   cudaEvent_t ev_start = nullptr, ev_stop = nullptr;
+  struct HostStats { unsigned long long sum; double mean; } *h_stats = nullptr;  // pinned
   int nslots = 3;
   int chunk_cfg = 0;
   int path = SHARP_PATH_AUTO;  // SHARP_FORCE_GENERIC=1 at sharp_create selects SHARP_PATH_TWO_PASS
@@ -440,15 +441,15 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   ctx->stats.kernels = launches;
   if (async) return SHARP_OK;
   CK(cudaEventRecord(ctx->ev_stop, ctx->stream));
-  CK(cudaEventSynchronize(ctx->ev_stop));
+  // frame 0's S and mean ride on the stream into pinned host memory: one
+  // synchronisation per call instead of two more blocking copies
+  CK(cudaMemcpyAsync(&ctx->h_stats->sum, ctx->sums, sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaMemcpyAsync(&ctx->h_stats->mean, ctx->means, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
   float ms = 0.0f;
   CK(cudaEventElapsedTime(&ms, ctx->ev_start, ctx->ev_stop));
-  unsigned long long s0 = 0;
-  double m0 = 0.0;
-  CK(cudaMemcpy(&s0, ctx->sums, sizeof(s0), cudaMemcpyDeviceToHost));
-  CK(cudaMemcpy(&m0, ctx->means, sizeof(m0), cudaMemcpyDeviceToHost));
-  ctx->stats.edge_sum = s0;
-  ctx->stats.edge_mean = m0;
+  ctx->stats.edge_sum = ctx->h_stats->sum;
+  ctx->stats.edge_mean = ctx->h_stats->mean;
   ctx->stats.device_ms = ms;
   ctx->stats.total_ms =
       std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
@@ -725,6 +726,7 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
     ctx->stream = ctx->own_stream;
     if ((e = cudaEventCreate(&ctx->ev_start)) != cudaSuccess) break;
     if ((e = cudaEventCreate(&ctx->ev_stop)) != cudaSuccess) break;
+    if ((e = cudaHostAlloc(&ctx->h_stats, sizeof(*ctx->h_stats), cudaHostAllocDefault)) != cudaSuccess) break;
     for (int i = 0; i < ctx->nslots && e == cudaSuccess; ++i) {
       e = cudaStreamCreateWithFlags(&ctx->slots[i].stream, cudaStreamNonBlocking);
       if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->slots[i].done, cudaEventDisableTiming);
@@ -776,6 +778,7 @@ void sharp_destroy(sharp_ctx *ctx) {
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
   if (ctx->ev_stop) cudaEventDestroy(ctx->ev_stop);
+  if (ctx->h_stats) cudaFreeHost(ctx->h_stats);
   if (ctx->own_stream) cudaStreamDestroy(ctx->own_stream);
   cudaGetLastError();
   delete ctx;
