@@ -119,6 +119,29 @@ def dist_setup():
     return world, rank, local
 
 
+def bind_to_gpu_numa_node(torch, local):
+    """Pin this rank's threads to the CPUs of its GPU's NUMA node (before the
+    pinned host buffers are first touched), so the e2e leg's H2D / D2H read
+    and write NUMA-local memory.  Best effort: returns the node or None."""
+    try:
+        pr = torch.cuda.get_device_properties(local)
+        bus = f"{pr.pci_domain_id:04x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+        node = int(open(f"/sys/bus/pci/devices/{bus}/numa_node").read())
+        if node < 0:
+            return None
+        cpus = set()
+        for part in open(f"/sys/devices/system/node/node{node}/cpulist").read().strip().split(","):
+            a, _, b = part.partition("-")
+            cpus.update(range(int(a), int(b or a) + 1))
+        cpus &= os.sched_getaffinity(0)
+        if cpus:
+            os.sched_setaffinity(0, cpus)
+            return node
+    except (OSError, ValueError, AttributeError):
+        pass
+    return None
+
+
 def init_group(torch, dist, local):
     if SHARE_GPU:
         dist.init_process_group("gloo")
@@ -483,6 +506,7 @@ def main():
     if world > 1:
         init_group(torch, dist, local)
     W, H = args.width, args.height
+    numa = bind_to_gpu_numa_node(torch, local) if world > 1 else None
     if args.scaling == "weak":
         start, n = rank * args.frames, args.frames
     else:
@@ -623,6 +647,7 @@ def main():
             "cpu_baseline": cpu,
             "paper_context": paper_context,
             "parity": parity,
+            "host_numa_binding": "ranks pinned to their GPU's NUMA node" if numa is not None else None,
         }
         print(json.dumps(line), flush=True)
     sh.close()
