@@ -22,7 +22,7 @@ NVCC_FLAGS := $(ARCH) -O3 -lineinfo -std=c++17 --fmad=false -Xptxas -v \
 SHARP_SRCS := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 SHARP_HDRS := $(wildcard $(PKG)/csrc/*.cuh) $(wildcard $(PKG)/csrc/*.h) include/sharp.h
 
-all: oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so
+all: oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so tests/c_abi_check
 
 oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
 	$(HOSTCC) $(ORACLE_CFLAGS) -o $@ oracle/oracle.c -lm
@@ -33,9 +33,17 @@ synth/libsynth.so: synth/synth.c
 $(PKG)/libsharp.so: $(SHARP_SRCS) $(SHARP_HDRS)
 	$(NVCC) $(NVCC_FLAGS) -shared -o $@ $(SHARP_SRCS) 2> build/ptxas.log || (cat build/ptxas.log; false)
 
+# The C ABI used from plain C (tests/test_gpu_c_abi.py runs it); links the
+# oracle and the synthetic-input generator as test infrastructure.
+tests/c_abi_check: tests/c_abi_check.c include/sharp.h oracle/oracle.h oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so
+	$(HOSTCC) -std=c11 -O2 -Wall -Wextra -I include -I $(CUDA_HOME)/include -o $@ tests/c_abi_check.c \
+	  -L $(PKG) -lsharp -L oracle -loracle -L synth -lsynth -L $(CUDA_HOME)/lib64 -lcudart \
+	  -Wl,-rpath,'$$ORIGIN/../$(PKG)' -Wl,-rpath,'$$ORIGIN/../oracle' -Wl,-rpath,'$$ORIGIN/../synth' \
+	  -Wl,-rpath,$(CUDA_HOME)/lib64
+
 $(shell mkdir -p build)
 
 clean:
-	rm -f oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so
+	rm -f oracle/liboracle.so synth/libsynth.so $(PKG)/libsharp.so tests/c_abi_check
 
 .PHONY: all clean

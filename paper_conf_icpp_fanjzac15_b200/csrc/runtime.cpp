@@ -989,7 +989,8 @@ const char *sharp_strerror(int code) {
 const char *sharp_last_error(const sharp_ctx *ctx) { return ctx ? ctx->err : "no context"; }
 
 const char *sharp_version(void) {
-  return "libsharp 0.1 (sm_100a; two-pass fused sharpen: edge_sum + sharpen; f16x2 SIMD Sobel)";
+  return "libsharp 0.2 (sm_100a; persistent TMA step kernel, two-pass and staged paths; general layouts; "
+         "reading switches; peer-memory row bands)";
 }
 
 }  // extern "C"

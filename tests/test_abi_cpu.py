@@ -75,3 +75,14 @@ def test_no_cpu_fallback_create_fails_loudly_without_gpu():
     import paper_conf_icpp_fanjzac15_b200 as p
     with pytest.raises(p.SharpError):
         p.sharp_create()
+
+
+def test_c_program_links_against_the_abi():
+    """tests/c_abi_check.c compiles against include/sharp.h and links
+    libsharp.so with plain gcc (no GPU needed to build)."""
+    import subprocess
+    exe = os.path.join(ROOT, "tests", "c_abi_check")
+    subprocess.run(["make", "-C", ROOT, "-s", "tests/c_abi_check"], check=True)
+    assert os.path.exists(exe)
+    out = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
+    assert "libsharp.so" in out and "not found" not in out
