@@ -291,3 +291,28 @@ def test_full_size_16384_sampled_rows():
     for r0 in (0, 8192 - 32, H - 64):
         np.testing.assert_array_equal(out[r0:r0 + 64], oracle_rows(img, mean_ref, r0, r0 + 64))
     s.close()
+
+
+@pytest.mark.parametrize("W,H,path", [(32768, 16384, "step"), (32768, 16392, "two-pass")])
+def test_maximum_sizes_at_the_step_kernel_limit(W, H, path):
+    """Edge of the step kernel's domain (W*H <= 2^29: the packed arrival count
+    + 40-bit sum of `acc`) with worst-case content (uniform
+    noise, large pEdge everywhere), and just past it (the two-pass path takes
+    over).  S exact against the oracle's full-image Sobel + reduction; top,
+    middle and bottom row bands bit-exact."""
+    img = synth.image(W, H, "noise", seed=synth.BASE_SEED + 6)
+    s = Sharpener()
+    d = torch.from_numpy(img).cuda()
+    o = torch.empty_like(d)
+    s.set_profiling(True)
+    s.run(d, DEFAULT, o)
+    torch.cuda.synchronize()
+    kt = s.kernel_times()
+    assert (kt.step_launches > 0) == (path == "step")
+    st = s.stats()
+    S_ref, mean_ref = oracle.reduce(oracle.sobel(img))
+    assert st.edge_sum == S_ref and st.edge_mean == mean_ref
+    out = o.cpu().numpy()
+    for r0 in (0, (H // 2) & ~3, H - 32):
+        np.testing.assert_array_equal(out[r0:r0 + 32], oracle_rows(img, mean_ref, r0, r0 + 32))
+    s.close()
