@@ -32,6 +32,12 @@ __device__ __forceinline__ float add_f32_f16(uint16_t a, float c) {
   asm("add.f32.f16 %0, %1, %2;" : "=f"(d) : "h"(a), "f"(c));
   return d;
 }
+// f16 * f16 + f32 (sm_100 mixed-precision FMA, one FHFMA); exact for the values used.
+__device__ __forceinline__ float fma_f32_f16(uint16_t a, uint16_t b, float c) {
+  float d;
+  asm("fma.rn.f32.f16 %0, %1, %2, %3;" : "=f"(d) : "h"(a), "h"(b), "f"(c));
+  return d;
+}
 __device__ __forceinline__ uint16_t lo16(uint32_t u) { return (uint16_t)(u & 0xffffu); }
 __device__ __forceinline__ uint16_t hi16(uint32_t u) { return (uint16_t)(u >> 16); }
 // Round half to even and saturate to [0, 255] (R14 + the final clamp of Fig. 8).

@@ -621,11 +621,13 @@ __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rm
       const RowD rc = derive_w<false>(row_words(aw, m + a + 2), lane);
       uint32_t pe[4];
       sobel(ra, rb, rc, pe);
-      if ((unsigned)(r - 1) < (unsigned)rmax1) {  // 1 <= r <= rmax1: Sobel frame rows are 0 (L160)
+      // 1 <= r <= rmax1: Sobel frame rows are 0 (L160).  The row weight (1.0 or
+      // 0.0 as f16) goes into a mixed-precision FMA -- no predicated updates
+      // (they cost a move per accumulator and row).
+      const uint16_t on = ((unsigned)(r - 1) < (unsigned)rmax1) ? (uint16_t)0x3C00u : (uint16_t)0u;
 #pragma unroll
-        for (int x = 0; x < 8; ++x)
-          acc[x] = add_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), acc[x]);
-      }
+      for (int x = 0; x < 8; ++x)
+        acc[x] = fma_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), on, acc[x]);
       ra = rb;
       rb = rc;
     }
