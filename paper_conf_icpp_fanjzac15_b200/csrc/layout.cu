@@ -14,54 +14,89 @@
 namespace sharp {
 namespace {
 
-// One thread per 4 dense output bytes (one 32-bit store), grid-stride.
+// A block per (unit, row) pair (grid-stride over rows), threads across the
+// row: no 64-bit index divisions per byte.
+
+// Dense padded row r of unit u <- source row min(r, h-1), columns clamped to
+// w-1 (replicate, R1'); one 32-bit store per 4 bytes.
 __global__ void gather_kernel(const uint8_t *__restrict__ src, size_t fs, size_t pitch, int es, int C, int w, int h,
                               int W4, int H4, int units, uint8_t *__restrict__ dst) {
   const int q4 = W4 >> 2;
-  const size_t total = (size_t)units * H4 * q4;
-  for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < total; t += (size_t)gridDim.x * blockDim.x) {
-    const int q = (int)(t % q4);
-    const size_t ur = t / q4;
-    const int r = (int)(ur % H4), u = (int)(ur / H4);
-    const uint8_t *row = src + (size_t)(u / C) * fs + (size_t)(u % C) + (size_t)min(r, h - 1) * pitch;
-    uint32_t v = 0;
+  for (unsigned ur = blockIdx.x; ur < (unsigned)units * (unsigned)H4; ur += gridDim.x) {
+    const unsigned u = ur / (unsigned)H4, r = ur - u * (unsigned)H4;
+    const uint8_t *row = src + (size_t)(u / C) * fs + (size_t)(u % C) + (size_t)min((int)r, h - 1) * pitch;
+    uint32_t *drow = reinterpret_cast<uint32_t *>(dst + (size_t)ur * W4);
+    for (int q = threadIdx.x; q < q4; q += blockDim.x) {
+      uint32_t v = 0;
+      if (es == 1 && 4 * q + 3 < w) {
+        // 4 contiguous source bytes: the aligned word(s) holding them and a
+        // funnel shift (an aligned word with a valid byte never crosses a page)
+        const uintptr_t a = (uintptr_t)(row + 4 * q);
+        const uint32_t *al = reinterpret_cast<const uint32_t *>(a & ~(uintptr_t)3);
+        const uint32_t sh = (uint32_t)(a & 3) * 8;
+        v = sh ? __funnelshift_r(al[0], al[1], sh) : al[0];
+      } else {
 #pragma unroll
-    for (int k = 0; k < 4; ++k) v |= (uint32_t)row[(size_t)min(4 * q + k, w - 1) * es] << (8 * k);
-    reinterpret_cast<uint32_t *>(dst)[t] = v;
+        for (int k = 0; k < 4; ++k) v |= (uint32_t)row[(size_t)min(4 * q + k, w - 1) * es] << (8 * k);
+      }
+      drow[q] = v;
+    }
   }
 }
 
-// One thread per output byte of the w x h crop, grid-stride.
+// Single-channel rows (elem_stride 1): per destination row, 16-byte stores
+// where the destination is aligned (the row interior), bytes at the ends.
+__global__ void scatter_rows_kernel(const uint8_t *__restrict__ src, int W4, int H4, int units, int w, int h,
+                                    uint8_t *__restrict__ dst, size_t fs, size_t pitch) {
+  for (unsigned ur = blockIdx.x; ur < (unsigned)units * (unsigned)h; ur += gridDim.x) {
+    const unsigned u = ur / (unsigned)h, r = ur - u * (unsigned)h;
+    uint8_t *drow = dst + (size_t)u * fs + (size_t)r * pitch;
+    const uint8_t *srow = src + ((size_t)u * H4 + r) * W4;
+    const int lead = min(w, (int)((16 - ((uintptr_t)drow & 15)) & 15));  // bytes before the first aligned one
+    const int nvec = (w - lead) / 16;
+    for (int c = threadIdx.x; c < lead; c += blockDim.x) drow[c] = srow[c];
+    for (int k = threadIdx.x; k < nvec; k += blockDim.x) {
+      const int c0 = lead + 16 * k;
+      uint4 v;
+      uint8_t *b = reinterpret_cast<uint8_t *>(&v);
+#pragma unroll
+      for (int j = 0; j < 16; ++j) b[j] = srow[c0 + j];
+      *reinterpret_cast<uint4 *>(drow + c0) = v;
+    }
+    for (int c = lead + 16 * nvec + threadIdx.x; c < w; c += blockDim.x) drow[c] = srow[c];
+  }
+}
+
+// Any layout (interleaved channels): a byte per thread.
 __global__ void scatter_kernel(const uint8_t *__restrict__ src, int W4, int H4, int units, int w, int h,
                                uint8_t *__restrict__ dst, size_t fs, size_t pitch, int es, int C) {
-  const size_t total = (size_t)units * h * w;
-  for (size_t t = blockIdx.x * (size_t)blockDim.x + threadIdx.x; t < total; t += (size_t)gridDim.x * blockDim.x) {
-    const int c = (int)(t % w);
-    const size_t ur = t / w;
-    const int r = (int)(ur % h), u = (int)(ur / h);
-    dst[(size_t)(u / C) * fs + (size_t)(u % C) + (size_t)r * pitch + (size_t)c * es] =
-        src[((size_t)u * H4 + r) * W4 + c];
+  for (unsigned ur = blockIdx.x; ur < (unsigned)units * (unsigned)h; ur += gridDim.x) {
+    const unsigned u = ur / (unsigned)h, r = ur - u * (unsigned)h;
+    uint8_t *drow = dst + (size_t)(u / C) * fs + (size_t)(u % C) + (size_t)r * pitch;
+    const uint8_t *srow = src + ((size_t)u * H4 + r) * W4;
+    for (int c = threadIdx.x; c < w; c += blockDim.x) drow[(size_t)c * es] = srow[c];
   }
 }
 
-unsigned grid_for(size_t work) {
-  const size_t b = (work + 255) / 256;
-  return (unsigned)(b < 148 * 32 ? (b ? b : 1) : 148 * 32);
-}
+unsigned rows_grid(size_t rows) { return (unsigned)(rows < 148 * 16 ? (rows ? rows : 1) : 148 * 16); }
 
 }  // namespace
 
 cudaError_t launch_gather(const uint8_t *src, size_t frame_stride, size_t pitch, int elem_stride, int C, int w,
                           int h, int W4, int H4, int units, uint8_t *dst, cudaStream_t st) {
-  gather_kernel<<<grid_for((size_t)units * H4 * (W4 / 4)), 256, 0, st>>>(src, frame_stride, pitch, elem_stride, C, w,
-                                                                         h, W4, H4, units, dst);
+  gather_kernel<<<rows_grid((size_t)units * H4), 128, 0, st>>>(src, frame_stride, pitch, elem_stride, C, w, h, W4, H4,
+                                                                units, dst);
   return cudaGetLastError();
 }
 
 cudaError_t launch_scatter(const uint8_t *src, int W4, int H4, int units, int w, int h, uint8_t *dst,
                            size_t frame_stride, size_t pitch, int elem_stride, int C, cudaStream_t st) {
-  scatter_kernel<<<grid_for((size_t)units * h * w), 256, 0, st>>>(src, W4, H4, units, w, h, dst, frame_stride, pitch,
-                                                                   elem_stride, C);
+  if (elem_stride == 1 && C == 1)
+    scatter_rows_kernel<<<rows_grid((size_t)units * h), 128, 0, st>>>(src, W4, H4, units, w, h, dst, frame_stride,
+                                                                       pitch);
+  else
+    scatter_kernel<<<rows_grid((size_t)units * h), 128, 0, st>>>(src, W4, H4, units, w, h, dst, frame_stride, pitch,
+                                                                  elem_stride, C);
   return cudaGetLastError();
 }
 
@@ -69,6 +104,7 @@ cudaError_t preload_layout() {
   cudaFuncAttributes a;
   cudaError_t e;
   if ((e = cudaFuncGetAttributes(&a, gather_kernel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, scatter_rows_kernel)) != cudaSuccess) return e;
   return cudaFuncGetAttributes(&a, scatter_kernel);
 }
 
