@@ -38,6 +38,7 @@ constexpr int kWarpCols = 32 * kPx;    // 256 columns per warp tile
 constexpr int kTileRows = 32;          // rows per warp tile (multiple of 4)
 constexpr int kWarps = 4;              // warps per CTA
 constexpr int kThreads = kWarps * 32;
+constexpr int kLutEven = 766;          // entries k = pEdge / 2, pEdge in [0, 1530]
 
 using namespace dev;
 
@@ -171,8 +172,10 @@ __global__ void __launch_bounds__(kThreads) edge_sum_kernel(const uint8_t *__res
   __threadfence();
   const unsigned long long S = atomicAdd(&sums[f], 0ull);
   const double mean = frame_mean(S, W, H, prm.flags);
-  for (int p = threadIdx.x; p < kLutSize; p += kThreads)
-    luts[(size_t)f * kLutSize + p] = p <= 1530 ? lut_entry(p, mean, prm) : make_float2(0.0f, 0.0f);
+  // even pEdge values only (pEdge is always even: Gx and Gy have the parity
+  // of the sum of the window's corners): entry k = lut(2k), k < kLutEven
+  for (int k = threadIdx.x; k < kLutEven; k += kThreads)
+    luts[(size_t)f * kLutSize + k] = lut_entry(2 * k, mean, prm);
   if (threadIdx.x == 0) {
     means[f] = mean;
     counters[f] = 0u;  // re-arm for the next launch
@@ -186,15 +189,19 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
                                                            int tiles_x, int tiles_y,
                                                            const float2 *__restrict__ luts,
                                                            uint8_t *__restrict__ outs, int flags) {
-  __shared__ float2 lut[kLutSize];
+  __shared__ float2 lut[kLutEven];
   const int f = blockIdx.y;
-  for (int i = threadIdx.x; i < kLutSize; i += kThreads) lut[i] = luts[(size_t)f * kLutSize + i];
+  for (int i = threadIdx.x; i < kLutEven; i += kThreads) lut[i] = luts[(size_t)f * kLutSize + i];
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int tile = blockIdx.x * kWarps + warp;
   if (tile >= tiles_x * tiles_y) return;
   // LDS address of lut[p] from the bits of (2^23 + p) as f32: q*8 + base'.
-  const uint32_t lut_base = (uint32_t)__cvta_generic_to_shared(lut) - (0x4B000000u << 3);
+  // byte offset of entry k = pEdge/2: the f32 bits of 2^21 + pEdge minus
+  // 0x4A000000 (ulp 1/4, so 8k); the shared base is uniform (LDS [R+UR])
+  // (the vote makes the base provably warp-uniform: ptxas keeps it in a uniform register)
+  const uint32_t lut_base =
+      (__any_sync(0xffffffffu, (threadIdx.x & 31) == 0) ? (uint32_t)__cvta_generic_to_shared(lut) : 0u) - 0x4A000000u;
 
   const int tx = tile % tiles_x, ty = tile / tiles_x;
   const int c0 = tx * kWarpCols + lane * kPx;
@@ -284,8 +291,8 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
           const uint16_t c_h = hi ? hi16(rb.c[p]) : lo16(rb.c[p]);
           const uint16_t mx_h = hi ? hi16(MX[p]) : lo16(MX[p]);
           const uint16_t mn_h = hi ? hi16(MN[p]) : lo16(MN[p]);
-          const uint32_t q = __float_as_uint(add_f32_f16(pe_h, 8388608.0f));  // 2^23 + pEdge
-          const float2 L = lds_f2(q * 8u + lut_base);                        // {adj, osc}
+          const uint32_t q8 = __float_as_uint(add_f32_f16(pe_h, 2097152.0f));  // 2^21 + pEdge
+          const float2 L = lds_f2(q8 + lut_base);                               // {adj, osc}
           const float E = add_f32_f16(c_h, NU[x]);                           // pError = O - U (L148)
           const float P = __fmaf_rn(L.x, E, -NU[x]);                         // preliminary (L178)
           const float mxf = add_f32_f16(mx_h, 0.0f), mnf = add_f32_f16(mn_h, 0.0f);
