@@ -560,6 +560,28 @@ def main():
         torch.cuda.synchronize()
     kt = sh.kernel_times()
     sh.set_profiling(False)
+    # Latency regime: the same calls captured in a CUDA graph and replayed
+    # ("graph of 1000 reps / 1000"): the device cost of a call
+    # without the host's per-call launch work.
+    graph = None
+    if latency_regime:
+        try:
+            reps = 200
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                for _ in range(reps):
+                    sh.enqueue_batch(d_in, d_out, prm)
+            g.replay()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(5):
+                g.replay()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            graph = {"reps_per_graph": reps, "ms_per_call": e0.elapsed_time(e1) / (5 * reps)}
+        except Exception as ex:  # capture is an extra, never a failure of the run
+            graph = {"unavailable": f"{type(ex).__name__}: {ex}"[:200]}
     total_px = args.frames * fb * (world if args.scaling == "weak" else 1)  # all ranks' frames
     value = total_px / (ms_step * 1e-3) / 1e6
 
@@ -647,6 +669,7 @@ def main():
             "cpu_baseline": cpu,
             "paper_context": paper_context,
             "parity": parity,
+            "cuda_graph": graph,
             "host_numa_binding": "ranks pinned to their GPU's NUMA node" if numa is not None else None,
         }
         print(json.dumps(line), flush=True)
