@@ -316,3 +316,29 @@ def test_maximum_sizes_at_the_step_kernel_limit(W, H, path):
     for r0 in (0, (H // 2) & ~3, H - 32):
         np.testing.assert_array_equal(out[r0:r0 + 32], oracle_rows(img, mean_ref, r0, r0 + 32))
     s.close()
+
+
+def test_randomised_parameters_bit_exact():
+    """300 seeded random parameter sets (A, gamma, G, K over their ranges) x
+    random natural / noise frames: every output bit-exact, S exact.  Stresses
+    the f64 pow / exp of the tables (CUDA libm vs glibc, R19) and
+    the f32 overshoot chain far from the default parameters."""
+    rng = np.random.default_rng(20151016)
+    s = Sharpener()
+    kinds = ["natural", "noise"]
+    imgs = [synth.image(96, 64, kinds[i % 2], seed=synth.BASE_SEED + 900 + i) for i in range(12)]
+    d = [torch.from_numpy(im).cuda() for im in imgs]
+    o = torch.empty_like(d[0])
+    for case in range(300):
+        prm = (float(rng.uniform(0, 16)), float(rng.uniform(0, 4)), float(rng.uniform(0, 1)),
+               float(np.exp(rng.uniform(np.log(1e-3), np.log(1e3)))))
+        prm = tuple(float(np.float32(v)) for v in prm)
+        k = case % len(imgs)
+        s.run(d[k], prm, o)
+        torch.cuda.synchronize()
+        ref, S_ref, _ = oracle.sharpen(imgs[k], *prm)
+        got = o.cpu().numpy()
+        assert s.stats().edge_sum == S_ref
+        bad = np.argwhere(got != ref)
+        assert bad.size == 0, f"case {case} params {prm}: {len(bad)} mismatches, first {bad[:3].tolist()}"
+    s.close()
