@@ -157,10 +157,14 @@ int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int
  * SHARP_EUNSUPPORTED).  Unknown bits -> SHARP_EINVAL.
  *
  * Dense single-channel inputs with w, h multiples of 4 take exactly the
- * sharp_run_batch path (host buffers pipelined, device buffers in one launch);
- * everything else is gathered into dense scratch on the device (host buffers:
- * their byte range is copied up first), run, and scattered back, one chunk of
- * frames at a time.  Synchronous. */
+ * sharp_run_batch path (host buffers pipelined, device buffers in one launch).
+ * Single-channel DEVICE frames with w % 8 == 0, h % 4 == 0, a 16-byte aligned
+ * input with pitch / frame stride multiples of 16 and an 8-byte aligned output
+ * with pitch / frame stride multiples of 8 (e.g. an aligned ROI) run straight
+ * through the step kernel, zero-copy.  Everything else is gathered into padded
+ * scratch on the device (host buffers: their byte range is copied up first),
+ * run (on the step kernel when the padded width is a multiple of 8), and
+ * scattered back, one chunk of frames at a time.  Synchronous. */
 typedef struct {
   size_t pitch;        /* bytes from one row to the next          (0 -> w * elem_stride) */
   size_t frame_stride; /* bytes from one frame to the next        (0 -> pitch * h)       */

@@ -41,16 +41,18 @@ cudaError_t launch_sharpen(const uint8_t *imgs, int n, int W, int H, const float
 // General layouts (layout.cu): units u = f * C + c
 // (frame f, channel c) of a strided source -> dense [units][H4][W4] with the
 // last column / row replicated (R1'), and back (top-left w x h only).
+// The padded units are [units][H4][P] (row pitch P >= W4; P = W4 is dense).
 cudaError_t launch_gather(const uint8_t *src, size_t frame_stride, size_t pitch, int elem_stride, int C, int w,
-                          int h, int W4, int H4, int units, uint8_t *dst, cudaStream_t st);
-cudaError_t launch_scatter(const uint8_t *src, int W4, int H4, int units, int w, int h, uint8_t *dst,
+                          int h, int W4, int H4, int P, int units, uint8_t *dst, cudaStream_t st);
+cudaError_t launch_scatter(const uint8_t *src, int P, int H4, int units, int w, int h, uint8_t *dst,
                            size_t frame_stride, size_t pitch, int elem_stride, int C, cudaStream_t st);
 cudaError_t preload_layout();
 
 // TMA-staged, persistent, dynamically scheduled kernel (kernels_tma.cu) for a
 // whole batch in ONE launch (pass 1, per-frame LUT build and pass 2 as tasks
 // with in-kernel dependencies), used when tma_supported() (W % 16 == 0,
-// W*H <= 2^29, 16-byte aligned input, 8-byte aligned output).
+// W*H <= 2^29, 16-byte aligned input, 8-byte aligned output) or, for strided
+// frames, tma_supported_strided().
 struct BatchLaunch {
   const uint8_t *in = nullptr;  // [n][H][W]
   int n = 0;
@@ -64,8 +66,17 @@ struct BatchLaunch {
   // row-band launches only (launch_band_tma):
   unsigned long long *partial = nullptr;      // pass 1 out: the band's S
   const unsigned long long *total = nullptr;  // pass 2 in: the all-reduced S
+  // strided frames (sharp_run_ex): bytes between rows / frames; 0 -> dense
+  size_t in_pitch = 0, in_fs = 0, out_pitch = 0, out_fs = 0;
 };
+// Dense [n][H][W] frames: W % 16 == 0 (the TMA row stride), 16-byte aligned
+// input, 8-byte aligned output, H >= 8, W * H <= 2^29.
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);
+// Strided frames: W % 8 == 0 (lane tiles end on the image's last column),
+// in_pitch / in_fs multiples of 16 (TMA strides), out_pitch / out_fs
+// multiples of 8 (8-byte stores), the same base alignments and limits.
+bool tma_supported_strided(const uint8_t *imgs, size_t in_pitch, size_t in_fs, const uint8_t *outs, size_t out_pitch,
+                           size_t out_fs, int W, int H);
 cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
 
 // One row band [row_lo, row_hi) of a W x H image (sec. 8(e)): a.in holds

@@ -252,6 +252,7 @@ struct StepParams {
   float2 *luts;             // per frame: kLutSize entries {adj, osc}
   unsigned int *lut_done;   // per frame: finished LUT-task warps; zero on entry
   uint8_t *out;
+  size_t out_pitch, out_fs;  // output bytes between rows / frames
   unsigned int *task_counter;  // zero on entry
 };
 // acc packing: S <= 1530 * W * H < 2^40 for W * H <= 2^29 (tma_supported),
@@ -514,7 +515,7 @@ struct Ring {
 // ring tests -- is 40% SLOWER: ~36 KB of straight-line code overflows the
 // instruction cache.  The hot loops must stay small.)
 __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint32_t lut0, int lut_odd,
-                                        uint8_t *__restrict__ out,
+                                        uint8_t *__restrict__ out, size_t out_pitch,
                                         int W, int H, int row_lo, int row_hi, int C0w, int R0, int warp,
                                         int lane) {
 #ifdef SHARP_EXP_NO_P2  // timing experiment only
@@ -526,7 +527,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 #endif
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
-  // W % 16 == 0: image columns 0,1 are in the lane with c0 == 0, columns
+  // W % 8 == 0: image columns 0,1 are in the lane with c0 == 0, columns
   // W-2,W-1 in the lane with c0 == W-8.
   const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
@@ -552,7 +553,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   float4 slope = f4twice_diff(D1, Dp);
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
-  uint8_t *orow = out + (size_t)(R0 - row_lo) * W + c0;
+  uint8_t *orow = out + (size_t)(R0 - row_lo) * out_pitch + c0;
 #pragma unroll 1
   for (int k = 0; k < nsub; ++k) {
     const int R0k = R0 + k * kTH;
@@ -580,7 +581,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
         const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
         p2_row<true>(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
         V = f4add(V, slope);
-        orow += W;
+        orow += out_pitch;
         ra = rb;
         rb = rc;
       }
@@ -787,7 +788,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       const int C0 = d.z, R0 = d.w, C0w = C0 + warp * kTW;
       if (lane == 0) TL_MIN(5);
       if (C0w < g.W) {
-        p2_warp(ring, s, aux.x, lutbase, aux.y, sp.out + (size_t)d.y * g.W * g.H, g.W, g.H,
+        p2_warp(ring, s, aux.x, lutbase, aux.y, sp.out + (size_t)d.y * sp.out_fs, sp.out_pitch, g.W, g.H,
                 g.row_lo, g.row_hi, C0w, R0, warp, lane);
       } else {  // no columns for this warp: follow the stages
         for (int k = 0; k < aux.x; ++k) {
@@ -848,11 +849,12 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, int box_cols, int box_rows) {
+bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, size_t pitch, size_t fs, int box_cols,
+              int box_rows) {
   auto fn = encode_fn();
   if (!fn) return false;
-  const cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)n};  // [n][H][W]
-  const cuuint64_t strides[2] = {(cuuint64_t)W, (cuuint64_t)W * H};
+  const cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)n};  // [n][H][W] at the given strides
+  const cuuint64_t strides[2] = {(cuuint64_t)pitch, (cuuint64_t)fs};
   const cuuint32_t box[3] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows, 1};
   const cuuint32_t estr[3] = {1, 1, 1};
   return fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, (void *)imgs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -898,8 +900,14 @@ extern "C" int sharp_debug_waitstat(unsigned long long *out, int reset) {
 #endif
 
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
-  return (W % 16) == 0 && (((uintptr_t)imgs) & 15) == 0 && (((uintptr_t)outs) & 7) == 0 && H >= 8 &&
-         (size_t)W * H <= (1u << 29) && encode_fn() != nullptr;
+  return (W % 16) == 0 && tma_supported_strided(imgs, W, (size_t)W * H, outs, W, (size_t)W * H, W, H);
+}
+
+bool tma_supported_strided(const uint8_t *imgs, size_t in_pitch, size_t in_fs, const uint8_t *outs, size_t out_pitch,
+                           size_t out_fs, int W, int H) {
+  return (W % 8) == 0 && W >= 8 && (((uintptr_t)imgs) & 15) == 0 && (in_pitch % 16) == 0 && (in_fs % 16) == 0 &&
+         in_pitch >= (size_t)W && (((uintptr_t)outs) & 7) == 0 && (out_pitch % 8) == 0 && (out_fs % 8) == 0 &&
+         out_pitch >= (size_t)W && H >= 8 && (size_t)W * H <= (1u << 29) && encode_fn() != nullptr;
 }
 
 // Row-band helpers (one thread): arm a band's pass-2 launch with the
@@ -930,8 +938,11 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   if (sg.n <= 0 || sg.row_hi <= sg.row_lo) return cudaSuccess;
   CUtensorMap m1A, m1B, m2A, m2B;  // the same frames: pass-1 / pass-2 box heights, regions A / B
   const int R = sg.rows_in;
-  if (!make_map(&m1A, a.in, sg.n, W, R, kPitch, kRows1) || !make_map(&m1B, a.in, sg.n, W, R, kPitchB, kRows1) ||
-      !make_map(&m2A, a.in, sg.n, W, R, kPitch, kRows2) || !make_map(&m2B, a.in, sg.n, W, R, kPitchB, kRows2))
+  const size_t ip = a.in_pitch ? a.in_pitch : (size_t)W, ifs = a.in_fs ? a.in_fs : ip * R;
+  if (!make_map(&m1A, a.in, sg.n, W, R, ip, ifs, kPitch, kRows1) ||
+      !make_map(&m1B, a.in, sg.n, W, R, ip, ifs, kPitchB, kRows1) ||
+      !make_map(&m2A, a.in, sg.n, W, R, ip, ifs, kPitch, kRows2) ||
+      !make_map(&m2B, a.in, sg.n, W, R, ip, ifs, kPitchB, kRows2))
     return cudaErrorInvalidValue;
   StepParams sp;
   sp.g.W = W;
@@ -1002,6 +1013,8 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.luts = a.luts;
   sp.lut_done = a.lut_done;
   sp.out = a.out;
+  sp.out_pitch = a.out_pitch ? a.out_pitch : (size_t)W;
+  sp.out_fs = a.out_fs ? a.out_fs : sp.out_pitch * (size_t)H;
   sp.task_counter = a.task_counter;
   if (mode == kStepPass2) {
     band_prep_kernel<<<1, 1, 0, stream>>>(a.acc, a.lut_done, a.task_counter, a.total,

@@ -20,12 +20,12 @@ namespace {
 // Dense padded row r of unit u <- source row min(r, h-1), columns clamped to
 // w-1 (replicate, R1'); one 32-bit store per 4 bytes.
 __global__ void gather_kernel(const uint8_t *__restrict__ src, size_t fs, size_t pitch, int es, int C, int w, int h,
-                              int W4, int H4, int units, uint8_t *__restrict__ dst) {
+                              int W4, int H4, int P, int units, uint8_t *__restrict__ dst) {
   const int q4 = W4 >> 2;
   for (unsigned ur = blockIdx.x; ur < (unsigned)units * (unsigned)H4; ur += gridDim.x) {
     const unsigned u = ur / (unsigned)H4, r = ur - u * (unsigned)H4;
     const uint8_t *row = src + (size_t)(u / C) * fs + (size_t)(u % C) + (size_t)min((int)r, h - 1) * pitch;
-    uint32_t *drow = reinterpret_cast<uint32_t *>(dst + (size_t)ur * W4);
+    uint32_t *drow = reinterpret_cast<uint32_t *>(dst + (size_t)ur * P);
     for (int q = threadIdx.x; q < q4; q += blockDim.x) {
       uint32_t v = 0;
       if (es == 1 && 4 * q + 3 < w) {
@@ -46,12 +46,12 @@ __global__ void gather_kernel(const uint8_t *__restrict__ src, size_t fs, size_t
 
 // Single-channel rows (elem_stride 1): per destination row, 16-byte stores
 // where the destination is aligned (the row interior), bytes at the ends.
-__global__ void scatter_rows_kernel(const uint8_t *__restrict__ src, int W4, int H4, int units, int w, int h,
+__global__ void scatter_rows_kernel(const uint8_t *__restrict__ src, int P, int H4, int units, int w, int h,
                                     uint8_t *__restrict__ dst, size_t fs, size_t pitch) {
   for (unsigned ur = blockIdx.x; ur < (unsigned)units * (unsigned)h; ur += gridDim.x) {
     const unsigned u = ur / (unsigned)h, r = ur - u * (unsigned)h;
     uint8_t *drow = dst + (size_t)u * fs + (size_t)r * pitch;
-    const uint8_t *srow = src + ((size_t)u * H4 + r) * W4;
+    const uint8_t *srow = src + ((size_t)u * H4 + r) * P;
     const int lead = min(w, (int)((16 - ((uintptr_t)drow & 15)) & 15));  // bytes before the first aligned one
     const int nvec = (w - lead) / 16;
     for (int c = threadIdx.x; c < lead; c += blockDim.x) drow[c] = srow[c];
@@ -68,12 +68,12 @@ __global__ void scatter_rows_kernel(const uint8_t *__restrict__ src, int W4, int
 }
 
 // Any layout (interleaved channels): a byte per thread.
-__global__ void scatter_kernel(const uint8_t *__restrict__ src, int W4, int H4, int units, int w, int h,
+__global__ void scatter_kernel(const uint8_t *__restrict__ src, int P, int H4, int units, int w, int h,
                                uint8_t *__restrict__ dst, size_t fs, size_t pitch, int es, int C) {
   for (unsigned ur = blockIdx.x; ur < (unsigned)units * (unsigned)h; ur += gridDim.x) {
     const unsigned u = ur / (unsigned)h, r = ur - u * (unsigned)h;
     uint8_t *drow = dst + (size_t)(u / C) * fs + (size_t)(u % C) + (size_t)r * pitch;
-    const uint8_t *srow = src + ((size_t)u * H4 + r) * W4;
+    const uint8_t *srow = src + ((size_t)u * H4 + r) * P;
     for (int c = threadIdx.x; c < w; c += blockDim.x) drow[(size_t)c * es] = srow[c];
   }
 }
@@ -83,19 +83,19 @@ unsigned rows_grid(size_t rows) { return (unsigned)(rows < 148 * 16 ? (rows ? ro
 }  // namespace
 
 cudaError_t launch_gather(const uint8_t *src, size_t frame_stride, size_t pitch, int elem_stride, int C, int w,
-                          int h, int W4, int H4, int units, uint8_t *dst, cudaStream_t st) {
+                          int h, int W4, int H4, int P, int units, uint8_t *dst, cudaStream_t st) {
   gather_kernel<<<rows_grid((size_t)units * H4), 128, 0, st>>>(src, frame_stride, pitch, elem_stride, C, w, h, W4, H4,
-                                                                units, dst);
+                                                                P, units, dst);
   return cudaGetLastError();
 }
 
-cudaError_t launch_scatter(const uint8_t *src, int W4, int H4, int units, int w, int h, uint8_t *dst,
+cudaError_t launch_scatter(const uint8_t *src, int P, int H4, int units, int w, int h, uint8_t *dst,
                            size_t frame_stride, size_t pitch, int elem_stride, int C, cudaStream_t st) {
   if (elem_stride == 1 && C == 1)
-    scatter_rows_kernel<<<rows_grid((size_t)units * h), 128, 0, st>>>(src, W4, H4, units, w, h, dst, frame_stride,
+    scatter_rows_kernel<<<rows_grid((size_t)units * h), 128, 0, st>>>(src, P, H4, units, w, h, dst, frame_stride,
                                                                        pitch);
   else
-    scatter_kernel<<<rows_grid((size_t)units * h), 128, 0, st>>>(src, W4, H4, units, w, h, dst, frame_stride, pitch,
+    scatter_kernel<<<rows_grid((size_t)units * h), 128, 0, st>>>(src, P, H4, units, w, h, dst, frame_stride, pitch,
                                                                   elem_stride, C);
   return cudaGetLastError();
 }

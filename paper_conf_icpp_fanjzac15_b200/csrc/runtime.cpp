@@ -299,10 +299,18 @@ void stage_rec(void *vctx, int stage, int begin, cudaStream_t st) {
 //    launch c+1 re-reads it.  LUT buffers alternate between chunk parities.
 //  * generic path: pass 1 then pass 2 per chunk.
 // `tc` points at this call's zeroed task counters (one per step launch).
+// Byte strides of device frames (0 = dense); only the step kernel takes
+// strided frames, the other paths need dense ones.
+struct Strides {
+  size_t in_pitch = 0, in_fs = 0, out_pitch = 0, out_fs = 0;
+  bool dense() const { return !in_pitch && !in_fs && !out_pitch && !out_fs; }
+};
+
 int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, const sharp::Params &prm,
                    uint8_t *dout, cudaStream_t st, Slot &slot, size_t chunk, size_t frame_base, int *launches,
-                   unsigned int *tc) {
+                   unsigned int *tc, const Strides &str = Strides()) {
   const size_t fb = (size_t)w * h;
+  if (!str.dense() && ctx->path == SHARP_PATH_STAGED) return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "strided frames on the staged path");
   const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
   if (ctx->path == SHARP_PATH_STAGED) {  // the paper's base design: K1..K7 per frame
     if ((rc_staged(ctx, w, h))) return SHARP_ENOMEM;
@@ -320,7 +328,11 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   }
   // The step kernel implements the LUT-only reading switches; R2 / R5 / R14
   // change per-pixel arithmetic and run on the two-pass path.
-  const bool tma_ok = sharp::tma_supported(din, dout, w, h) && !(prm.flags & sharp::kReadPerPixel);
+  const bool tma_ok = (str.dense() ? sharp::tma_supported(din, dout, w, h)
+                                    : sharp::tma_supported_strided(din, str.in_pitch, str.in_fs, dout, str.out_pitch,
+                                                                   str.out_fs, w, h)) &&
+                      !(prm.flags & sharp::kReadPerPixel);
+  if (!str.dense() && !tma_ok) return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "strided frames need the step kernel");
   if (ctx->path == SHARP_PATH_STEP && !tma_ok)
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
                    "SHARP_PATH_STEP needs w % 16 == 0, 16-byte aligned input, 8-byte aligned output, w*h <= 2^29 "
@@ -337,6 +349,10 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
     a.luts = ctx->luts + frame_base * sharp::kLutSize;
     a.lut_done = ctx->lut_done + frame_base;
     a.task_counter = tc;
+    a.in_pitch = str.in_pitch;
+    a.in_fs = str.in_fs;
+    a.out_pitch = str.out_pitch;
+    a.out_fs = str.out_fs;
     CK(timed(ctx, st, 3, (double)n * fb, [&] { return sharp::launch_batch_tma(a, w, h, prm, st); }));
     *launches += 1;
     return SHARP_OK;
@@ -491,7 +507,15 @@ constexpr size_t kGeneralChunkBytes = 256u << 20;  // dense padded bytes per chu
 int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int C, int w, int h,
                 const sharp::Params &prm, uint8_t *out, const Layout &Lo, Kind kin, Kind kout) {
   const int W4 = (w + 3) & ~3, H4 = (h + 3) & ~3;
-  const size_t ub = (size_t)W4 * H4;
+  // Units whose padded width is a multiple of 8 run on the step kernel from a
+  // scratch with a 16-byte row pitch (the TMA stride rule); others dense on
+  // the two-pass path.
+  const bool step = (W4 % 8) == 0 && H4 >= 8 && (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+                    !(prm.flags & sharp::kReadPerPixel) && (size_t)W4 * H4 <= (1u << 29);
+  const int P = step ? (W4 + 15) & ~15 : W4;
+  const size_t ub = (size_t)P * H4;
+  Strides str;
+  if (P != W4) str = Strides{(size_t)P, ub, (size_t)P, ub};
   // frames per chunk: sharp_config.chunk_frames if set, else ~kGeneralChunkBytes of padded units
   const int fpc = ctx->chunk_cfg > 0 ? std::min(ctx->chunk_cfg, n)
                                      : (int)std::max<size_t>(1, std::min<size_t>((size_t)n, kGeneralChunkBytes / (ub * C)));
@@ -517,25 +541,25 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
       CK(cudaMemcpyAsync(ctx->gx_src, src, span, cudaMemcpyHostToDevice, ctx->stream));
       src = ctx->gx_src;
     }
-    CK(sharp::launch_gather(src, Li.fs, Li.pitch, Li.es, C, w, h, W4, H4, units, ctx->gx_in, ctx->stream));
+    CK(sharp::launch_gather(src, Li.fs, Li.pitch, Li.es, C, w, h, W4, H4, P, units, ctx->gx_in, ctx->stream));
     CK(cudaMemsetAsync(ctx->sums + u0, 0, units * sizeof(unsigned long long), ctx->stream));
     CK(cudaMemsetAsync(ctx->lut_done + u0, 0, units * sizeof(unsigned int), ctx->stream));
     CK(cudaMemsetAsync(ctx->acc + u0, 0, units * sizeof(unsigned long long), ctx->stream));
     CK(cudaMemsetAsync(ctx->tcounters, 0, sizeof(unsigned int), ctx->stream));
     if ((rc = enqueue_device(ctx, ctx->gx_in, units, W4, H4, prm, ctx->gx_out, ctx->stream, ctx->slots[0],
-                             std::min(chunk, (size_t)units), u0, &launches, ctx->tcounters)))
+                             std::min(chunk, (size_t)units), u0, &launches, ctx->tcounters, str)))
       return rc;
     // the w x h crops into the caller's layout (a host destination goes
     // through a device copy of its byte range, so bytes between the pixels
     // keep their values)
     uint8_t *dst = out + (size_t)f0 * Lo.fs;
     if (kout == kDevice) {
-      CK(sharp::launch_scatter(ctx->gx_out, W4, H4, units, w, h, dst, Lo.fs, Lo.pitch, Lo.es, C, ctx->stream));
+      CK(sharp::launch_scatter(ctx->gx_out, P, H4, units, w, h, dst, Lo.fs, Lo.pitch, Lo.es, C, ctx->stream));
     } else {
       const size_t span = layout_span(Lo, fn, C, w, h);
       if ((rc = grow(ctx, &ctx->gx_dst, &ctx->gx_dst_cap, span))) return rc;
       CK(cudaMemcpyAsync(ctx->gx_dst, dst, span, cudaMemcpyHostToDevice, ctx->stream));
-      CK(sharp::launch_scatter(ctx->gx_out, W4, H4, units, w, h, ctx->gx_dst, Lo.fs, Lo.pitch, Lo.es, C,
+      CK(sharp::launch_scatter(ctx->gx_out, P, H4, units, w, h, ctx->gx_dst, Lo.fs, Lo.pitch, Lo.es, C,
                                ctx->stream));
       CK(cudaMemcpyAsync(dst, ctx->gx_dst, span, cudaMemcpyDeviceToHost, ctx->stream));
     }
@@ -557,6 +581,36 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
   ctx->stats.edge_mean = m0;
   ctx->stats.device_ms = ms;
   ctx->stats.total_ms = ms;
+  return SHARP_OK;
+}
+
+// Device-resident strided frames straight through the step kernel (no
+// copies): an ROI / pitched batch whose strides meet the TMA rules.
+int run_device_strided(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int w, int h,
+                       const sharp::Params &prm, uint8_t *out, const Layout &Lo) {
+  const auto t0 = std::chrono::steady_clock::now();
+  int rc;
+  if ((rc = ensure_frames(ctx, (size_t)n))) return rc;
+  if ((rc = ensure_slots(ctx, 1, (size_t)w * h, false))) return rc;
+  CK(cudaMemsetAsync(ctx->zero_block, 0, ctx->zero_bytes, ctx->stream));
+  CK(cudaEventRecord(ctx->ev_start, ctx->stream));
+  int launches = 0;
+  if ((rc = enqueue_device(ctx, in, n, w, h, prm, out, ctx->stream, ctx->slots[0], (size_t)n, 0, &launches,
+                           ctx->tcounters, Strides{Li.pitch, Li.fs, Lo.pitch, Lo.fs})))
+    return rc;
+  CK(cudaEventRecord(ctx->ev_stop, ctx->stream));
+  CK(cudaMemcpyAsync(&ctx->h_stats->sum, ctx->sums, sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaMemcpyAsync(&ctx->h_stats->mean, ctx->means, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  float ms = 0.0f;
+  CK(cudaEventElapsedTime(&ms, ctx->ev_start, ctx->ev_stop));
+  ctx->last_frames = n;
+  ctx->stats.frames = n;
+  ctx->stats.kernels = launches;
+  ctx->stats.edge_sum = ctx->h_stats->sum;
+  ctx->stats.edge_mean = ctx->h_stats->mean;
+  ctx->stats.device_ms = ms;
+  ctx->stats.total_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
   return SHARP_OK;
 }
 
@@ -593,6 +647,13 @@ int run_ex_impl(sharp_ctx *ctx, const uint8_t *in, const sharp_layout *lin, int 
   int rc;
   if ((rc = classify(ctx, in, &kin)) || (rc = classify(ctx, out, &kout))) return rc;
   CK(cudaSetDevice(ctx->device));
+  // zero-copy: single-channel device frames with w % 8 == 0, h % 4 == 0 and
+  // strides the TMA step kernel takes directly
+  if (C == 1 && Li.es == 1 && Lo.es == 1 && !overlap && kin == kDevice && kout == kDevice && !(w & 7) && !(h & 3) &&
+      w >= 8 && h >= 8 && (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+      !(flags & sharp::kReadPerPixel) &&
+      sharp::tma_supported_strided(in, Li.pitch, Li.fs, out, Lo.pitch, Lo.fs, w, h))
+    return run_device_strided(ctx, in, Li, n, w, h, prm, out, Lo);
   return run_general(ctx, in, Li, n, C, w, h, prm, out, Lo, kin, kout);
 }
 

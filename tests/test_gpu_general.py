@@ -251,3 +251,47 @@ def test_reading_switches_host_pipeline(flags):
         check(out[f].numpy(), refs[f], f"frame {f}")
     assert s.batch_sums(5) == sums
     s.close()
+
+
+@pytest.mark.parametrize("W,H,pitch_in,pitch_out", [(1928, 64, 2000, 1944), (488, 36, 528, 496), (960, 12, 1008, 968)])
+def test_zero_copy_strided_roi_on_the_step_kernel(W, H, pitch_in, pitch_out):
+    """Device ROIs whose strides meet the TMA rules (W % 8 == 0, input pitch
+    % 16, output pitch % 8, aligned bases) run straight through the step
+    kernel -- no gather / scatter copies -- including W % 16 == 8."""
+    s = Sharpener()
+    big = synth.frames(2, pitch_in, H + 8, "natural", seed=synth.BASE_SEED + W)
+    t = torch.from_numpy(big).cuda()
+    roi = t[:, 4:4 + H, 32:32 + W]                      # base 16-byte aligned (offset 4 * pitch + 32)
+    ob = torch.full((2, H + 4, pitch_out), 7, dtype=torch.uint8, device="cuda")
+    out = ob[:, 2:2 + H, 8:8 + W]                       # 8-byte aligned
+    s.set_profiling(True)
+    s.run_ex(roi, STRONG, out=out)
+    torch.cuda.synchronize()
+    kt = s.kernel_times()
+    assert kt.step_launches == 1 and s.stats().kernels == 1   # one launch, no layout kernels
+    refs, sums = ref_units([np.ascontiguousarray(big[f, 4:4 + H, 32:32 + W]) for f in range(2)], STRONG, 0)
+    o = ob.cpu().numpy()
+    for f in range(2):
+        check(o[f, 2:2 + H, 8:8 + W], refs[f], f"frame {f}")
+    mask = np.ones(o.shape, bool)
+    mask[:, 2:2 + H, 8:8 + W] = False
+    assert np.all(o[mask] == 7)
+    assert s.batch_sums(2) == sums
+    s.close()
+
+
+@pytest.mark.parametrize("W,H", [(1925, 30), (5, 8), (61, 21)])
+def test_general_sizes_padded_to_a_16_byte_pitch(W, H):
+    """Padded width W4 % 16 == 8: the gathered scratch gets a 16-byte row pitch
+    and the units run on the step kernel with strided tensor maps."""
+    s = Sharpener()
+    imgs = np.ascontiguousarray(synth.frames(2, W + 3, H + 3, "natural", seed=synth.BASE_SEED + 3 * W)[:, :H, :W])
+    s.set_profiling(True)
+    out = s.run_ex(torch.from_numpy(imgs).cuda(), STRONG)
+    torch.cuda.synchronize()
+    assert s.kernel_times().step_launches == 1
+    refs, sums = ref_units(list(imgs), STRONG, 0)
+    for f in range(2):
+        check(out[f].cpu().numpy(), refs[f], f"frame {f}")
+    assert s.batch_sums(2) == sums
+    s.close()
