@@ -158,7 +158,7 @@ int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int
  *
  * Dense single-channel inputs with w, h multiples of 4 take exactly the
  * sharp_run_batch path (host buffers pipelined, device buffers in one launch).
- * Single-channel DEVICE frames with w % 8 == 0, h % 4 == 0, a 16-byte aligned
+ * Single-channel DEVICE frames with w % 8 == 0 (w >= 16), h % 4 == 0, a 16-byte aligned
  * input with pitch / frame stride multiples of 16 and an 8-byte aligned output
  * with pitch / frame stride multiples of 8 (e.g. an aligned ROI) run straight
  * through the step kernel, zero-copy.  Everything else is gathered into padded

@@ -905,7 +905,8 @@ bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
 
 bool tma_supported_strided(const uint8_t *imgs, size_t in_pitch, size_t in_fs, const uint8_t *outs, size_t out_pitch,
                            size_t out_fs, int W, int H) {
-  return (W % 8) == 0 && W >= 8 && (((uintptr_t)imgs) & 15) == 0 && (in_pitch % 16) == 0 && (in_fs % 16) == 0 &&
+  // (W >= 16: columns 0,1 and W-2,W-1 must sit in different lanes)
+  return (W % 8) == 0 && W >= 16 && (((uintptr_t)imgs) & 15) == 0 && (in_pitch % 16) == 0 && (in_fs % 16) == 0 &&
          in_pitch >= (size_t)W && (((uintptr_t)outs) & 7) == 0 && (out_pitch % 8) == 0 && (out_fs % 8) == 0 &&
          out_pitch >= (size_t)W && H >= 8 && (size_t)W * H <= (1u << 29) && encode_fn() != nullptr;
 }

@@ -373,6 +373,13 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   return SHARP_OK;
 }
 
+struct Layout {
+  size_t pitch, fs;
+  int es;
+};
+int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int C, int w, int h,
+                const sharp::Params &prm, uint8_t *out, const Layout &Lo, Kind kin, Kind kout);
+
 int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp_params *pp, uint8_t *out,
              bool async, int flags = 0) {
   int rc = validate(ctx, in, out, n, w, h, pp);
@@ -388,6 +395,15 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   if ((kin == kDevice && ((uintptr_t)in & 3)) || (kout == kDevice && ((uintptr_t)out & 3)))
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "device buffers must be 4-byte aligned");
   CK(cudaSetDevice(ctx->device));
+  // Device frames with w % 16 == 8 cannot be TMA tensors in place (16-byte
+  // row stride): through a 16-byte-pitch scratch they still run on the step
+  // kernel (gather + scatter cost 4 B/px, far less than the two-pass path's
+  // compute at these widths).  Synchronous calls only.
+  if (!async && kin == kDevice && kout == kDevice && (w % 16) == 8 && w >= 24 && !(prm.flags & sharp::kReadPerPixel) &&
+      (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) && (size_t)w * h <= (1u << 29)) {
+    const Layout L{(size_t)w, (size_t)w * h, 1};
+    return run_general(ctx, in, L, n, 1, w, h, prm, out, L, kin, kout);
+  }
   const auto t0 = std::chrono::steady_clock::now();
   const size_t fb = (size_t)w * h;
   const bool staged = !(kin == kDevice && kout == kDevice);
@@ -474,11 +490,6 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
 
 
 // ---- General layouts (R1').
-struct Layout {
-  size_t pitch, fs;
-  int es;
-};
-
 bool layout_of(const sharp_layout *l, int w, int h, Layout *o) {
   o->es = (l && l->elem_stride > 0) ? l->elem_stride : 1;
   o->pitch = (l && l->pitch) ? l->pitch : (size_t)w * o->es;
@@ -510,7 +521,7 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
   // Units whose padded width is a multiple of 8 run on the step kernel from a
   // scratch with a 16-byte row pitch (the TMA stride rule); others dense on
   // the two-pass path.
-  const bool step = (W4 % 8) == 0 && H4 >= 8 && (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+  const bool step = (W4 % 8) == 0 && W4 >= 16 && H4 >= 8 && (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
                     !(prm.flags & sharp::kReadPerPixel) && (size_t)W4 * H4 <= (1u << 29);
   const int P = step ? (W4 + 15) & ~15 : W4;
   const size_t ub = (size_t)P * H4;

@@ -280,7 +280,7 @@ def test_zero_copy_strided_roi_on_the_step_kernel(W, H, pitch_in, pitch_out):
     s.close()
 
 
-@pytest.mark.parametrize("W,H", [(1925, 30), (5, 8), (61, 21)])
+@pytest.mark.parametrize("W,H", [(1925, 30), (13, 8), (61, 21)])
 def test_general_sizes_padded_to_a_16_byte_pitch(W, H):
     """Padded width W4 % 16 == 8: the gathered scratch gets a 16-byte row pitch
     and the units run on the step kernel with strided tensor maps."""
@@ -294,4 +294,21 @@ def test_general_sizes_padded_to_a_16_byte_pitch(W, H):
     for f in range(2):
         check(out[f].cpu().numpy(), refs[f], f"frame {f}")
     assert s.batch_sums(2) == sums
+    s.close()
+
+
+@pytest.mark.parametrize("W,H", [(1928, 40), (24, 16), (3848, 12)])
+def test_dense_width_8_mod_16_runs_on_the_step_kernel(W, H):
+    """sharp_run_batch on device frames with W % 16 == 8 (not a TMA row stride
+    in place): through a 16-byte-pitch scratch onto the step kernel."""
+    s = Sharpener()
+    imgs = synth.frames(3, W, H, "natural", seed=synth.BASE_SEED + W + H)
+    d = torch.from_numpy(imgs).cuda()
+    s.set_profiling(True)
+    out = s.run_batch(d, STRONG)
+    torch.cuda.synchronize()
+    assert s.kernel_times().step_launches == 1
+    ref, sums = oracle.sharpen_batch(imgs, *STRONG)
+    check(out.cpu().numpy(), ref, f"{W}x{H}")
+    assert s.batch_sums(3) == [int(x) for x in sums]
     s.close()
