@@ -515,7 +515,7 @@ struct Ring {
 // ring tests -- is 40% SLOWER: ~36 KB of straight-line code overflows the
 // instruction cache.  The hot loops must stay small.)
 __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint32_t lut0, int lut_odd,
-                                        uint8_t *__restrict__ out, size_t out_pitch,
+                                        uint8_t *__restrict__ out, uint32_t out_pitch,
                                         int W, int H, int row_lo, int row_hi, int C0w, int R0, int warp,
                                         int lane) {
 #ifdef SHARP_EXP_NO_P2  // timing experiment only
@@ -788,7 +788,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       const int C0 = d.z, R0 = d.w, C0w = C0 + warp * kTW;
       if (lane == 0) TL_MIN(5);
       if (C0w < g.W) {
-        p2_warp(ring, s, aux.x, lutbase, aux.y, sp.out + (size_t)d.y * sp.out_fs, sp.out_pitch, g.W, g.H,
+        p2_warp(ring, s, aux.x, lutbase, aux.y, sp.out + (size_t)d.y * sp.out_fs, (uint32_t)sp.out_pitch, g.W, g.H,
                 g.row_lo, g.row_hi, C0w, R0, warp, lane);
       } else {  // no columns for this warp: follow the stages
         for (int k = 0; k < aux.x; ++k) {
