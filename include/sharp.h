@@ -281,7 +281,8 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
  *   SHARP_PATH_AUTO     the step kernel where it applies, else the two-pass path (default)
  *   SHARP_PATH_STEP     one persistent TMA-staged launch per batch (kernels_tma.cu): pass 1,
  *                       per-frame LUT and pass 2 as dynamically scheduled tasks with
- *                       in-kernel dependencies; needs w % 16 == 0, 16-byte aligned input,
+ *                       in-kernel dependencies; needs w % 16 == 0 (sharp_run_ex: any w % 8 == 0,
+ *                       w >= 16, through strided tensor maps), 16-byte aligned input,
  *                       8-byte aligned output, w*h <= 2^29, else SHARP_EUNSUPPORTED
  *   SHARP_PATH_TWO_PASS two fused kernels per chunk of frames (kernels.cu): Sobel +
  *                       reduction + LUT, then everything else; any w % 4 == 0
