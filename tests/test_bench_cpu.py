@@ -1,0 +1,56 @@
+"""CPU checks of bench.py's contract logic (no GPU): the workload description
+for weak / strong scaling, the reference arm's line, the NUMA cpulist
+parsing.  The timed paths themselves need a B200 (driver runs)."""
+import argparse
+import importlib.util
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def load_bench():
+    spec = importlib.util.spec_from_file_location("bench", os.path.join(ROOT, "bench.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    return m
+
+
+def test_workload_config_weak_and_strong():
+    b = load_bench()
+    a = argparse.Namespace(frames=1024, width=1920, height=1080, scaling="weak")
+    w = b.workload_config(a, 8)
+    assert w["frames"] == 8 * 1024 and w["frames_per_gpu"] == 1024 and "per GPU" in w["workload"]
+    a.scaling = "strong"
+    st = b.workload_config(a, 8)
+    assert st["frames"] == 1024 and st["frames_per_gpu"] is None and "split over 8" in st["parallelism"]
+    a.scaling = "weak"
+    assert b.workload_config(a, 1)["frames"] == b.workload_config(argparse.Namespace(
+        frames=1024, width=1920, height=1080, scaling="strong"), 1)["frames"]
+
+
+def test_reference_arm_line_on_cpu():
+    """--impl reference runs the oracle on host cores (no GPU) and prints the
+    contract's line with impl, cpu_baseline and a zero-transfer e2e."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--steps", "1",
+                        "--warmup", "0", "--ref-sample", "2", "--width", "256", "--height", "128", "--frames", "8"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr
+    line = json.loads(r.stdout.strip().splitlines()[-1])
+    assert line["impl"] == "reference" and line["unit"] == "Mpix/s" and line["value"] > 0
+    assert line["cpu_baseline"]["kind"] == "oracle" and line["e2e"]["h2d_bytes_per_step"] == 0
+    assert line["scaling"] == "weak" and line["higher_is_better"] is True
+
+
+def test_numa_binding_is_best_effort_without_a_gpu():
+    b = load_bench()
+
+    class NoGpu:
+        class cuda:
+            @staticmethod
+            def get_device_properties(i):
+                raise AttributeError("no GPU")
+
+    assert b.bind_to_gpu_numa_node(NoGpu, 0) is None
