@@ -561,6 +561,10 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
   if ((rc = grow(ctx, &ctx->gx_in, &ctx->gx_cap, cu_max * ub))) return rc;
   if ((rc = grow(ctx, &ctx->gx_out, &ctx->gx_out_cap, cu_max * ub))) return rc;
   int launches = 0;
+  // one memset zeroes every unit's acc / sums / lut_done and the task
+  // counters (chunk c uses counter c)
+  if ((rc = ensure_task_counters(ctx, (size_t)((n + fpc - 1) / fpc) + 1))) return rc;
+  CK(cudaMemsetAsync(ctx->zero_block, 0, ctx->zero_bytes, ctx->stream));
   CK(cudaEventRecord(ctx->ev_start, ctx->stream));
   for (int f0 = 0; f0 < n; f0 += fpc) {
     const int fn = std::min(fpc, n - f0), units = fn * C;
@@ -574,12 +578,8 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
       src = ctx->gx_src;
     }
     CK(sharp::launch_gather(src, Li.fs, Li.pitch, Li.es, C, w, h, W4, H4, P, units, ctx->gx_in, ctx->stream));
-    CK(cudaMemsetAsync(ctx->sums + u0, 0, units * sizeof(unsigned long long), ctx->stream));
-    CK(cudaMemsetAsync(ctx->lut_done + u0, 0, units * sizeof(unsigned int), ctx->stream));
-    CK(cudaMemsetAsync(ctx->acc + u0, 0, units * sizeof(unsigned long long), ctx->stream));
-    CK(cudaMemsetAsync(ctx->tcounters, 0, sizeof(unsigned int), ctx->stream));
     if ((rc = enqueue_device(ctx, ctx->gx_in, units, W4, H4, prm, ctx->gx_out, ctx->stream, ctx->slots[0],
-                             std::min(chunk, (size_t)units), u0, &launches, ctx->tcounters, str)))
+                             std::min(chunk, (size_t)units), u0, &launches, ctx->tcounters + f0 / fpc, str)))
       return rc;
     // the w x h crops into the caller's layout (a host destination goes
     // through a device copy of its byte range, so bytes between the pixels
@@ -596,21 +596,20 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
       CK(cudaMemcpyAsync(dst, ctx->gx_dst, span, cudaMemcpyDeviceToHost, ctx->stream));
     }
     launches += 2;
-    CK(cudaStreamSynchronize(ctx->stream));  // host ranges / scratch are reused by the next chunk
+    // host byte ranges (pageable or pinned) are reused by the next chunk
+    if (kin != kDevice || kout != kDevice) CK(cudaStreamSynchronize(ctx->stream));
   }
   CK(cudaEventRecord(ctx->ev_stop, ctx->stream));
-  CK(cudaEventSynchronize(ctx->ev_stop));
+  CK(cudaMemcpyAsync(&ctx->h_stats->sum, ctx->sums, sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaMemcpyAsync(&ctx->h_stats->mean, ctx->means, sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
   float ms = 0.0f;
   CK(cudaEventElapsedTime(&ms, ctx->ev_start, ctx->ev_stop));
-  unsigned long long s0 = 0;
-  double m0 = 0.0;
-  CK(cudaMemcpy(&s0, ctx->sums, sizeof(s0), cudaMemcpyDeviceToHost));
-  CK(cudaMemcpy(&m0, ctx->means, sizeof(m0), cudaMemcpyDeviceToHost));
   ctx->last_frames = (int)units_all;
   ctx->stats.frames = (int)units_all;
   ctx->stats.kernels = launches;
-  ctx->stats.edge_sum = s0;
-  ctx->stats.edge_mean = m0;
+  ctx->stats.edge_sum = ctx->h_stats->sum;
+  ctx->stats.edge_mean = ctx->h_stats->mean;
   ctx->stats.device_ms = ms;
   ctx->stats.total_ms = ms;
   return SHARP_OK;
