@@ -33,6 +33,7 @@
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -996,14 +997,32 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
 #ifndef SHARP_EXP_LAG_MUL
 #define SHARP_EXP_LAG_MUL 2  // measured: 2x the minimal lags removes most dependency waits
 #endif
+    // The lag rounds past the last frame hold only empty tasks, so short
+    // batches use shorter lags: 2x the in-flight distance when the batch is at
+    // least that long, 1x from 4 frames on (a few empty rounds cost less than
+    // pass-2 producers stalling on their LUTs), else the minimal lags (one to
+    // three images: the empty rounds' latency would dominate).  Measured on
+    // 1080p (tools/small_batch_sweep.py): 8 frames 84 -> 61 us, 24 frames
+    // 227 -> 118 us, 1-2 frames and >= 32 frames unchanged.  A dependency
+    // wait stalls one producer; it cannot deadlock -- every dependency was
+    // grabbed, and issued, earlier.
+    static int policy = -1;  // SHARP_EXP_LAG_POLICY (timing experiments): 0 = 2x or minimal,
+    if (policy < 0) {        // 1 = 1x from L1 frames, 2 = 1x from 4 frames (default), 3 = from 2
+      const char *e = getenv("SHARP_EXP_LAG_POLICY");
+      policy = e ? atoi(e) : 2;
+    }
+    const int L1u = sp.L1, L2u = sp.L2;
     sp.L1 *= SHARP_EXP_LAG_MUL;
     sp.L2 *= SHARP_EXP_LAG_MUL;
-    // The lag rounds past the last frame hold only empty tasks: for a short
-    // batch use the minimal lags (a dependency wait stalls one producer; it
-    // cannot deadlock -- every dependency was grabbed, and issued, earlier).
     if (sg.n < sp.L2) {
-      sp.L1 = 1;
-      sp.L2 = 2;
+      const int tier = policy == 1 ? L1u : policy == 2 ? 4 : policy == 3 ? 2 : 1 << 30;
+      if (sg.n >= tier) {
+        sp.L1 = L1u;
+        sp.L2 = L2u;
+      } else {
+        sp.L1 = 1;
+        sp.L2 = 2;
+      }
     }
     sp.ntasks = (sg.n + sp.L2) * sp.per_round;
   }
