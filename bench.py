@@ -275,10 +275,11 @@ def run_bands_workload(args, world, rank, local):
     torch.cuda.set_stream(stream)
     sh = Sharpener(device=local)
     sh.set_stream(stream)
-    if args.exchange == "p2p":
-        # fused peer-memory exchange: halos and the u64 partials stored
-        # straight into the neighbours' / all ranks' windows (CUDA IPC over
-        # NVLink), epoch-flagged; no NCCL on the data path
+    if args.exchange in ("p2p", "fused"):
+        # peer-memory exchange: halos and the u64 partials stored straight
+        # into the neighbours' / all ranks' windows (CUDA IPC over NVLink),
+        # epoch-flagged; no NCCL on the data path.  "fused": the partials'
+        # all-reduce runs inside the band's single step-kernel launch.
         from paper_conf_icpp_fanjzac15_b200.bands import P2PBand
         p2p = P2PBand(sh, W, H)
         epoch = [0]
@@ -286,7 +287,10 @@ def run_bands_workload(args, world, rank, local):
         def step(src, dst):
             p2p.own.copy_(src)  # this image's rows into the window (the NCCL path copies them too)
             epoch[0] += 1
-            p2p.step(epoch[0], dst, PARAMS)
+            if args.exchange == "fused":
+                p2p.step_fused(epoch[0], dst, PARAMS)
+            else:
+                p2p.step(epoch[0], dst, PARAMS)
     else:
         def step(src, dst):
             band = exchange_halos(src, H, r0, r1)
@@ -310,9 +314,14 @@ def run_bands_workload(args, world, rank, local):
     kt = sh.kernel_times()
     sh.set_profiling(False)
     value = W * H / (ms_step * 1e-3) / 1e6
-    # dominant kernel: the band's pass-2 launch (reads its rows + halo, writes its rows)
-    k_avg = kt.pass2_ms / max(1, kt.pass2_launches)
-    px = kt.pixels / max(1, kt.pass2_launches)
+    # dominant kernel: the band's pass-2 launch (reads its rows + halo, writes
+    # its rows), or the fused band launch (pass 1 + all-reduce + pass 2)
+    if args.exchange == "fused":
+        k_avg = kt.step_ms / max(1, kt.step_launches)
+        px = kt.pixels / max(1, kt.step_launches)
+    else:
+        k_avg = kt.pass2_ms / max(1, kt.pass2_launches)
+        px = kt.pixels / max(1, kt.pass2_launches)
     pk, pk_src = peaks()
     peak = float(pk["hbm_gbs"])
     achieved = ALG_BYTES_PER_PX * px / (k_avg * 1e-3) / 1e9
@@ -345,17 +354,20 @@ def run_bands_workload(args, world, rank, local):
                        "parallelism": ("row bands: 4-row halo exchange (NCCL send/recv) + u64 all-reduce"
                                        if args.exchange == "nccl" else
                                        "row bands: halo rows + u64 partials stored into peer windows "
-                                       "(CUDA IPC / NVLink, epoch flags), no NCCL on the data path"),
+                                       "(CUDA IPC / NVLink, epoch flags), no NCCL on the data path" +
+                                       ("; pass 1 + all-reduce + pass 2 in one launch per band"
+                                        if args.exchange == "fused" else "")),
                        "l2": f"inputs rotated over {ncopy} copies (>= 256 MB > 126 MB L2)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None, "kernel": "step_kernel (band pass 2)",
+                         "frac": achieved / peak, "traffic": None,
+                         "kernel": "step_kernel (fused band)" if args.exchange == "fused" else "step_kernel (band pass 2)",
                          "peak_source": pk_src, "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px,
                          "kernel_avg_ms": k_avg, "pass1_avg_ms": kt.pass1_ms / max(1, kt.pass1_launches)},
             "e2e": {"value": W * H / (e2e_ms * 1e-3) / 1e6, "unit": UNIT, "h2d_bytes_per_step": W * H,
                     "d2h_bytes_per_step": W * H, "ms_per_step": e2e_ms,
                     "api": "bands.sharpen_band (pinned host rows -> device -> pinned host)"},
             # per band: [halo] + step(pass 1) + finish + [all-reduce] + arm + step(pass 2)
-            "gpu_launches": (6 if args.exchange == "p2p" else 4) * args.steps,
+            "gpu_launches": {"p2p": 6, "fused": 2, "nccl": 4}[args.exchange] * args.steps,
             "clocks": clk.summary(),
             "cpu_baseline": None,
             "parity": parity,
@@ -474,8 +486,9 @@ def main():
     ap.add_argument("--ref-sample", type=int, default=16)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--workload", default="batch", choices=["batch", "bands", "ladder"])
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
-                    help="bands workload: NCCL send/recv + all-reduce, or the fused peer-memory exchange")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p", "fused"],
+                    help="bands workload: NCCL send/recv + all-reduce, the peer-memory exchange kernels, or "
+                         "the peer-memory halo push + ONE fused launch per band (all-reduce inside)")
     args = ap.parse_args()
     world, rank, local = dist_setup()
     if args.workload == "bands" and args.width == 1920 and args.height == 1080:

@@ -256,6 +256,19 @@ int sharp_band_p2p_halo(sharp_ctx *ctx, uint8_t *self_window, int w, int rows_ow
                         int up_rows_own, uint8_t *down_window, uint64_t epoch);
 int sharp_band_p2p_allreduce(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank,
                              const uint64_t *d_partial, uint64_t epoch, uint64_t *d_total);
+/* sharp_band_p2p_sharpen: pass 1, the cross-band all-reduce of the pEdge
+ * partials and pass 2 of this band in ONE persistent launch -- the step
+ * kernel's LUT tasks publish the band's partial into slot `rank` of every
+ * window (the same epoch-parity slots as sharp_band_p2p_allreduce) and poll
+ * this window's n_ranks slots for `epoch`, so the collective runs inside the
+ * compute kernel over NVLink.  Call after sharp_band_p2p_halo of the same
+ * epoch (the band's input is its window's rows); writes rows [row0, row1)
+ * to `out` (device, 8-byte aligned, (row1-row0) x w).  grid_cap > 0 limits
+ * the persistent grid (CTAs): bands that share ONE GPU must co-reside, so
+ * their caps must sum to at most 3 x SMs (one band per GPU: 0 = all SMs).
+ * Asynchronous on the context's stream. */
+int sharp_band_p2p_sharpen(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
+                           int row1, uint64_t epoch, const sharp_params *params, uint8_t *out, int grid_cap);
 int sharp_ipc_get_handle(const void *d_ptr, void *handle);
 int sharp_ipc_open_handle(const void *handle, void **d_ptr);
 int sharp_ipc_close_handle(void *d_ptr);

@@ -181,6 +181,19 @@ class P2PBand:
         self.sh.band_sharpen(self.band, self.w, self.h, self.row0, self.row1, self.total, out, params)
         return out
 
+    def step_fused(self, epoch, out, params=None, grid_cap=0):
+        """Halo push, then pass 1 + the peer-memory all-reduce + pass 2 in ONE
+        step-kernel launch (sharp_band_p2p_sharpen).  grid_cap: CTAs of the
+        persistent grid (bands sharing one GPU must co-reside)."""
+        B, g = self.B, self.rank
+        up = self.windows[g - 1] if g > 0 else None
+        dn = self.windows[g + 1] if g < self.world - 1 else None
+        up_rows = self.rows[g - 1][1] - self.rows[g - 1][0] if g > 0 else 0
+        B.sharp_band_p2p_halo(self.sh.ctx, self.window, self.w, self.rows_own, up, up_rows, dn, epoch)
+        B.sharp_band_p2p_sharpen(self.sh.ctx, self.windows, g, self.w, self.h, self.row0, self.row1, epoch, params,
+                                 out, grid_cap)
+        return out
+
     def close(self):
         for p in self._opened:
             self.B.sharp_ipc_close_handle(p)

@@ -95,6 +95,8 @@ _SIGS = {
     "sharp_set_path": ([_P, _I], _I),
     "sharp_get_path": ([_P], _I),
     "sharp_get_stage_times": ([_P, ctypes.POINTER(ctypes.c_float), _I], _I),
+    "sharp_band_p2p_sharpen": ([_P, ctypes.POINTER(_P), _I, _I, _I, _I, _I, _I, ctypes.c_uint64,
+                                ctypes.POINTER(SharpParams), _P, _I], _I),
     "sharp_run_ex": ([_P, _P, ctypes.POINTER(SharpLayout), _I, _I, _I, _I, ctypes.POINTER(SharpParams), _I, _P,
                       ctypes.POINTER(SharpLayout)], _I),
 }
@@ -317,6 +319,12 @@ def sharp_band_p2p_allreduce(ctx, windows, rank, d_partial, epoch, d_total):
     arr = (_P * len(windows))(*windows)
     return _check(lib().sharp_band_p2p_allreduce(ctx, arr, len(windows), rank, _addr(d_partial), int(epoch),
                                                  _addr(d_total)), ctx)
+
+
+def sharp_band_p2p_sharpen(ctx, windows, rank, w, h, row0, row1, epoch, params, out, grid_cap=0):
+    arr = (_P * len(windows))(*windows)
+    return _check(lib().sharp_band_p2p_sharpen(ctx, arr, len(windows), rank, w, h, row0, row1, int(epoch),
+                                               _pp(params), _addr(out), int(grid_cap)), ctx)
 
 
 def sharp_ipc_get_handle(d_ptr):

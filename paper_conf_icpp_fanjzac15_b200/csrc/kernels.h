@@ -8,6 +8,7 @@ namespace sharp {
 // Lookup tables built once per frame by the last CTA of pass 1: entry p
 // (p = pEdge value, 0..1530 = 6*255) holds {adj(p), osc(p)} (R9, R11).
 constexpr int kLutSize = 1536;
+constexpr int kMaxRanks = 32;  // row bands of one image (peer-memory exchange slots)
 
 struct Params {
   float amount, gamma, osc_gain, osc_scale;
@@ -68,6 +69,13 @@ struct BatchLaunch {
   const unsigned long long *total = nullptr;  // pass 2 in: the all-reduced S
   // strided frames (sharp_run_ex): bytes between rows / frames; 0 -> dense
   size_t in_pitch = 0, in_fs = 0, out_pitch = 0, out_fs = 0;
+  // kStepBandFused: slot[rank] of every rank's window (peer mappings), this
+  // rank's own slots, the epoch, the number of ranks; grid_cap > 0 limits the
+  // persistent grid (several bands sharing one GPU must co-reside)
+  unsigned long long *peer_slots[kMaxRanks] = {};
+  const unsigned long long *my_slots = nullptr;
+  unsigned long long epoch = 0;
+  int ranks = 0, rank = 0, grid_cap = 0;
 };
 // Dense [n][H][W] frames: W % 16 == 0 (the TMA row stride), 16-byte aligned
 // input, 8-byte aligned output, H >= 8, W * H <= 2^29.
@@ -85,7 +93,10 @@ cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p
 // pEdge into *a.partial (a.acc, a.task_counter zero on entry); kStepPass2
 // builds the LUT from *a.total and writes the band (3 launches: arm, step,
 // nothing else).  n = 1 frame; a.out is offset internally.
-enum StepMode { kStepAll = 0, kStepPass1 = 1, kStepPass2 = 2 };
+// kStepBandFused: pass 1, the cross-band all-reduce of S through peer
+// memory (the partial slots of the bands_p2p.cu windows) and pass 2 of one
+// band in ONE launch (a.peer_slots / a.my_slots / a.epoch / a.ranks).
+enum StepMode { kStepAll = 0, kStepPass1 = 1, kStepPass2 = 2, kStepBandFused = 3 };
 cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int row_lo, int row_hi, int y0, int rows_in,
                             const Params &p, cudaStream_t stream);
 

@@ -255,6 +255,11 @@ struct StepParams {
   uint8_t *out;
   size_t out_pitch, out_fs;  // output bytes between rows / frames
   unsigned int *task_counter;  // zero on entry
+  // kStepBandFused (kernels.h)
+  unsigned long long *peer_slots[kMaxRanks];
+  const unsigned long long *my_slots;
+  unsigned long long epoch;
+  int ranks;
 };
 // acc packing: S <= 1530 * W * H < 2^40 for W * H <= 2^29 (tma_supported),
 // and the arrival count (4 per task) stays far below 2^24.
@@ -265,6 +270,11 @@ __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type,
   // tasks (S preset by band_prep_kernel) followed by the pass-2 tasks.
   if (sp.mode == kStepPass1) return make_int4(kP1, 0, t, 0);
   if (sp.mode == kStepPass2) return t < kLutTasks ? make_int4(kLut, 0, t, 0) : make_int4(kP2, 0, t - kLutTasks, 0);
+  if (sp.mode == kStepBandFused) {  // [pass 1][LUT][pass 2] of one band
+    const int pf1 = sp.g.per_frame1;
+    if (t < pf1) return make_int4(kP1, 0, t, 0);
+    return t < pf1 + kLutTasks ? make_int4(kLut, 0, t - pf1, 0) : make_int4(kP2, 0, t - pf1 - kLutTasks, 0);
+  }
   const int rho = t / sp.per_round, k = t - rho * sp.per_round;
   const int pf1 = sp.g.per_frame1;
   if (k < pf1) return rho < sp.n ? make_int4(kP1, rho, k, 0) : make_int4(kEmpty, 0, 0, 0);
@@ -294,6 +304,21 @@ __device__ __forceinline__ unsigned int ld_relaxed_u32(const unsigned int *p) {
   return v;
 }
 __device__ __forceinline__ void fence_acquire() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// Peer-memory all-reduce inside the launch (kStepBandFused): system-scope
+// release stores into the other bands' windows, acquire polls of our own.
+__device__ __forceinline__ void st_release_sys_u64(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long gtime_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
 
 // ------------------------------------------------------------- row window
 // Lane words of smem row s: lanes 0..29 own columns C0w+8l..+7 (region A);
@@ -698,6 +723,26 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         // every pass-1 warp of the frame has added its partial (the global
         // barrier of L174's reduction)
         while (((S = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(kPollNs);
+        if (sp.mode == kStepBandFused) {
+          // L174 across the bands: LUT task 0 publishes this band's partial
+          // (epoch << 40 | S_g) into slot[rank] of every band's window; every
+          // LUT task then sums the G slots of its own window once they all
+          // carry the epoch (a dead peer traps after 10 s, not a hang).
+          const unsigned long long mine = S & ((1ull << kAccShift) - 1), ep = sp.epoch & 0xffffffull;
+          if (d.z == 0)
+            for (int q = 0; q < sp.ranks; ++q) st_release_sys_u64(sp.peer_slots[q], (ep << 40) | mine);
+          unsigned long long tot = 0;
+          const unsigned long long t0 = gtime_ns();
+          for (int q = 0; q < sp.ranks; ++q) {
+            unsigned long long v;
+            while (((v = ld_acquire_sys_u64(sp.my_slots + q)) >> 40) != ep) {
+              __nanosleep(kPollNs);
+              if (gtime_ns() - t0 > 10000000000ull) __trap();
+            }
+            tot += v & ((1ull << kAccShift) - 1);
+          }
+          S = tot;
+        }
       }
       // (A pass-2 task's dependency -- its frame's LUT -- is resolved after
       // its first stage's tile loads are issued: the loads do not need it.)
@@ -979,13 +1024,17 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
         resident < 1)
       resident = 1;
   }
-  const int grid = std::min(SHARP_GRID_CTAS, resident) * num_sms();
+  int grid = std::min(SHARP_GRID_CTAS, resident) * num_sms();
+  if (a.grid_cap > 0) grid = std::min(grid, a.grid_cap);
   if (mode == kStepPass1) {
     sp.L1 = sp.L2 = 0;
     sp.ntasks = sp.g.per_frame1;
   } else if (mode == kStepPass2) {
     sp.L1 = sp.L2 = 0;
     sp.ntasks = kLutTasks + sp.g.per_frame;
+  } else if (mode == kStepBandFused) {
+    sp.L1 = sp.L2 = 0;
+    sp.ntasks = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
   } else {
     // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
     // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
@@ -1032,6 +1081,10 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.means = a.means;
   sp.luts = a.luts;
   sp.lut_done = a.lut_done;
+  for (int q = 0; q < kMaxRanks; ++q) sp.peer_slots[q] = a.peer_slots[q];
+  sp.my_slots = a.my_slots;
+  sp.epoch = a.epoch;
+  sp.ranks = a.ranks;
   sp.out = a.out;
   sp.out_pitch = a.out_pitch ? a.out_pitch : (size_t)W;
   sp.out_fs = a.out_fs ? a.out_fs : sp.out_pitch * (size_t)H;
@@ -1051,7 +1104,7 @@ cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p
 
 cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int row_lo, int row_hi, int y0, int rows_in,
                             const Params &p, cudaStream_t stream) {
-  if (mode != kStepPass1 && mode != kStepPass2) return cudaErrorInvalidValue;
+  if (mode != kStepPass1 && mode != kStepPass2 && mode != kStepBandFused) return cudaErrorInvalidValue;
   return launch_step(a, StepGeometry{1, rows_in, row_lo, row_hi, y0}, mode, W, H, p, stream);
 }
 

@@ -1009,6 +1009,57 @@ int sharp_band_p2p_halo(sharp_ctx *ctx, uint8_t *self_window, int w, int rows_ow
   return SHARP_OK;
 }
 
+int sharp_band_p2p_sharpen(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
+                           int row1, uint64_t epoch, const sharp_params *params, uint8_t *out, int grid_cap) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  int in0 = 0, in1 = 0;
+  if (!windows || !out || n_ranks < 1 || n_ranks > sharp::kMaxRanks || rank < 0 || rank >= n_ranks || epoch == 0 ||
+      grid_cap < 0)
+    return set_err(ctx, SHARP_EINVAL, "%s", "bad fused band request (1 <= n_ranks <= 32, epoch > 0)");
+  for (int g = 0; g < n_ranks; ++g)
+    if (!windows[g] || ((uintptr_t)windows[g] & 15)) return set_err(ctx, SHARP_EINVAL, "%s", "bad window pointer");
+  if (w < 16 || (w & 15) || band_halo(h, row0, row1, &in0, &in1) || row1 - row0 < 4)
+    return set_err(ctx, SHARP_EINVAL, "%s", "bad band geometry (w % 16 == 0, rows multiples of 4, >= 4 rows)");
+  if ((long long)w * h >= (1ll << 29)) return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "image larger than 2^29 pixels");
+  if (params && !params_ok(*params)) return set_err(ctx, SHARP_EINVAL, "%s", "parameter out of range or not finite");
+  const uint8_t *band = windows[rank] + SHARP_P2P_CTL_BYTES + (size_t)(in0 - (row0 - 4)) * w;
+  if (!sharp::tma_supported(band, out, w, h))
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "fused bands need the TMA path (8-byte aligned out)");
+  sharp_params p;
+  if (params) p = *params;
+  else sharp_default_params(&p);
+  const sharp::Params prm{p.amount, p.gamma, p.osc_gain, p.osc_scale};
+  CK(cudaSetDevice(ctx->device));
+  int rc;
+  if ((rc = ensure_frames(ctx, 1))) return rc;
+  CK(cudaMemsetAsync(ctx->zero_block, 0, ctx->zero_bytes, ctx->stream));
+  sharp::BatchLaunch a;
+  a.in = band;
+  a.n = 1;
+  a.out = out;
+  a.acc = ctx->acc;
+  a.sums = ctx->sums;
+  a.means = ctx->means;
+  a.luts = ctx->luts;
+  a.lut_done = ctx->lut_done;
+  a.task_counter = ctx->tcounters;
+  const int set = (int)(epoch & 1) * 32;  // the partial slots' epoch-parity set (bands_p2p.cu)
+  for (int g = 0; g < n_ranks; ++g) a.peer_slots[g] = reinterpret_cast<unsigned long long *>(windows[g]) + set + rank;
+  a.my_slots = reinterpret_cast<const unsigned long long *>(windows[rank]) + set;
+  a.epoch = epoch;
+  a.ranks = n_ranks;
+  a.grid_cap = grid_cap;
+  const double px = (double)(row1 - row0) * w;
+  CK(timed(ctx, ctx->stream, 3, px, [&] {
+    return sharp::launch_band_tma(a, sharp::kStepBandFused, w, h, row0, row1, in0, in1 - in0, prm, ctx->stream);
+  }));
+  ctx->last_frames = 1;
+  ctx->stats.frames = 1;
+  ctx->stats.kernels = 1;
+  return SHARP_OK;
+}
+
 int sharp_band_p2p_allreduce(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank,
                              const uint64_t *d_partial, uint64_t epoch, uint64_t *d_total) {
   if (!ctx) return SHARP_EINVAL;
