@@ -275,7 +275,7 @@ def run_bands_workload(args, world, rank, local):
     torch.cuda.set_stream(stream)
     sh = Sharpener(device=local)
     sh.set_stream(stream)
-    if args.exchange in ("p2p", "fused"):
+    if args.exchange in ("p2p", "fused", "one"):
         # peer-memory exchange: halos and the u64 partials stored straight
         # into the neighbours' / all ranks' windows (CUDA IPC over NVLink),
         # epoch-flagged; no NCCL on the data path.  "fused": the partials'
@@ -287,7 +287,9 @@ def run_bands_workload(args, world, rank, local):
         def step(src, dst):
             p2p.own.copy_(src)  # this image's rows into the window (the NCCL path copies them too)
             epoch[0] += 1
-            if args.exchange == "fused":
+            if args.exchange == "one":
+                p2p.step_one_launch(epoch[0], dst, PARAMS)
+            elif args.exchange == "fused":
                 p2p.step_fused(epoch[0], dst, PARAMS)
             else:
                 p2p.step(epoch[0], dst, PARAMS)
@@ -316,7 +318,7 @@ def run_bands_workload(args, world, rank, local):
     value = W * H / (ms_step * 1e-3) / 1e6
     # dominant kernel: the band's pass-2 launch (reads its rows + halo, writes
     # its rows), or the fused band launch (pass 1 + all-reduce + pass 2)
-    if args.exchange == "fused":
+    if args.exchange in ("fused", "one"):
         k_avg = kt.step_ms / max(1, kt.step_launches)
         px = kt.pixels / max(1, kt.step_launches)
     else:
@@ -355,19 +357,21 @@ def run_bands_workload(args, world, rank, local):
                                        if args.exchange == "nccl" else
                                        "row bands: halo rows + u64 partials stored into peer windows "
                                        "(CUDA IPC / NVLink, epoch flags), no NCCL on the data path" +
-                                       ("; pass 1 + all-reduce + pass 2 in one launch per band"
-                                        if args.exchange == "fused" else "")),
+                                       {"fused": "; pass 1 + all-reduce + pass 2 in one launch per band",
+                                        "one": "; halo push + pass 1 + all-reduce + pass 2 in ONE launch per band"}
+                                       .get(args.exchange, "")),
                        "l2": f"inputs rotated over {ncopy} copies (>= 256 MB > 126 MB L2)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": None,
-                         "kernel": "step_kernel (fused band)" if args.exchange == "fused" else "step_kernel (band pass 2)",
+                         "kernel": ("step_kernel (fused band)" if args.exchange in ("fused", "one")
+                                    else "step_kernel (band pass 2)"),
                          "peak_source": pk_src, "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px,
                          "kernel_avg_ms": k_avg, "pass1_avg_ms": kt.pass1_ms / max(1, kt.pass1_launches)},
             "e2e": {"value": W * H / (e2e_ms * 1e-3) / 1e6, "unit": UNIT, "h2d_bytes_per_step": W * H,
                     "d2h_bytes_per_step": W * H, "ms_per_step": e2e_ms,
                     "api": "bands.sharpen_band (pinned host rows -> device -> pinned host)"},
             # per band: [halo] + step(pass 1) + finish + [all-reduce] + arm + step(pass 2)
-            "gpu_launches": {"p2p": 6, "fused": 2, "nccl": 4}[args.exchange] * args.steps,
+            "gpu_launches": {"p2p": 6, "fused": 2, "one": 1, "nccl": 4}[args.exchange] * args.steps,
             "clocks": clk.summary(),
             "cpu_baseline": None,
             "parity": parity,
@@ -486,9 +490,10 @@ def main():
     ap.add_argument("--ref-sample", type=int, default=16)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--workload", default="batch", choices=["batch", "bands", "ladder"])
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p", "fused"],
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p", "fused", "one"],
                     help="bands workload: NCCL send/recv + all-reduce, the peer-memory exchange kernels, or "
-                         "the peer-memory halo push + ONE fused launch per band (all-reduce inside)")
+                         "the peer-memory halo push + ONE fused launch per band (all-reduce inside), or "
+                         "one launch per band with the halo push inside too")
     args = ap.parse_args()
     world, rank, local = dist_setup()
     if args.workload == "bands" and args.width == 1920 and args.height == 1080:

@@ -269,6 +269,17 @@ int sharp_band_p2p_allreduce(sharp_ctx *ctx, uint8_t *const *windows, int n_rank
  * Asynchronous on the context's stream. */
 int sharp_band_p2p_sharpen(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
                            int row1, uint64_t epoch, const sharp_params *params, uint8_t *out, int grid_cap);
+/* sharp_band_p2p_step: the same launch with the halo push folded in -- the
+ * kernel's first task sets this band's "ready" flags in the neighbours'
+ * windows, waits for theirs, and its warps store the band's first / last 4
+ * rows into the neighbours' halos with a system-wide fence and "data" flags;
+ * the pass-1 tiles at the band's edges wait for the neighbours' data flags.
+ * ONE launch per band per image (no sharp_band_p2p_halo call).  up_rows_own:
+ * the upper band's own row count (for its lower halo).  All bands of an image
+ * must run it concurrently (on one GPU: grid caps summing to at most 3 x SMs). */
+int sharp_band_p2p_step(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
+                        int row1, int up_rows_own, uint64_t epoch, const sharp_params *params, uint8_t *out,
+                        int grid_cap);
 int sharp_ipc_get_handle(const void *d_ptr, void *handle);
 int sharp_ipc_open_handle(const void *handle, void **d_ptr);
 int sharp_ipc_close_handle(void *d_ptr);

@@ -194,6 +194,15 @@ class P2PBand:
                                  out, grid_cap)
         return out
 
+    def step_one_launch(self, epoch, out, params=None, grid_cap=0):
+        """Halo push + pass 1 + the peer-memory all-reduce + pass 2 in ONE
+        step-kernel launch (sharp_band_p2p_step)."""
+        g = self.rank
+        up_rows = self.rows[g - 1][1] - self.rows[g - 1][0] if g > 0 else 0
+        self.B.sharp_band_p2p_step(self.sh.ctx, self.windows, g, self.w, self.h, self.row0, self.row1, up_rows, epoch,
+                                   params, out, grid_cap)
+        return out
+
     def close(self):
         for p in self._opened:
             self.B.sharp_ipc_close_handle(p)

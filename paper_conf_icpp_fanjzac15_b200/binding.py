@@ -97,6 +97,8 @@ _SIGS = {
     "sharp_get_stage_times": ([_P, ctypes.POINTER(ctypes.c_float), _I], _I),
     "sharp_band_p2p_sharpen": ([_P, ctypes.POINTER(_P), _I, _I, _I, _I, _I, _I, ctypes.c_uint64,
                                 ctypes.POINTER(SharpParams), _P, _I], _I),
+    "sharp_band_p2p_step": ([_P, ctypes.POINTER(_P), _I, _I, _I, _I, _I, _I, _I, ctypes.c_uint64,
+                             ctypes.POINTER(SharpParams), _P, _I], _I),
     "sharp_run_ex": ([_P, _P, ctypes.POINTER(SharpLayout), _I, _I, _I, _I, ctypes.POINTER(SharpParams), _I, _P,
                       ctypes.POINTER(SharpLayout)], _I),
 }
@@ -325,6 +327,12 @@ def sharp_band_p2p_sharpen(ctx, windows, rank, w, h, row0, row1, epoch, params, 
     arr = (_P * len(windows))(*windows)
     return _check(lib().sharp_band_p2p_sharpen(ctx, arr, len(windows), rank, w, h, row0, row1, int(epoch),
                                                _pp(params), _addr(out), int(grid_cap)), ctx)
+
+
+def sharp_band_p2p_step(ctx, windows, rank, w, h, row0, row1, up_rows_own, epoch, params, out, grid_cap=0):
+    arr = (_P * len(windows))(*windows)
+    return _check(lib().sharp_band_p2p_step(ctx, arr, len(windows), rank, w, h, row0, row1, up_rows_own, int(epoch),
+                                            _pp(params), _addr(out), int(grid_cap)), ctx)
 
 
 def sharp_ipc_get_handle(d_ptr):

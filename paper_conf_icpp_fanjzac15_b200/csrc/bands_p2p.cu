@@ -39,6 +39,9 @@ constexpr int kReadyUp = 2 * kSlots + 2;   // the band above accepts my first ro
 constexpr int kReadyDown = 2 * kSlots + 3; // the band below accepts my last rows
 constexpr unsigned long long kSumMask = (1ull << 40) - 1;
 static_assert((2 * kSlots + 4) * 8 <= kP2PCtlBytes, "control block");
+static_assert(kDataUp == kCtlDataUp && kDataDown == kCtlDataDown && kReadyUp == kCtlReadyUp &&
+                  kReadyDown == kCtlReadyDown && kSlots == kMaxRanks,
+              "the fused band launch (kernels_tma.cu) uses the same window layout");
 
 __device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
   asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");

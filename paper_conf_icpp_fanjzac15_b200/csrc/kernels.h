@@ -76,7 +76,16 @@ struct BatchLaunch {
   const unsigned long long *my_slots = nullptr;
   unsigned long long epoch = 0;
   int ranks = 0, rank = 0, grid_cap = 0;
+  // ... and the halo push in the same launch (halo_on): my window's control
+  // words, the neighbours' (NULL at the image edges), where my first / last 4
+  // rows go in their windows, and where they are in mine
+  int halo_on = 0, halo_bytes = 0;
+  unsigned long long *self_ctl = nullptr, *up_ctl = nullptr, *down_ctl = nullptr;
+  uint8_t *up_halo = nullptr, *down_halo = nullptr;
+  const uint8_t *own_top = nullptr, *own_bot = nullptr;
 };
+// Control words of a peer-memory window (bands_p2p.cu), u64 indices.
+constexpr int kCtlDataUp = 64, kCtlDataDown = 65, kCtlReadyUp = 66, kCtlReadyDown = 67;
 // Dense [n][H][W] frames: W % 16 == 0 (the TMA row stride), 16-byte aligned
 // input, 8-byte aligned output, H >= 8, W * H <= 2^29.
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);

@@ -238,7 +238,7 @@ struct Geo {
 // (slots for frames outside [0, n) are empty tasks).  The lags L1 < L2 are
 // chosen so that a frame's dependencies were grabbed long before (they are
 // normally complete when the producer checks them).
-enum TaskType { kEmpty = 0, kP1 = 1, kLut = 2, kP2 = 3, kEnd = -1 };
+enum TaskType { kEmpty = 0, kP1 = 1, kLut = 2, kP2 = 3, kHalo = 4, kEnd = -1 };
 struct StepParams {
   Geo g;
   int mode;       // kStepAll, or a row band's kStepPass1 / kStepPass2
@@ -260,6 +260,10 @@ struct StepParams {
   const unsigned long long *my_slots;
   unsigned long long epoch;
   int ranks;
+  int halo_on, halo_bytes;
+  unsigned long long *self_ctl, *up_ctl, *down_ctl;
+  uint8_t *up_halo, *down_halo;
+  const uint8_t *own_top, *own_bot;
 };
 // acc packing: S <= 1530 * W * H < 2^40 for W * H <= 2^29 (tma_supported),
 // and the arrival count (4 per task) stays far below 2^24.
@@ -270,7 +274,11 @@ __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type,
   // tasks (S preset by band_prep_kernel) followed by the pass-2 tasks.
   if (sp.mode == kStepPass1) return make_int4(kP1, 0, t, 0);
   if (sp.mode == kStepPass2) return t < kLutTasks ? make_int4(kLut, 0, t, 0) : make_int4(kP2, 0, t - kLutTasks, 0);
-  if (sp.mode == kStepBandFused) {  // [pass 1][LUT][pass 2] of one band
+  if (sp.mode == kStepBandFused) {  // [halo push][pass 1][LUT][pass 2] of one band
+    if (sp.halo_on) {
+      if (t == 0) return make_int4(kHalo, 0, 0, 0);
+      --t;
+    }
     const int pf1 = sp.g.per_frame1;
     if (t < pf1) return make_int4(kP1, 0, t, 0);
     return t < pf1 + kLutTasks ? make_int4(kLut, 0, t - pf1, 0) : make_int4(kP2, 0, t - pf1 - kLutTasks, 0);
@@ -744,6 +752,21 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           S = tot;
         }
       }
+      auto wait_sys = [&](const unsigned long long *p, unsigned long long want) {
+        const unsigned long long t0 = gtime_ns();
+        while (ld_acquire_sys_u64(p) != want) {
+          __nanosleep(kPollNs);
+          if (gtime_ns() - t0 > 10000000000ull) __trap();  // a dead peer: trap, not hang
+        }
+      };
+      if (d.x == kHalo) {
+        // (1) my previous launch is complete: the neighbours may fill my
+        // halos of this epoch; (2) wait until they accept my edge rows
+        if (sp.up_ctl) st_release_sys_u64(sp.up_ctl + kCtlReadyDown, sp.epoch);
+        if (sp.down_ctl) st_release_sys_u64(sp.down_ctl + kCtlReadyUp, sp.epoch);
+        if (sp.up_ctl) wait_sys(sp.self_ctl + kCtlReadyUp, sp.epoch);
+        if (sp.down_ctl) wait_sys(sp.self_ctl + kCtlReadyDown, sp.epoch);
+      }
       // (A pass-2 task's dependency -- its frame's LUT -- is resolved after
       // its first stage's tile loads are issued: the loads do not need it.)
       int C0 = 0, R0 = 0, nsub = 1, nw = 0;
@@ -764,11 +787,35 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         stage_t[b] = clock64();
 #endif
         if (d.x == kP1) {
+          if (sp.halo_on) {  // tiles at the band's edges read the neighbours' rows
+            bool waited = false;
+            if (sp.up_ctl && R0 == g.row_lo) {
+              wait_sys(sp.self_ctl + kCtlDataUp, sp.epoch);
+              waited = true;
+            }
+            if (sp.down_ctl && R0 + g.th1 >= g.row_hi) {
+              wait_sys(sp.self_ctl + kCtlDataDown, sp.epoch);
+              waited = true;
+            }
+            if (waited) fence_proxy_async_global();  // peer-written rows before the TMA reads them
+          }
           stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
           mbar_expect_tx(full, tile_bytes(nw, kRows1));
           tma_tiles(st, &map1A, &map1B, C0, nw, R0 - 1 - g.y0, d.y, full, pol_keep);
         } else if (d.x == kP2) {
           const int R0k = R0 + k * kTH;
+          if (sp.halo_on) {  // (tile loads go out before the LUT wait: check the halo flags here too)
+            bool waited = false;
+            if (sp.up_ctl && R0k - 4 < g.row_lo) {
+              wait_sys(sp.self_ctl + kCtlDataUp, sp.epoch);
+              waited = true;
+            }
+            if (sp.down_ctl && R0k + kTH + 4 > g.row_hi) {
+              wait_sys(sp.self_ctl + kCtlDataDown, sp.epoch);
+              waited = true;
+            }
+            if (waited) fence_proxy_async_global();
+          }
           stage_task[b] = make_int4(d.x, d.y, C0, R0k);
           stage_aux[b] = make_int2(nsub, j & 1);
           const uint32_t lut_bytes = k == 0 ? (uint32_t)kLutBytes : 0u;
@@ -848,7 +895,21 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     }
     if (d.x == kLut && lane == 0) TL_MIN(3);
     if (d.x == kP1 && lane == 0) TL_MIN(1);
-    if (d.x == kLut) {
+    if (d.x == kHalo) {
+      // push my first / last 4 rows into the neighbours' halos (16-byte peer
+      // stores), make them visible system-wide, then flag them
+      const int n16 = sp.halo_bytes / 16, tid = threadIdx.x;
+      for (int i = tid; i < n16; i += kWarpsT * 32) {
+        if (sp.up_halo) reinterpret_cast<uint4 *>(sp.up_halo)[i] = reinterpret_cast<const uint4 *>(sp.own_top)[i];
+        if (sp.down_halo) reinterpret_cast<uint4 *>(sp.down_halo)[i] = reinterpret_cast<const uint4 *>(sp.own_bot)[i];
+      }
+      __threadfence_system();
+      asm volatile("bar.sync 1, %0;" ::"n"(kWarpsT * 32) : "memory");  // the 4 consumer warps
+      if (tid == 0) {
+        if (sp.up_ctl) st_release_sys_u64(sp.up_ctl + kCtlDataDown, sp.epoch);
+        if (sp.down_ctl) st_release_sys_u64(sp.down_ctl + kCtlDataUp, sp.epoch);
+      }
+    } else if (d.x == kLut) {
       // LUT task: entries k = q*128 .. q*128+127 (pEdge p = 2k) of frame f
       // (R9, R11; f64, one rounding).  (Measured: splitting adj / osc over two
       // threads per entry does not shorten the build and costs 0.9% of the batch.)
@@ -1034,7 +1095,7 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     sp.ntasks = kLutTasks + sp.g.per_frame;
   } else if (mode == kStepBandFused) {
     sp.L1 = sp.L2 = 0;
-    sp.ntasks = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
+    sp.ntasks = (a.halo_on ? 1 : 0) + sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
   } else {
     // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
     // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
@@ -1085,6 +1146,15 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.my_slots = a.my_slots;
   sp.epoch = a.epoch;
   sp.ranks = a.ranks;
+  sp.halo_on = a.halo_on;
+  sp.halo_bytes = a.halo_bytes;
+  sp.self_ctl = a.self_ctl;
+  sp.up_ctl = a.up_ctl;
+  sp.down_ctl = a.down_ctl;
+  sp.up_halo = a.up_halo;
+  sp.down_halo = a.down_halo;
+  sp.own_top = a.own_top;
+  sp.own_bot = a.own_bot;
   sp.out = a.out;
   sp.out_pitch = a.out_pitch ? a.out_pitch : (size_t)W;
   sp.out_fs = a.out_fs ? a.out_fs : sp.out_pitch * (size_t)H;

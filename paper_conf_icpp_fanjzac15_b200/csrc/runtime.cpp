@@ -1009,8 +1009,27 @@ int sharp_band_p2p_halo(sharp_ctx *ctx, uint8_t *self_window, int w, int rows_ow
   return SHARP_OK;
 }
 
+static int band_fused_impl(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
+                           int row1, int up_rows_own, bool halo, uint64_t epoch, const sharp_params *params,
+                           uint8_t *out, int grid_cap);
+
 int sharp_band_p2p_sharpen(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
                            int row1, uint64_t epoch, const sharp_params *params, uint8_t *out, int grid_cap) {
+  return band_fused_impl(ctx, windows, n_ranks, rank, w, h, row0, row1, 0, false, epoch, params, out, grid_cap);
+}
+
+int sharp_band_p2p_step(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
+                        int row1, int up_rows_own, uint64_t epoch, const sharp_params *params, uint8_t *out,
+                        int grid_cap) {
+  if (rank > 0 && up_rows_own < 4)
+    return ctx ? set_err(ctx, SHARP_EINVAL, "%s", "up_rows_own < 4") : SHARP_EINVAL;
+  return band_fused_impl(ctx, windows, n_ranks, rank, w, h, row0, row1, up_rows_own, true, epoch, params, out,
+                         grid_cap);
+}
+
+static int band_fused_impl(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
+                           int row1, int up_rows_own, bool halo, uint64_t epoch, const sharp_params *params,
+                           uint8_t *out, int grid_cap) {
   if (!ctx) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
   int in0 = 0, in1 = 0;
@@ -1050,6 +1069,25 @@ int sharp_band_p2p_sharpen(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks,
   a.epoch = epoch;
   a.ranks = n_ranks;
   a.grid_cap = grid_cap;
+  if (halo) {  // the halo push of bands_p2p.cu inside the same launch
+    auto ctl = [](uint8_t *win) { return reinterpret_cast<unsigned long long *>(win); };
+    auto rows_of = [](uint8_t *win) { return win + SHARP_P2P_CTL_BYTES; };
+    const int rows_own = row1 - row0;
+    uint8_t *self = windows[rank];
+    a.halo_on = 1;
+    a.halo_bytes = 4 * w;
+    a.self_ctl = ctl(self);
+    a.own_top = rows_of(self) + (size_t)4 * w;
+    a.own_bot = rows_of(self) + (size_t)rows_own * w;  // rows 4 + rows_own - 4 .. 4 + rows_own - 1
+    if (rank > 0) {
+      a.up_ctl = ctl(windows[rank - 1]);
+      a.up_halo = rows_of(windows[rank - 1]) + (size_t)(4 + up_rows_own) * w;  // its lower halo
+    }
+    if (rank < n_ranks - 1) {
+      a.down_ctl = ctl(windows[rank + 1]);
+      a.down_halo = rows_of(windows[rank + 1]);  // its upper halo
+    }
+  }
   const double px = (double)(row1 - row0) * w;
   CK(timed(ctx, ctx->stream, 3, px, [&] {
     return sharp::launch_band_tma(a, sharp::kStepBandFused, w, h, row0, row1, in0, in1 - in0, prm, ctx->stream);

@@ -24,6 +24,7 @@ class Bands:
         self.w, self.h, self.G = w, h, G
         sms = torch.cuda.get_device_properties(0).multi_processor_count
         self.cap = max(1, (2 * sms) // G)  # leave room for the single-CTA halo kernels
+        self.cap1 = max(1, (3 * sms) // G)  # one launch per band: all bands' grids co-reside
         self.streams = [torch.cuda.Stream() for _ in range(G)]
         self.sh = [Sharpener() for _ in range(G)]
         for s, st in zip(self.sh, self.streams):
@@ -37,7 +38,7 @@ class Bands:
             b.sh.band_edge_sum(b.band, w, h, b.row0, b.row1, tmp)
         torch.cuda.synchronize()
 
-    def run(self, img, epoch, fused=True, prm=DEFAULT):
+    def run(self, img, epoch, fused=True, prm=DEFAULT, one_launch=False):
         outs = []
         d = torch.from_numpy(img).cuda()
         torch.cuda.synchronize()
@@ -45,14 +46,16 @@ class Bands:
             with torch.cuda.stream(st):
                 b.own.copy_(d[b.row0:b.row1])
                 o = torch.full((b.rows_own, self.w), 7, dtype=torch.uint8, device="cuda")
-                if fused:
+                if one_launch:
+                    b.step_one_launch(epoch, o, prm, grid_cap=self.cap1)
+                elif fused:
                     b.step_fused(epoch, o, prm, grid_cap=self.cap)
                 else:
                     b.step(epoch, o, prm)
                 outs.append(o)
         torch.cuda.synchronize()
         out = torch.cat(outs).cpu().numpy()
-        sums = [b.sh.batch_sums(1)[0] if fused else int(b.total.item()) for b in self.bands]
+        sums = [b.sh.batch_sums(1)[0] if (fused or one_launch) else int(b.total.item()) for b in self.bands]
         return out, sums
 
     def close(self):
@@ -106,3 +109,23 @@ def test_fused_rejections():
                 assert e.value.code == SHARP_EINVAL
         finally:
             sharp_p2p_window_destroy(win)
+
+
+@pytest.mark.parametrize("W,H,G", [(1920, 1080, 2), (1920, 1080, 3), (3840, 2160, 4), (256, 64, 8), (960, 40, 5)])
+def test_one_launch_per_band_equal_whole_image_over_epochs(W, H, G):
+    """sharp_band_p2p_step: the halo push folded into the fused launch too --
+    one launch per band per image; mixed over epochs with the separate-kernel
+    paths (same window protocol)."""
+    bands = Bands(W, H, G)
+    try:
+        plan = [("natural", 1, "one"), ("noise", 2, "one"), ("natural", 3, "fused"), ("natural", 4, "p2p"),
+                ("noise", 5, "one")]
+        for epoch, (kind, seed, how) in enumerate(plan, start=1):
+            img = synth.image(W, H, kind, seed=synth.BASE_SEED + 100 * G + seed)
+            out, sums = bands.run(img, epoch, fused=(how == "fused"), one_launch=(how == "one"))
+            ref, S, _ = oracle.sharpen(img, *DEFAULT)
+            assert sums == [S] * G, (epoch, how, sums, S)
+            bad = np.argwhere(out != ref)
+            assert bad.size == 0, f"epoch {epoch} {how}: {len(bad)} mismatches, first {bad[:5].tolist()}"
+    finally:
+        bands.close()
