@@ -268,13 +268,14 @@ struct StepParams {
 // acc packing: S <= 1530 * W * H < 2^40 for W * H <= 2^29 (tma_supported),
 // and the arrival count (4 per task) stays far below 2^24.
 constexpr int kAccShift = 40;
+template <bool kFused>
 __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type, frame, sub, 0}
   if (t >= sp.ntasks) return make_int4(kEnd, 0, 0, 0);
   // A row band's two launches (one frame): pass-1 tasks only; or the LUT
   // tasks (S preset by band_prep_kernel) followed by the pass-2 tasks.
   if (sp.mode == kStepPass1) return make_int4(kP1, 0, t, 0);
   if (sp.mode == kStepPass2) return t < kLutTasks ? make_int4(kLut, 0, t, 0) : make_int4(kP2, 0, t - kLutTasks, 0);
-  if (sp.mode == kStepBandFused) {  // [halo push][pass 1][LUT][pass 2] of one band
+  if (kFused) {  // kStepBandFused: [halo push][pass 1][LUT][pass 2] of one band
     if (sp.halo_on) {
       if (t == 0) return make_int4(kHalo, 0, 0, 0);
       --t;
@@ -691,6 +692,10 @@ __device__ unsigned long long g_waitstat[40][2];
 __shared__ long long stage_t[2];  // producer: clock64 at issue
 #endif
 // ============================================================== the kernel
+// kFused: the one-band fused launch (kStepBandFused: in-kernel peer-memory
+// all-reduce and halo push); a separate instantiation, so the batch kernel's
+// code and registers are exactly those without it.
+template <bool kFused>
 __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     step_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
                 const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, StepParams sp) {
@@ -724,14 +729,14 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     // last stage of the pass-2 task that used LUT buffer b.
     int lut_last[2] = {-kStages, -kStages};
     for (int s = 0, j = 0;;) {
-      const int4 d = decode(sp, t_next);
+      const int4 d = decode<kFused>(sp, t_next);
       // Resolve the task's dependency first (before waiting for a stage).
       unsigned long long S = 0;
       if (d.x == kLut) {
         // every pass-1 warp of the frame has added its partial (the global
         // barrier of L174's reduction)
         while (((S = ld_relaxed_u64(&sp.acc[d.y])) & ~((1ull << kAccShift) - 1)) != arrivals) __nanosleep(kPollNs);
-        if (sp.mode == kStepBandFused) {
+        if (kFused) {
           // L174 across the bands: LUT task 0 publishes this band's partial
           // (epoch << 40 | S_g) into slot[rank] of every band's window; every
           // LUT task then sums the G slots of its own window once they all
@@ -759,7 +764,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           if (gtime_ns() - t0 > 10000000000ull) __trap();  // a dead peer: trap, not hang
         }
       };
-      if (d.x == kHalo) {
+      if (kFused && d.x == kHalo) {
         // (1) my previous launch is complete: the neighbours may fill my
         // halos of this epoch; (2) wait until they accept my edge rows
         if (sp.up_ctl) st_release_sys_u64(sp.up_ctl + kCtlReadyDown, sp.epoch);
@@ -787,7 +792,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         stage_t[b] = clock64();
 #endif
         if (d.x == kP1) {
-          if (sp.halo_on) {  // tiles at the band's edges read the neighbours' rows
+          if (kFused && sp.halo_on) {  // tiles at the band's edges read the neighbours' rows
             bool waited = false;
             if (sp.up_ctl && R0 == g.row_lo) {
               wait_sys(sp.self_ctl + kCtlDataUp, sp.epoch);
@@ -804,7 +809,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           tma_tiles(st, &map1A, &map1B, C0, nw, R0 - 1 - g.y0, d.y, full, pol_keep);
         } else if (d.x == kP2) {
           const int R0k = R0 + k * kTH;
-          if (sp.halo_on) {  // (tile loads go out before the LUT wait: check the halo flags here too)
+          if (kFused && sp.halo_on) {  // (tile loads go out before the LUT wait: check the halo flags here too)
             bool waited = false;
             if (sp.up_ctl && R0k - 4 < g.row_lo) {
               wait_sys(sp.self_ctl + kCtlDataUp, sp.epoch);
@@ -895,7 +900,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     }
     if (d.x == kLut && lane == 0) TL_MIN(3);
     if (d.x == kP1 && lane == 0) TL_MIN(1);
-    if (d.x == kHalo) {
+    if (kFused && d.x == kHalo) {
       // push my first / last 4 rows into the neighbours' halos (16-byte peer
       // stores), make them visible system-wide, then flag them
       const int n16 = sp.halo_bytes / 16, tid = threadIdx.x;
@@ -1040,7 +1045,8 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
                         cudaStream_t stream) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
+    cudaFuncSetAttribute(step_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
+    cudaFuncSetAttribute(step_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
     attr = true;
   }
   if (sg.n <= 0 || sg.row_hi <= sg.row_lo) return cudaSuccess;
@@ -1081,7 +1087,7 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
 #endif
   static int resident = 0;  // CTAs per SM that actually fit (registers, smem)
   if (!resident) {
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, step_kernel, kThreadsT, kSmem) != cudaSuccess ||
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, step_kernel<false>, kThreadsT, kSmem) != cudaSuccess ||
         resident < 1)
       resident = 1;
   }
@@ -1163,7 +1169,10 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     band_prep_kernel<<<1, 1, 0, stream>>>(a.acc, a.lut_done, a.task_counter, a.total,
                                           (unsigned long long)(sp.g.per_frame1 * kWarpsT) << kAccShift);
   }
-  step_kernel<<<grid, kThreadsT, kSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
+  if (mode == kStepBandFused)
+    step_kernel<true><<<grid, kThreadsT, kSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
+  else
+    step_kernel<false><<<grid, kThreadsT, kSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
   if (mode == kStepPass1) band_finish_kernel<<<1, 1, 0, stream>>>(a.acc, a.partial);
   return cudaGetLastError();
 }
@@ -1182,7 +1191,8 @@ cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int ro
 cudaError_t preload_step() {
   cudaFuncAttributes a;
   cudaError_t e;
-  if ((e = cudaFuncGetAttributes(&a, step_kernel)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, step_kernel<false>)) != cudaSuccess) return e;
+  if ((e = cudaFuncGetAttributes(&a, step_kernel<true>)) != cudaSuccess) return e;
   if ((e = cudaFuncGetAttributes(&a, band_prep_kernel)) != cudaSuccess) return e;
   if ((e = cudaFuncGetAttributes(&a, band_finish_kernel)) != cudaSuccess) return e;
   return cudaSuccess;
