@@ -532,7 +532,9 @@ def main():
     fb = W * H
     # Inputs: pinned host (for e2e) and a device copy (device-resident value).
     h_in = torch.empty((n, H, W), dtype=torch.uint8).pin_memory()
-    synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 5 + start, out=h_in.numpy())
+    # (torchrun sets OMP_NUM_THREADS=1: give each rank its share of the cores for input generation)
+    gen_threads = max(1, len(os.sched_getaffinity(0)) // max(1, world))
+    synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 5 + start, out=h_in.numpy(), threads=gen_threads)
     h_out = torch.empty_like(h_in).pin_memory()
     d_in = h_in.to(f"cuda:{local}")
     d_out = torch.empty_like(d_in)
