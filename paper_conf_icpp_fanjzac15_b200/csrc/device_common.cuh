@@ -229,6 +229,23 @@ __device__ __forceinline__ float2 lut_entry(int p, double mean, const Params &pr
   return make_float2(lut_adj(p, mean, prm), lut_osc(p, mean, prm));
 }
 
+// The same with truncation (the R14 alternative): cvt.rzi then the saturating pack.
+__device__ __forceinline__ uint32_t pack4_rzi_u8(float a, float b, float c, float d) {
+  uint32_t r;
+  asm("{\n"
+      ".reg .b32 t0, t1, t2, t3, lo;\n"
+      "cvt.rzi.s32.f32 t2, %3;\n"
+      "cvt.rzi.s32.f32 t3, %4;\n"
+      "cvt.pack.sat.u8.s32.b32 lo, t3, t2, 0;\n"
+      "cvt.rzi.s32.f32 t0, %1;\n"
+      "cvt.rzi.s32.f32 t1, %2;\n"
+      "cvt.pack.sat.u8.s32.b32 %0, t1, t0, lo;\n"
+      "}"
+      : "=r"(r)
+      : "f"(a), "f"(b), "f"(c), "f"(d));
+  return r;
+}
+
 // Packs 8 bytes (low byte of each word) into two words.
 __device__ __forceinline__ uint2 pack8(const uint32_t o[8]) {
   const uint32_t a = prmt(prmt(o[0], o[1], 0x0040), prmt(o[2], o[3], 0x0040), 0x5410);

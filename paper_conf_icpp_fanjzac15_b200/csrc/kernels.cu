@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
             if (c < W && (r < 2 || r >= H - 2 || c < 2 || c >= W - 2)) NU[x] = -ring_u(r, c, W, H, j0, Sc, Sn, col_wins);
           }
         }
-        uint32_t o[8];
+        float F8[8];
 #pragma unroll
         for (int x = 0; x < 8; ++x) {
           const int p = pair_of(x);
@@ -297,11 +297,11 @@ __global__ void __launch_bounds__(kThreads) sharpen_kernel(const uint8_t *__rest
           const float P = __fmaf_rn(L.x, E, -NU[x]);                         // preliminary (L178)
           const float mxf = add_f32_f16(mx_h, 0.0f), mnf = add_f32_f16(mn_h, 0.0f);
           const float t = fminf(fmaxf(P, mnf), mxf);                         // Fig. 8 branch target
-          const float F = __fmaf_rn(L.y, __fsub_rn(P, t), t);                // osc max / osc min / P
-          o[x] = trunc ? cvt_u8_rz(F) : cvt_u8(F);                           // clamp [0,255], RNE (R14)
+          F8[x] = __fmaf_rn(L.y, __fsub_rn(P, t), t);                        // osc max / osc min / P
         }
-        const uint32_t o0 = prmt(prmt(o[0], o[1], 0x0040), prmt(o[2], o[3], 0x0040), 0x5410);
-        const uint32_t o1 = prmt(prmt(o[4], o[5], 0x0040), prmt(o[6], o[7], 0x0040), 0x5410);
+        // clamp [0,255] + RNE (R14) or truncation (the R14 alternative), packed 4 per word
+        const uint32_t o0 = trunc ? pack4_rzi_u8(F8[0], F8[1], F8[2], F8[3]) : pack4_rni_u8(F8[0], F8[1], F8[2], F8[3]);
+        const uint32_t o1 = trunc ? pack4_rzi_u8(F8[4], F8[5], F8[6], F8[7]) : pack4_rni_u8(F8[4], F8[5], F8[6], F8[7]);
         uint8_t *orow = out + (size_t)r * W;
         if (c0 < W) *reinterpret_cast<uint32_t *>(orow + c0) = o0;
         if (c0 + 4 < W) *reinterpret_cast<uint32_t *>(orow + c0 + 4) = o1;
