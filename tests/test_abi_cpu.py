@@ -86,3 +86,17 @@ def test_c_program_links_against_the_abi():
     assert os.path.exists(exe)
     out = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
     assert "libsharp.so" in out and "not found" not in out
+
+
+def test_reading_switch_values_agree_across_header_binding_and_oracle():
+    """SHARP_READ_* (include/sharp.h), the binding's constants and the
+    oracle's ORACLE_READ_* are defined independently (no shared code); they
+    must name the same bits."""
+    hdr = open(os.path.join(ROOT, "include", "sharp.h")).read()
+    orc = open(os.path.join(ROOT, "oracle", "oracle.h")).read()
+    import oracle
+    import paper_conf_icpp_fanjzac15_b200 as p
+    for name in ["INT_DOWNSCALE", "COLUMN_WINS", "INTERIOR_MEAN", "STRENGTH_EXP", "OSC_CONST", "TRUNCATE"]:
+        h = int(re.search(rf"SHARP_READ_{name}\s*=\s*(\d+)", hdr).group(1))
+        o = int(re.search(rf"#define ORACLE_READ_{name}\s+(\d+)", orc).group(1))
+        assert h == o == getattr(p, f"SHARP_READ_{name}") == getattr(oracle, f"READ_{name}"), name
