@@ -472,6 +472,31 @@ def run_ladder_workload(args, world, rank, local):
     print(json.dumps(line), flush=True)
 
 
+def free_port():
+    import socket
+    with socket.socket(socket.AF_INET, socket.SOCK_STREAM) as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def self_launch(args):
+    """`--gpus N` (N > 1) outside torchrun: re-run this command as N ranks under
+    torch.distributed.run (one process per GPU, rendezvous on 127.0.0.1), the
+    launch the driver uses; returns the exit code.  Fails loudly when N
+    exceeds the visible GPUs (the reference arm runs on host cores and the
+    SHARP_BENCH_SHARE_GPU test hook maps ranks onto the visible GPUs)."""
+    import subprocess
+    if args.impl != "reference" and not SHARE_GPU:
+        import torch
+        n = torch.cuda.device_count()
+        if args.gpus > n:
+            print(f"bench.py: --gpus {args.gpus} but only {n} GPU(s) are visible", file=sys.stderr)
+            return 2
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.run(cmd, env=dict(os.environ, OMP_NUM_THREADS=os.environ.get("OMP_NUM_THREADS", "1"))).returncode
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -495,7 +520,13 @@ def main():
                          "the peer-memory halo push + ONE fused launch per band (all-reduce inside), or "
                          "one launch per band with the halo push inside too")
     args = ap.parse_args()
+    if args.gpus < 1:
+        ap.error("--gpus must be >= 1")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(self_launch(args))
     world, rank, local = dist_setup()
+    if "WORLD_SIZE" in os.environ and world != args.gpus and rank == 0:
+        print(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}; measuring {world} rank(s)", file=sys.stderr)
     if args.workload == "bands" and args.width == 1920 and args.height == 1080:
         args.width, args.height = 7680, 4320  # configs[3]: 8K
     if args.impl == "reference":

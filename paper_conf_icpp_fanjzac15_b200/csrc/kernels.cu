@@ -86,22 +86,24 @@ __device__ __forceinline__ void load_block(Block &B, const uint8_t *__restrict__
 __device__ __forceinline__ float ring_u(int r, int c, int W, int H, int j0, const float (&Sc)[4], const float (&Sn)[4],
                                         bool col_wins) {
   const int w = W >> 2, h = H >> 2;
-  auto col = [&](int j) { return j - j0 + 1; };  // index into Sc/Sn
+  auto col = [&](int j) { return j - j0 + 1; };  // index into Sc/Sn (0..3)
+  // register selects instead of a dynamically indexed local array (no stack frame)
+  auto at = [](const float(&a)[4], int i) { return i <= 0 ? a[0] : i == 1 ? a[1] : i == 2 ? a[2] : a[3]; };
   if (r >= H - 2 && c >= W - 2) {                 // (vii): third last of last column = D[h-1][w-1]
-    return __fmul_rn(Sc[col(w - 1)], 1.0f / 16.0f);
+    return __fmul_rn(at(Sc, col(w - 1)), 1.0f / 16.0f);
   }
   if ((c <= 1 || c >= W - 2) && r <= H - 3) {     // (vi)/(ii)/(iv): column lines
     const int j = (c <= 1) ? 0 : w - 1;
-    if (c <= 1 && r <= 1 && !col_wins) return __fmul_rn(Sc[col(0)], 1.0f / 16.0f);  // (v) then (vi): D[0][0]
+    if (c <= 1 && r <= 1 && !col_wins) return __fmul_rn(at(Sc, col(0)), 1.0f / 16.0f);  // (v) then (vi): D[0][0]
     const int rr = (r == H - 3) ? H - 4 : r;   // third last <- fourth last
     const int k = rr & 3;                      // rr>>2 == current D row (rr in the block of r)
-    return line_val(Sc[col(j)], Sn[col(j)], k);
+    return line_val(at(Sc, col(j)), at(Sn, col(j)), k);
   }
   // rows 0/1 (line of D row 0) or H-2/H-1 (line of D row h-1); Sc is that D row.
   const int cc = (c == W - 3) ? W - 4 : c;
   const int jj = cc >> 2, k = cc & 3;
-  const float x = Sc[col(jj)];
-  const float y = (k == 0) ? x : Sc[col(jj + 1)];
+  const float x = at(Sc, col(jj));
+  const float y = (k == 0) ? x : at(Sc, col(jj + 1));
   (void)h;
   return line_val(x, y, k);
 }

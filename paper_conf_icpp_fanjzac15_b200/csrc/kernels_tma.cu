@@ -37,6 +37,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <atomic>
 
 #include "device_common.cuh"
 #include "kernels.h"
@@ -122,18 +123,6 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
-// Polling wait that never suspends the warp (test_wait is non-blocking).
-__device__ __forceinline__ void mbar_wait_spin(uint32_t bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "WAIT_%=:\n"
-      "mbarrier.test_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra WAIT_%=;\n"
-      "}\n" ::"r"(bar),
-      "r"(parity)
-      : "memory");
-}
 // One 3-D box {cols, rows, 1} of the [n][H][W] frames at (x, r, f) (x 16-B aligned).
 // L2 eviction-priority policies (createpolicy): pass-1 loads keep the frame
 // in L2 for its pass-2 re-read (evict_last); pass-2 loads and the output
@@ -145,11 +134,7 @@ __device__ __forceinline__ uint64_t policy_evict_last() {
 }
 __device__ __forceinline__ uint64_t policy_evict_first() {
   uint64_t p;
-#ifdef SHARP_EXP_NORMAL_FIRST
-  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
-#else
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-#endif
   return p;
 }
 __device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, int x, int r, int f, uint32_t bar,
@@ -171,15 +156,10 @@ __device__ __forceinline__ void tma_tiles(uint32_t st, const CUtensorMap *mapA, 
   if (nw == kWarpsT) tma_box(st + kRegB, mapB, C0 + kWarpsT * kTW, r, f, bar, policy);
 }
 // Output store.  (Measured: an L2::cache_hint store costs ~5% of the step
-// through extra issue; plain STG.64 it is -- SHARP_EXP_HINT_STORE to compare.)
+// through extra issue; plain STG.64 it is.)
 __device__ __forceinline__ void st_stream_u64(uint8_t *p, uint2 v, uint64_t policy) {
-#ifndef SHARP_EXP_HINT_STORE
   (void)policy;
   *reinterpret_cast<uint2 *>(p) = v;
-#else
-  asm volatile("st.global.L2::cache_hint.v2.b32 [%0], {%1, %2}, %3;" ::"l"(p), "r"(v.x), "r"(v.y), "l"(policy)
-               : "memory");
-#endif
 }
 __device__ __forceinline__ void bulk_copy(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
@@ -531,11 +511,7 @@ struct Ring {
   __device__ __forceinline__ static uint32_t phase(int s) { return ((unsigned)s / kStages) & 1u; }
   __device__ __forceinline__ uint32_t stage(int s) const { return sbase + (uint32_t)(buf(s) * kStage); }
   __device__ __forceinline__ void wait_full(int s) const {
-#ifdef SHARP_EXP_SPIN_WAIT
-    mbar_wait_spin(full0 + 8u * buf(s), phase(s));
-#else
     mbar_wait(full0 + 8u * buf(s), phase(s));
-#endif
   }
   __device__ __forceinline__ void release(int s, int lane) const {  // one arrival per consumer warp
     __syncwarp();
@@ -553,13 +529,6 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
                                         uint8_t *__restrict__ out, uint32_t out_pitch,
                                         int W, int H, int row_lo, int row_hi, int C0w, int R0, int warp,
                                         int lane) {
-#ifdef SHARP_EXP_NO_P2  // timing experiment only
-  for (int k = 0; k < nsub; ++k) {
-    if (k) ring.wait_full(s + k);
-    ring.release(s + k, lane);
-  }
-  return;
-#endif
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
   // W % 8 == 0: image columns 0,1 are in the lane with c0 == 0, columns
@@ -632,9 +601,6 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 // slower.)
 __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rmax1, int th1, int C0w, int R0,
                                         int lane) {
-#ifdef SHARP_EXP_NO_P1  // timing experiment only
-  return 0.0f;
-#endif
   const int c0 = C0w + 8 * lane;
   const LaneRow aw = lane_row(stage, warp, lane);
   // Sobel-body pixels of this lane (not frame columns, not beyond the image).
@@ -674,7 +640,7 @@ __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rm
   return sum;
 }
 
-#ifdef SHARP_EXP_TIMELINE  // timing experiment: globaltimer of the launch's phases (min / max over CTAs)
+#ifdef SHARP_DIAG_TIMELINE  // timing experiment: globaltimer of the launch's phases (min / max over CTAs)
 __device__ unsigned long long g_tl[8];
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -686,10 +652,6 @@ __device__ __forceinline__ unsigned long long gtimer() {
 #else
 #define TL_MIN(i)
 #define TL_MAX(i)
-#endif
-#ifdef SHARP_EXP_WAITSTAT  // timing experiment: consumer full-barrier wait cycles by (previous, awaited) task type
-__device__ unsigned long long g_waitstat[40][2];
-__shared__ long long stage_t[2];  // producer: clock64 at issue
 #endif
 // ============================================================== the kernel
 // kFused: the one-band fused launch (kStepBandFused: in-kernel peer-memory
@@ -788,9 +750,6 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         // task's loads and the next empty-wait.
         if (k == 0 && d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
         const uint32_t full = ring.full0 + 8u * b, st = ring.stage(s);
-#ifdef SHARP_EXP_WAITSTAT
-        stage_t[b] = clock64();
-#endif
         if (d.x == kP1) {
           if (kFused && sp.halo_on) {  // tiles at the band's edges read the neighbours' rows
             bool waited = false;
@@ -852,31 +811,10 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
   }
 
   // -------------------------------------------------------------- consumers
-#ifdef SHARP_EXP_WAITSTAT
-  int prev_type = 0;
-  const long long t_begin = clock64();
-#endif
   for (int s = 0;;) {
     const int b = Ring::buf(s);
-#ifdef SHARP_EXP_WAITSTAT
-    const long long tw0 = clock64();
-#endif
     ring.wait_full(s);
     const int4 d = stage_task[b];
-#ifdef SHARP_EXP_WAITSTAT
-    if (lane == 0) {
-      const int cur = d.x < 0 ? 4 : d.x;
-      atomicAdd(&g_waitstat[prev_type * 5 + cur][0], (unsigned long long)(clock64() - tw0));
-      atomicAdd(&g_waitstat[prev_type * 5 + cur][1], 1ull);
-      prev_type = cur;
-      const long long now = clock64();
-      if (warp == 0 && now - tw0 > 200) {  // waited: the load completed ~now
-        atomicAdd(&g_waitstat[26 + cur][0], (unsigned long long)(now - stage_t[b]));
-        atomicAdd(&g_waitstat[26 + cur][1], 1ull);
-      }
-      if (d.x == kEnd) atomicAdd(&g_waitstat[25][0], (unsigned long long)(clock64() - t_begin));
-    }
-#endif
     if (d.x == kEnd) {
       if (lane == 0) TL_MAX(7);
       break;
@@ -974,20 +912,24 @@ bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, size_t p
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Per-device launch facts, filled by preload_step() (sharp_create calls it
+// after selecting the context's device): SM count and the step kernel's
+// resident CTAs per SM.  Atomics: contexts may be created from several threads.
+constexpr int kMaxDevices = 64;
+std::atomic<int> g_sms[kMaxDevices], g_resident[kMaxDevices];
+int cur_device() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return (dev >= 0 && dev < kMaxDevices) ? dev : 0;
+}
 int num_sms() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
-  }
-  return sms;
+  const int v = g_sms[cur_device()].load(std::memory_order_relaxed);
+  return v > 0 ? v : 148;
 }
 
 }  // namespace
 
-#ifdef SHARP_EXP_TIMELINE
+#ifdef SHARP_DIAG_TIMELINE
 extern "C" int sharp_debug_timeline(unsigned long long *out, int reset) {
   cudaDeviceSynchronize();
   cudaMemcpyFromSymbol(out, g_tl, sizeof(g_tl));
@@ -995,17 +937,6 @@ extern "C" int sharp_debug_timeline(unsigned long long *out, int reset) {
     unsigned long long z[8];
     for (int i = 0; i < 8; ++i) z[i] = (i == 0 || i == 1 || i == 3 || i == 5) ? ~0ull : 0ull;
     cudaMemcpyToSymbol(g_tl, z, sizeof(z));
-  }
-  return 0;
-}
-#endif
-#ifdef SHARP_EXP_WAITSTAT
-extern "C" int sharp_debug_waitstat(unsigned long long *out, int reset) {
-  cudaDeviceSynchronize();
-  cudaMemcpyFromSymbol(out, g_waitstat, sizeof(g_waitstat));
-  if (reset) {
-    static unsigned long long z[40][2] = {};
-    cudaMemcpyToSymbol(g_waitstat, z, sizeof(z));
   }
   return 0;
 }
@@ -1043,12 +974,6 @@ struct StepGeometry {
 
 cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, int W, int H, const Params &p,
                         cudaStream_t stream) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(step_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
-    cudaFuncSetAttribute(step_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
-    attr = true;
-  }
   if (sg.n <= 0 || sg.row_hi <= sg.row_lo) return cudaSuccess;
   CUtensorMap m1A, m1B, m2A, m2B;  // the same frames: pass-1 / pass-2 box heights, regions A / B
   const int R = sg.rows_in;
@@ -1085,12 +1010,7 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
 #ifndef SHARP_GRID_CTAS
 #define SHARP_GRID_CTAS kCtasPerSm
 #endif
-  static int resident = 0;  // CTAs per SM that actually fit (registers, smem)
-  if (!resident) {
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, step_kernel<false>, kThreadsT, kSmem) != cudaSuccess ||
-        resident < 1)
-      resident = 1;
-  }
+  const int resident = std::max(1, g_resident[cur_device()].load(std::memory_order_relaxed));
   int grid = std::min(SHARP_GRID_CTAS, resident) * num_sms();
   if (a.grid_cap > 0) grid = std::min(grid, a.grid_cap);
   if (mode == kStepPass1) {
@@ -1110,9 +1030,6 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     const int in_flight = 3 * grid;
     sp.L1 = (in_flight + sp.per_round - 1) / sp.per_round + 1;
     sp.L2 = sp.L1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
-#ifndef SHARP_EXP_LAG_MUL
-#define SHARP_EXP_LAG_MUL 2  // measured: 2x the minimal lags removes most dependency waits
-#endif
     // The lag rounds past the last frame hold only empty tasks, so short
     // batches use shorter lags: 2x the in-flight distance when the batch is at
     // least that long, 1x from 4 frames on (a few empty rounds cost less than
@@ -1122,17 +1039,11 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     // 227 -> 118 us, 1-2 frames and >= 32 frames unchanged.  A dependency
     // wait stalls one producer; it cannot deadlock -- every dependency was
     // grabbed, and issued, earlier.
-    static int policy = -1;  // SHARP_EXP_LAG_POLICY (timing experiments): 0 = 2x or minimal,
-    if (policy < 0) {        // 1 = 1x from L1 frames, 2 = 1x from 4 frames (default), 3 = from 2
-      const char *e = getenv("SHARP_EXP_LAG_POLICY");
-      policy = e ? atoi(e) : 2;
-    }
     const int L1u = sp.L1, L2u = sp.L2;
-    sp.L1 *= SHARP_EXP_LAG_MUL;
-    sp.L2 *= SHARP_EXP_LAG_MUL;
+    sp.L1 *= 2;  // measured: 2x the minimal lags removes most dependency waits
+    sp.L2 *= 2;
     if (sg.n < sp.L2) {
-      const int tier = policy == 1 ? L1u : policy == 2 ? 4 : policy == 3 ? 2 : 1 << 30;
-      if (sg.n >= tier) {
+      if (sg.n >= 4) {
         sp.L1 = L1u;
         sp.L2 = L2u;
       } else {
@@ -1191,6 +1102,19 @@ cudaError_t launch_band_tma(const BatchLaunch &a, int mode, int W, int H, int ro
 cudaError_t preload_step() {
   cudaFuncAttributes a;
   cudaError_t e;
+  // the dynamic smem opt-in is a per-device function attribute: set it for
+  // the current (the context's) device
+  if ((e = cudaFuncSetAttribute(step_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem)) != cudaSuccess)
+    return e;
+  if ((e = cudaFuncSetAttribute(step_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem)) != cudaSuccess)
+    return e;
+  const int dev = cur_device();
+  int sms = 0, res = 0;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&res, step_kernel<false>, kThreadsT, kSmem)) != cudaSuccess)
+    return e;
+  g_sms[dev].store(sms > 0 ? sms : 148);
+  g_resident[dev].store(res > 0 ? res : 1);
   if ((e = cudaFuncGetAttributes(&a, step_kernel<false>)) != cudaSuccess) return e;
   if ((e = cudaFuncGetAttributes(&a, step_kernel<true>)) != cudaSuccess) return e;
   if ((e = cudaFuncGetAttributes(&a, band_prep_kernel)) != cudaSuccess) return e;

@@ -57,6 +57,10 @@ struct Slot {
   uint8_t *h_in = nullptr, *h_out = nullptr;   // pinned staging (chunk)
   unsigned int *counters = nullptr;            // per chunk frame
   float2 *luts = nullptr;                      // per chunk frame
+  // SHARP_PATH_STAGED scratch (D, U, pEdge, strength of one frame): one per
+  // slot, since the host pipeline runs the slots' chunks concurrently
+  void *staged = nullptr;
+  size_t staged_cap = 0;
 };
 
 }  // namespace
@@ -70,8 +74,6 @@ struct sharp_ctx {
   int nslots = 3;
   int chunk_cfg = 0;
   int path = SHARP_PATH_AUTO;  // SHARP_FORCE_GENERIC=1 at sharp_create selects SHARP_PATH_TWO_PASS
-  void *staged = nullptr;      // SHARP_PATH_STAGED scratch (D, U, pEdge, strength of one frame)
-  size_t staged_cap = 0;
   cudaEvent_t stage_open[sharp::kNumStages] = {};
   Slot slots[kMaxSlots];
   size_t slot_chunk_frames = 0, slot_stage_bytes = 0;  // capacity of the slot buffers
@@ -201,6 +203,9 @@ void free_slot(Slot &s) {
   cudaFreeHost(s.h_out);
   cudaFree(s.counters);
   cudaFree(s.luts);
+  cudaFree(s.staged);
+  s.staged = nullptr;
+  s.staged_cap = 0;
   s.d_in = s.d_out = s.h_in = s.h_out = nullptr;
   s.counters = nullptr;
   s.luts = nullptr;
@@ -284,19 +289,20 @@ cudaError_t timed(sharp_ctx *ctx, cudaStream_t st, int kind, double px, F launch
   return e;
 }
 
-// Staged-path scratch for one w x h frame (grown on demand).
-int rc_staged(sharp_ctx *ctx, int w, int h) {
+// Staged-path scratch of a slot for one w x h frame (grown on demand).
+int rc_staged(sharp_ctx *ctx, Slot &slot, cudaStream_t st, int w, int h) {
   const size_t need = sharp::staged_scratch_bytes(w, h);
-  if (need <= ctx->staged_cap) return SHARP_OK;
+  if (need <= slot.staged_cap) return SHARP_OK;
+  cudaStreamSynchronize(st);
   cudaStreamSynchronize(ctx->stream);
-  cudaFree(ctx->staged);
-  ctx->staged = nullptr;
-  ctx->staged_cap = 0;
-  if (cudaMalloc(&ctx->staged, need) != cudaSuccess) {
+  cudaFree(slot.staged);
+  slot.staged = nullptr;
+  slot.staged_cap = 0;
+  if (cudaMalloc(&slot.staged, need) != cudaSuccess) {
     cudaGetLastError();
     return SHARP_ENOMEM;
   }
-  ctx->staged_cap = need;
+  slot.staged_cap = need;
   return SHARP_OK;
 }
 
@@ -334,14 +340,14 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   if (!str.dense() && ctx->path == SHARP_PATH_STAGED) return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "strided frames on the staged path");
   const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
   if (ctx->path == SHARP_PATH_STAGED) {  // the paper's base design: K1..K7 per frame
-    if ((rc_staged(ctx, w, h))) return SHARP_ENOMEM;
+    if ((rc_staged(ctx, slot, st, w, h))) return SHARP_ENOMEM;
     sharp::StageTimer tm;
     if (ctx->profiling) {
       tm.ctx = ctx;
       tm.rec = stage_rec;
     }
     for (int f = 0; f < n; ++f) {
-      CK(sharp::launch_staged(din + (size_t)f * fb, w, h, prm, ctx->staged, ctx->sums + frame_base + f,
+      CK(sharp::launch_staged(din + (size_t)f * fb, w, h, prm, slot.staged, ctx->sums + frame_base + f,
                               ctx->means + frame_base + f, dout + (size_t)f * fb, st, tm));
       *launches += sharp::kStagedLaunches;
     }
@@ -858,7 +864,6 @@ void sharp_destroy(sharp_ctx *ctx) {
   cudaFree(ctx->zero_block);
   cudaFree(ctx->means);
   cudaFree(ctx->luts);
-  cudaFree(ctx->staged);
   cudaFree(ctx->gx_in);
   cudaFree(ctx->gx_out);
   cudaFree(ctx->gx_src);
@@ -879,7 +884,18 @@ void sharp_destroy(sharp_ctx *ctx) {
 int sharp_set_stream(sharp_ctx *ctx, void *stream) {
   if (!ctx) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
-  ctx->stream = stream ? (cudaStream_t)stream : ctx->own_stream;
+  cudaStream_t next = stream ? (cudaStream_t)stream : ctx->own_stream;
+  if (next != ctx->stream) {
+    // work already queued on the old stream (a persistent launch, the scratch
+    // it uses) completes before anything issued on the new one
+    CK(cudaSetDevice(ctx->device));
+    cudaEvent_t e = pool_event(ctx);
+    if (!e) return set_err(ctx, SHARP_ECUDA, "%s", "cudaEventCreate failed");
+    CK(cudaEventRecord(e, ctx->stream));
+    CK(cudaStreamWaitEvent(next, e, 0));
+    ctx->ev_pool.push_back(e);
+  }
+  ctx->stream = next;
   return SHARP_OK;
 }
 

@@ -54,3 +54,25 @@ def test_numa_binding_is_best_effort_without_a_gpu():
                 raise AttributeError("no GPU")
 
     assert b.bind_to_gpu_numa_node(NoGpu, 0) is None
+
+
+def test_gpus_n_self_launches_n_ranks():
+    """`bench.py --gpus 2` without torchrun re-launches itself as 2 ranks
+    (torch.distributed.run on 127.0.0.1); rank 0 prints ONE line with
+    n_gpus == 2 (the reference arm, which runs on host cores, exercises the
+    launch without a GPU)."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
+                        "--steps", "1", "--warmup", "0", "--ref-sample", "2", "--width", "256", "--height", "128",
+                        "--frames", "8"], capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [json.loads(x) for x in r.stdout.strip().splitlines() if x.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    assert lines[0]["n_gpus"] == 2 and lines[0]["impl"] == "reference"
+
+
+def test_gpus_n_beyond_visible_fails_loudly():
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="")
+    env.pop("WORLD_SIZE", None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--steps", "1"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert r.returncode != 0 and "visible" in r.stderr

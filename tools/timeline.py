@@ -1,5 +1,5 @@
 """Phase timeline of single-image step launches (needs a library built with
--DSHARP_EXP_TIMELINE, copied over libsharp.so).  Prints, per size, the median
+-DSHARP_DIAG_TIMELINE, copied over libsharp.so).  Prints, per size, the median
 over repetitions of each phase's globaltimer offset (us) from the first CTA's
 start, plus the host-side event time of the call."""
 import ctypes
