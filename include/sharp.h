@@ -302,12 +302,18 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
 
 /* ---- Kernel paths: the optimisation ladder of PAPER.md sec. V (Fig. 12,
  * Fig. 14), every rung bit-identical to the oracle.
- *   SHARP_PATH_AUTO     the step kernel where it applies, else the two-pass path (default)
+ *   SHARP_PATH_AUTO     the resident kernel where it applies, else the step kernel, else the
+ *                       two-pass path (default)
  *   SHARP_PATH_STEP     one persistent TMA-staged launch per batch (kernels_tma.cu): pass 1,
  *                       per-frame LUT and pass 2 as dynamically scheduled tasks with
  *                       in-kernel dependencies; needs w % 16 == 0 (sharp_run_ex: any w % 8 == 0,
  *                       w >= 16, through strided tensor maps), 16-byte aligned input,
  *                       8-byte aligned output, w*h <= 2^29, else SHARP_EUNSUPPORTED
+ *   SHARP_PATH_RES      one persistent TMA-staged launch per batch whose pass 1 leaves each
+ *                       tile's pEdge in tensor memory for pass 2 of the same tile (kernels_res.cu:
+ *                       no second Sobel, no pEdge traffic); the step kernel's geometry rules plus
+ *                       at most 2 x (resident grid) tiles of 960 x 12 per frame (up to ~10 Mpx,
+ *                       4K included), else SHARP_EUNSUPPORTED
  *   SHARP_PATH_TWO_PASS two fused kernels per chunk of frames (kernels.cu): Sobel +
  *                       reduction + LUT, then everything else; any w % 4 == 0
  *   SHARP_PATH_STAGED   the paper's BASE GPU design (sec. IV): one kernel per
@@ -315,7 +321,7 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
  *                       7 launches per frame); the per-stage breakdown of Fig. 13
  * Takes effect at the next call.  Row-band calls need AUTO or STEP.  Environment
  * SHARP_FORCE_GENERIC=1 at sharp_create selects SHARP_PATH_TWO_PASS. */
-enum { SHARP_PATH_AUTO = 0, SHARP_PATH_STEP = 1, SHARP_PATH_TWO_PASS = 2, SHARP_PATH_STAGED = 3 };
+enum { SHARP_PATH_AUTO = 0, SHARP_PATH_STEP = 1, SHARP_PATH_TWO_PASS = 2, SHARP_PATH_STAGED = 3, SHARP_PATH_RES = 4 };
 int sharp_set_path(sharp_ctx *ctx, int path);
 int sharp_get_path(const sharp_ctx *ctx);
 

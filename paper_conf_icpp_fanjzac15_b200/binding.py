@@ -23,6 +23,7 @@ SHARP_PATH_AUTO = 0
 SHARP_PATH_STEP = 1
 SHARP_PATH_TWO_PASS = 2
 SHARP_PATH_STAGED = 3
+SHARP_PATH_RES = 4
 STAGE_NAMES = ("downscale", "border", "center", "sobel", "reduction", "strength", "sharpness")
 SHARP_NUM_STAGES = len(STAGE_NAMES)
 

@@ -63,6 +63,7 @@ struct BatchLaunch {
   double *means = nullptr;             // n; out: S / (W H)
   float2 *luts = nullptr;              // n * kLutSize (scratch)
   unsigned int *lut_done = nullptr;    // n; zero on entry
+  unsigned int *lut_next = nullptr;    // n; zero on entry (res kernel: table chunks grabbed)
   unsigned int *task_counter = nullptr;  // 1; zero on entry
   // row-band launches only (launch_band_tma):
   unsigned long long *partial = nullptr;      // pass 1 out: the band's S
@@ -95,6 +96,21 @@ bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H);
 bool tma_supported_strided(const uint8_t *imgs, size_t in_pitch, size_t in_fs, const uint8_t *outs, size_t out_pitch,
                            size_t out_fs, int W, int H);
 cudaError_t launch_batch_tma(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
+
+// TMEM-resident kernel (kernels_res.cu): pass 1 leaves each tile's pEdge in
+// tensor memory, pass 2 of the same tile (same CTA) reads it back -- no
+// second Sobel; the producers build a frame's tables while they wait for
+// them.  Same frames / strides / scratch as launch_batch_tma plus lut_next.
+// res_supported: frames of at most 2 x (resident grid) tiles of 960 x 12
+// (~10 Mpx: up to 4K); else the step kernel.  Returns cudaErrorNotSupported
+// when not applicable.
+bool res_supported(int W, int H, int n);
+cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream);
+cudaError_t preload_res();
+// cuTensorMapEncodeTiled of [n][H][W] u8 frames at the given byte strides.
+#include <cuda.h>
+bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, size_t pitch, size_t fs, int box_cols,
+              int box_rows);
 
 // One row band [row_lo, row_hi) of a W x H image (sec. 8(e)): a.in holds
 // image rows [y0, y0 + rows_in) (the band plus its halo rows), a.out the

@@ -41,45 +41,21 @@
 
 #include "device_common.cuh"
 #include "kernels.h"
+#include "tma_common.cuh"
 
 namespace sharp {
 namespace {
 using namespace dev;
 
-constexpr int kTW = 240;     // output columns per warp tile (lanes 0..29 x 8 px)
-constexpr int kTH = 12;      // output rows per warp tile
 constexpr int kCtasPerSm = 3;  // smem ~67 KB per CTA
 #ifndef SHARP_LB_CTAS
 #define SHARP_LB_CTAS kCtasPerSm
 #endif
-constexpr int kWarpsT = 4;   // compute warps = warp tiles per CTA tile
-constexpr int kCtaCols = kTW * kWarpsT;
-constexpr int kThreadsT = 32 * (kWarpsT + 1);  // + producer warp
 constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task (one per thread)
-// pEdge = |Gx| + |Gy| is always even (Gx and Gy both have the parity of the
-// sum of the four window corners), so the step kernel's tables hold the even
-// entries only: entry k = pEdge / 2, k < kLut2 (766 used).
-constexpr int kLut2 = 768;
 constexpr int kLutTasks = kLut2 / kLutPerTask;
-constexpr unsigned kPollNs = 100;  // dependency polling interval of the producer
-// A warp tile needs columns C0w-8 .. C0w+247.  TMA box starts must be
-// 16-byte aligned in the innermost dimension and a box dimension is at most
-// 256, so a warp tile is fetched as one 256-column box of the [n][H][W]
-// frames, region A = columns C0w-16 .. C0w+239 (smem pitch 256).  Its right
-// halo C0w+240.. is the first own column of the next warp's region A (offset
-// kCol0 there); only the CTA tile's last warp needs one more box, region B =
-// 16 columns C0w+240 .. C0w+255 (smem pitch 16) after the four slots.  (When
-// the next warp has no columns, the halo lies beyond the image and only feeds
-// pixels that are either not stored or on the overridden frame column W-1.)
-constexpr int kPitch = 256;           // region A pitch
-constexpr int kPitchB = 16;           // region B pitch
-constexpr int kCol0 = 16;             // region-A column of C0w
-constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+kTH+3
 constexpr int kTH1 = 18;              // pass-1 output rows per warp tile (fits the same slot)
 constexpr int kRows1 = kTH1 + 2;      // pass-1 box rows: R0-1 .. R0+kTH1
-constexpr int kSlot = kPitch * kRows2;  // per-warp smem slot: region A (128-B aligned)
 static_assert(kRows1 <= kRows2 && kSlot % 128 == 0, "pass-1 tiles fit the slots");
-constexpr int kLutBytes = kLut2 * 8;
 // A pass-2 task is kSub vertically adjacent CTA tiles ("sub-tiles") of one
 // frame: each sub-tile fills one stage, the frame's LUT is copied once per
 // task into one of two LUT buffers (task parity), and the warps carry their
@@ -92,7 +68,6 @@ constexpr int kSub = SHARP_P2_SUB;
 #define SHARP_STAGES 2  // measured: 3 stages +0.3%, 2 stages (this layout) +0.6% vs the old layout
 #endif
 constexpr int kStages = SHARP_STAGES;          // smem ring depth
-constexpr int kRegB = kWarpsT * kSlot;         // region B of the last warp
 constexpr int kStage = (kRegB + kPitchB * kRows2 + 127) / 128 * 128;  // one stage
 constexpr int kLutOff = kStages * kStage;      // two LUT buffers after the stages
 constexpr int kBarOff = kLutOff + 2 * kLutBytes;
@@ -101,102 +76,6 @@ static_assert(kSlot % 128 == 0 && kStage % 128 == 0, "TMA smem destinations must
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
 static_assert(kTH1 % 3 == 0, "pass-1 tiles (3-row loop)");
 static_assert(kLut2 % kLutPerTask == 0 && kLut2 <= kLutSize && 2 * (kLut2 - 1) >= 1530, "LUT tasks");
-
-// ------------------------------------------------------------ TMA / mbarrier
-__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 1000000;\n"  // suspend (not spin) up to 1 ms
-      "@!p bra WAIT_%=;\n"
-      "}\n" ::"r"(bar),
-      "r"(parity)
-      : "memory");
-}
-// One 3-D box {cols, rows, 1} of the [n][H][W] frames at (x, r, f) (x 16-B aligned).
-// L2 eviction-priority policies (createpolicy): pass-1 loads keep the frame
-// in L2 for its pass-2 re-read (evict_last); pass-2 loads and the output
-// stores are the last touch (evict_first).
-__device__ __forceinline__ uint64_t policy_evict_last() {
-  uint64_t p;
-  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-__device__ __forceinline__ uint64_t policy_evict_first() {
-  uint64_t p;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-__device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, int x, int r, int f, uint32_t bar,
-                                        uint64_t policy) {
-  asm volatile(
-      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, "
-      "{%2, %3, %4}], [%5], %6;" ::"r"(dst),
-      "l"(map), "r"(x), "r"(r), "r"(f), "r"(bar), "l"(policy)
-      : "memory");
-}
-// The boxes of a CTA tile of nw warp tiles into stage st: region A per warp,
-// and region B (the last warp's right halo) when all kWarpsT warps have columns.
-__device__ __forceinline__ uint32_t tile_bytes(int nw, int rows) {
-  return (uint32_t)((nw * kPitch + (nw == kWarpsT ? kPitchB : 0)) * rows);
-}
-__device__ __forceinline__ void tma_tiles(uint32_t st, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0, int nw,
-                                          int r, int f, uint32_t bar, uint64_t policy) {
-  for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, mapA, C0 + w * kTW - kCol0, r, f, bar, policy);
-  if (nw == kWarpsT) tma_box(st + kRegB, mapB, C0 + kWarpsT * kTW, r, f, bar, policy);
-}
-// Output store.  (Measured: an L2::cache_hint store costs ~5% of the step
-// through extra issue; plain STG.64 it is.)
-__device__ __forceinline__ void st_stream_u64(uint8_t *p, uint2 v, uint64_t policy) {
-  (void)policy;
-  *reinterpret_cast<uint2 *>(p) = v;
-}
-__device__ __forceinline__ void bulk_copy(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
-}
-__device__ __forceinline__ void fence_barrier_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
-__device__ __forceinline__ unsigned int ld_acquire(const unsigned int *p) {
-  unsigned int v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-// ----------------------------------------------------------- packed f32x2
-__device__ __forceinline__ unsigned long long f2pack(float a, float b) {
-  unsigned long long r;
-  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
-  return r;
-}
-__device__ __forceinline__ float2 f2unpack(unsigned long long r) {
-  float2 v;
-  asm("mov.b64 {%0, %1}, %2;" : "=f"(v.x), "=f"(v.y) : "l"(r));
-  return v;
-}
-// (a*x + b*y) for a lane pair with the same (x, y): FMUL2 then FFMA2, each
-// single-rounding per lane -- bit-identical to the scalar fmul/fma pair.
-__device__ __forceinline__ float2 lin2(float x, float y, unsigned long long a, unsigned long long b) {
-  unsigned long long t, r;
-  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(t) : "l"(f2pack(x, x)), "l"(a));
-  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(f2pack(y, y)), "l"(b), "l"(t));
-  return f2unpack(r);
-}
-__device__ __forceinline__ float2 sub2(float2 a, float2 b) {
-  unsigned long long r;
-  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(f2pack(a.x, a.y)), "l"(f2pack(b.x, b.y)));
-  return f2unpack(r);
-}
 
 // ------------------------------------------------------------------ tasks
 struct Geo {
@@ -280,158 +159,12 @@ __device__ __forceinline__ void tile_xy(const Geo &g, int sub, int th, int &C0, 
   C0 = (sub - ty * g.tiles_x) * kCtaCols;
   R0 = g.row_lo + ty * th;
 }
-// Polling loads: relaxed (no L1 invalidation per poll); the caller issues
-// one acquire fence after the awaited value was seen.
-__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *p) {
-  unsigned long long v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ unsigned int ld_relaxed_u32(const unsigned int *p) {
-  unsigned int v;
-  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void fence_acquire() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
-// Peer-memory all-reduce inside the launch (kStepBandFused): system-scope
-// release stores into the other bands' windows, acquire polls of our own.
-__device__ __forceinline__ void st_release_sys_u64(unsigned long long *p, unsigned long long v) {
-  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned long long *p) {
-  unsigned long long v;
-  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ unsigned long long gtime_ns() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-  return t;
-}
-
-// ------------------------------------------------------------- row window
-// Lane words of smem row s: lanes 0..29 own columns C0w+8l..+7 (region A);
-// lane 31 the left halo C0w-8..C0w-1 (region A); lane 30 the right halo
-// C0w+240..247 (the next warp's region A, or region B for the last warp).
-struct LaneRow {
-  uint32_t base, pitch;
-};
-__device__ __forceinline__ LaneRow lane_row(uint32_t stage, int warp, int lane) {
-  if (lane == 30) {
-    if (warp == kWarpsT - 1) return LaneRow{stage + (uint32_t)kRegB, (uint32_t)kPitchB};
-    return LaneRow{stage + (uint32_t)((warp + 1) * kSlot + kCol0), (uint32_t)kPitch};
-  }
-  return LaneRow{stage + (uint32_t)(warp * kSlot + kCol0 + 8 * (lane < 31 ? lane : -1)), (uint32_t)kPitch};
-}
-__device__ __forceinline__ uint2 row_words(const LaneRow &a, int s) { return lds_u64(a.base + (uint32_t)s * a.pitch); }
-
-// Converts a row of words into the window data.  Neighbour pairs come from
-// the adjacent lanes (shuffle), so each lane loads only its own 8 bytes.
-template <bool kMinMax>
-__device__ __forceinline__ RowD derive_w(uint2 w, int lane) {
-  const uint32_t E0 = hadd(prmt(w.x, kF16Bias, 0x4240), kMinus1024);  // (c0, c0+2)
-  const uint32_t O0 = hadd(prmt(w.x, kF16Bias, 0x4341), kMinus1024);  // (c0+1, c0+3)
-  const uint32_t E1 = hadd(prmt(w.y, kF16Bias, 0x4240), kMinus1024);  // (c0+4, c0+6)
-  const uint32_t O1 = hadd(prmt(w.y, kF16Bias, 0x4341), kMinus1024);  // (c0+5, c0+7)
-  const uint32_t PO = __shfl_sync(0xffffffffu, O1, (lane + 31) & 31);  // (c0-3, c0-1)
-  const uint32_t NE = __shfl_sync(0xffffffffu, E0, (lane + 1) & 31);   // (c0+8, c0+10)
-  const uint32_t p[4] = {E0, O0, E1, O1};
-  const uint32_t l[4] = {prmt(PO, O0, 0x5432), E0, prmt(O0, O1, 0x5432), E1};
-  const uint32_t r[4] = {O0, prmt(E0, E1, 0x5432), O1, prmt(E1, NE, 0x5432)};
-  RowD d;
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    d.c[i] = p[i];
-    d.h[i] = hsub(r[i], l[i]);
-    d.s[i] = hadd(hfma(kTwo, p[i], l[i]), r[i]);
-    if (kMinMax) {
-      d.mx[i] = __vimax3_u16x2(l[i], p[i], r[i]);
-      d.mn[i] = __vimin3_u16x2(l[i], p[i], r[i]);
-    }
-  }
-  return d;
-}
-
-// D sums (16*D) of the block at smem rows s..s+3 for D columns j0-1..j0+2.
-__device__ __forceinline__ float4 dblock(const LaneRow &a, int s, int lane) {
-  const uint32_t o = a.base + (uint32_t)s * a.pitch;
-  const uint2 r0 = lds_u64(o), r1 = lds_u64(o + a.pitch), r2 = lds_u64(o + 2 * a.pitch), r3 = lds_u64(o + 3 * a.pitch);
-  const float d0 = (float)blk4(r0.x, r1.x, r2.x, r3.x);
-  const float d1 = (float)blk4(r0.y, r1.y, r2.y, r3.y);
-  const float dm1 = __shfl_sync(0xffffffffu, d1, (lane + 31) & 31);
-  const float d2 = __shfl_sync(0xffffffffu, d0, (lane + 1) & 31);
-  return make_float4(dm1, d0, d1, d2);
-}
-
 // ========================================================== pass 2, one row
 // Output row of this lane (window rows a = r-1, b = r, c = r+1).
 // V = vertical interpolation (x 128) of the four D columns (body, L146);
 // D0 / D1 = 16*D of D rows r>>2 and (r>>2)+1 for the lane's D columns
 // j0-1..j0+2 (border lines).  edge: 1 if the lane holds image columns 0,1,
 // 2 if it holds W-2,W-1 (W % 16 == 0: only c0 == 0 / c0 == W-8), else 0.
-// Packed horizontal weights -w/1024 for pixel pairs (x, x+1), in the constant
-// bank (loaded with LDC where used; as literals, ptxas kept rematerialising
-// them on every row under the 128-register cap -- measured 4% slower).
-// {lo, hi} = {-3, -1}, {-5, -7}, {-7, -5}, {-1, -3} / 1024 as f32 bit pairs.
-__constant__ unsigned long long c_wts[4] = {0xba800000bb400000ull, 0xbbe00000bba00000ull, 0xbba00000bbe00000ull,
-                                            0xbb400000ba800000ull};
-__device__ __forceinline__ unsigned long long cwt(int i) { return c_wts[i]; }
-__device__ __forceinline__ float div16(float s) { return __fmul_rn(s, 1.0f / 16.0f); }
-
-// The 2-pixel ring (L140-L142 upscale border, L160 Sobel frame, L208
-// overshoot frame): overrides of -U, pEdge and the overshoot window.
-__device__ __forceinline__ void set_frame_px(uint32_t pe[4], uint32_t MX[4], uint32_t MN[4], int x) {
-  set_px(pe, x, 0u);         // Sobel frame: 0
-  set_px(MX, x, kF16_255);   // overshoot frame: the clamped preliminary value,
-  set_px(MN, x, 0u);         // i.e. window [0, 255]
-}
-// Rows 0,1 (line of D row 0) and H-2,H-1 (line of D row h-1): here D0 is
-// that D row; the corners follow the step order (v)-(vii).
-__device__ __forceinline__ void ring_rows(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4],
-                                          const float4 &D0, const float4 &D1, int r, int c0, int W, int H,
-                                          int edge) {
-  const float q0 = D0.y, q1 = D0.z, q2 = D0.w;
-  float u[8] = {div16(q0),         line_val(q0, q1, 1), line_val(q0, q1, 2), line_val(q0, q1, 3),
-                div16(q1),         line_val(q1, q2, 1), line_val(q1, q2, 2), line_val(q1, q2, 3)};
-  if (c0 + 5 == W - 3) u[5] = div16(q1);  // third last <- fourth last
-  const bool top = r < 2;
-  if (edge == 1 && top) u[1] = div16(q0);  // (v)+(vi): top-left 2x2 = D[0][0]
-  if (edge == 2) {                         // columns W-2, W-1 (D column w-1 = j0+1)
-    const float v = (top && r == 1) ? line_val(D0.z, D1.z, 1) : div16(D0.z);
-    u[6] = v;
-    u[7] = v;
-  }
-#pragma unroll
-  for (int x = 0; x < 8; ++x) NU[x] = -u[x];
-  if (edge == 1) set_frame_px(pe, MX, MN, 0);  // column 0 (rows 1, H-2)
-  if (edge == 2) set_frame_px(pe, MX, MN, 7);  // column W-1
-  if (r == 0 || r == H - 1) {
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      pe[i] = 0u;
-      MX[i] = kF16_255 | (kF16_255 << 16);
-      MN[i] = 0u;
-    }
-  }
-}
-// Columns 0,1 / W-2,W-1 on rows 2..H-3 (lines of D columns 0 / w-1).
-__device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4],
-                                          const float4 &D0, const float4 &D1, int r, int H, int edge) {
-  const int rr = (r == H - 3) ? H - 4 : r;  // third last <- fourth last
-  const int k = rr & 3;
-  const float x0 = edge == 1 ? D0.y : D0.z, x1 = edge == 1 ? D1.y : D1.z;
-  const float v = -(k == 0 ? div16(x0) : line_val(x0, x1, k));
-  if (edge == 1) {
-    NU[0] = v;
-    NU[1] = v;
-    set_frame_px(pe, MX, MN, 0);
-  } else if (edge == 2) {
-    NU[6] = v;
-    NU[7] = v;
-    set_frame_px(pe, MX, MN, 7);
-  }
-}
-
 template <bool kRingRows>
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
                                        const float4 &D0, const float4 &D1, uint32_t lut_q,
@@ -488,36 +221,7 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   if (store) st_stream_u64(orow, o, pol_out);
 }
 
-__device__ __forceinline__ float4 f4fma(float a, const float4 &x, const float4 &y) {  // a*x + y, exact here
-  return make_float4(__fmaf_rn(a, x.x, y.x), __fmaf_rn(a, x.y, y.y), __fmaf_rn(a, x.z, y.z), __fmaf_rn(a, x.w, y.w));
-}
-__device__ __forceinline__ float4 f4add(const float4 &x, const float4 &y) {  // two packed f32x2 adds
-  unsigned long long lo, hi;
-  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(lo) : "l"(f2pack(x.x, x.y)), "l"(f2pack(y.x, y.y)));
-  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(hi) : "l"(f2pack(x.z, x.w)), "l"(f2pack(y.z, y.w)));
-  const float2 a = f2unpack(lo), b = f2unpack(hi);
-  return make_float4(a.x, a.y, b.x, b.y);
-}
-__device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y) {  // 2 (x - y), exact here
-  return make_float4(__fmul_rn(2.0f, __fsub_rn(x.x, y.x)), __fmul_rn(2.0f, __fsub_rn(x.y, y.y)),
-                     __fmul_rn(2.0f, __fsub_rn(x.z, y.z)), __fmul_rn(2.0f, __fsub_rn(x.w, y.w)));
-}
-
-// Stage ring shared by the producer and the consumers: stage s (a running
-// count) lives in buffer s % kStages and completes phase (s / kStages) & 1.
-struct Ring {
-  uint32_t sbase, full0, empty0;
-  __device__ __forceinline__ static int buf(int s) { return (unsigned)s % kStages; }
-  __device__ __forceinline__ static uint32_t phase(int s) { return ((unsigned)s / kStages) & 1u; }
-  __device__ __forceinline__ uint32_t stage(int s) const { return sbase + (uint32_t)(buf(s) * kStage); }
-  __device__ __forceinline__ void wait_full(int s) const {
-    mbar_wait(full0 + 8u * buf(s), phase(s));
-  }
-  __device__ __forceinline__ void release(int s, int lane) const {  // one arrival per consumer warp
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty0 + 8u * buf(s));
-  }
-};
+using Ring = RingT<kStages, kStage>;
 
 // Pass 2 of one warp over a task of nsub sub-tiles (stages s .. s+nsub-1,
 // the first already waited for).  out: first row of the output rows
@@ -899,18 +603,6 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, size_t pitch, size_t fs, int box_cols,
-              int box_rows) {
-  auto fn = encode_fn();
-  if (!fn) return false;
-  const cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)n};  // [n][H][W] at the given strides
-  const cuuint64_t strides[2] = {(cuuint64_t)pitch, (cuuint64_t)fs};
-  const cuuint32_t box[3] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows, 1};
-  const cuuint32_t estr[3] = {1, 1, 1};
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, (void *)imgs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
 
 // Per-device launch facts, filled by preload_step() (sharp_create calls it
 // after selecting the context's device): SM count and the step kernel's
@@ -941,6 +633,19 @@ extern "C" int sharp_debug_timeline(unsigned long long *out, int reset) {
   return 0;
 }
 #endif
+
+bool make_map(CUtensorMap *m, const uint8_t *imgs, int n, int W, int H, size_t pitch, size_t fs, int box_cols,
+              int box_rows) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  const cuuint64_t dims[3] = {(cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)n};  // [n][H][W] at the given strides
+  const cuuint64_t strides[2] = {(cuuint64_t)pitch, (cuuint64_t)fs};
+  const cuuint32_t box[3] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows, 1};
+  const cuuint32_t estr[3] = {1, 1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, (void *)imgs, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
 
 bool tma_supported(const uint8_t *imgs, const uint8_t *outs, int W, int H) {
   return (W % 16) == 0 && tma_supported_strided(imgs, W, (size_t)W * H, outs, W, (size_t)W * H, W, H);

@@ -84,7 +84,8 @@ struct sharp_ctx {
   size_t frames_cap = 0;
   unsigned int *tcounters = nullptr;  // dynamic-scheduling task counters, one per step launch
   size_t tcounters_cap = 0;
-  unsigned int *lut_done = nullptr;   // per frame: finished LUT-task warps (batch kernel)
+  unsigned int *lut_done = nullptr;   // per frame: finished LUT-task warps / table chunks
+  unsigned int *lut_next = nullptr;   // per frame: table chunks grabbed (resident kernel)
   unsigned long long *acc = nullptr;  // per frame: pass-1 arrivals << 40 | partial sum (batch kernel)
   float2 *luts = nullptr;             // per frame lookup tables (batch kernel)
   // general layouts (sharp_run_ex): dense padded in / out, device copies of host byte ranges
@@ -132,6 +133,9 @@ int cuda_fail(sharp_ctx *c, cudaError_t e, const char *where) {
     if (e__ != cudaSuccess) return cuda_fail(ctx, e__, #expr); \
   } while (0)
 
+// Paths served by the TMA-staged kernels (the resident kernel or the step kernel).
+bool tma_family(int path) { return path == SHARP_PATH_AUTO || path == SHARP_PATH_STEP || path == SHARP_PATH_RES; }
+
 bool params_ok(const sharp_params &p) {
   // R16 ranges; NaN fails every comparison.
   return p.amount >= 0.0f && p.amount <= 16.0f && p.gamma >= 0.0f && p.gamma <= 4.0f &&
@@ -174,19 +178,20 @@ int ensure_frames(sharp_ctx *ctx, size_t n, size_t n_tc = 0) {
   cudaFree(ctx->luts);
   ctx->zero_block = nullptr;
   ctx->sums = ctx->acc = nullptr;
-  ctx->lut_done = ctx->tcounters = nullptr;
+  ctx->lut_done = ctx->lut_next = ctx->tcounters = nullptr;
   ctx->means = nullptr;
   ctx->luts = nullptr;
   ctx->frames_cap = ctx->tcounters_cap = ctx->zero_bytes = 0;
   const size_t cap = std::max(n, ctx->frames_cap), tcap = std::max(need_tc, 2 * cap + 2);
   const size_t b_acc = cap * 8, b_sums = cap * 8, b_done = (cap * 4 + 7) & ~(size_t)7, b_tc = tcap * 4;
-  CK(cudaMalloc(&ctx->zero_block, b_acc + b_sums + b_done + b_tc));
+  CK(cudaMalloc(&ctx->zero_block, b_acc + b_sums + 2 * b_done + b_tc));
   uint8_t *z = static_cast<uint8_t *>(ctx->zero_block);
   ctx->acc = reinterpret_cast<unsigned long long *>(z);
   ctx->sums = reinterpret_cast<unsigned long long *>(z + b_acc);
   ctx->lut_done = reinterpret_cast<unsigned int *>(z + b_acc + b_sums);
-  ctx->tcounters = reinterpret_cast<unsigned int *>(z + b_acc + b_sums + b_done);
-  ctx->zero_bytes = b_acc + b_sums + b_done + b_tc;
+  ctx->lut_next = reinterpret_cast<unsigned int *>(z + b_acc + b_sums + b_done);
+  ctx->tcounters = reinterpret_cast<unsigned int *>(z + b_acc + b_sums + 2 * b_done);
+  ctx->zero_bytes = b_acc + b_sums + 2 * b_done + b_tc;
   CK(cudaMalloc(&ctx->means, cap * sizeof(double)));
   CK(cudaMalloc(&ctx->luts, cap * sharp::kLutSize * sizeof(float2)));
   ctx->frames_cap = cap;
@@ -364,7 +369,14 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
                    "SHARP_PATH_STEP needs w % 16 == 0, 16-byte aligned input, 8-byte aligned output, w*h <= 2^29 "
                    "and no per-pixel reading switch (R2, R5, R14)");
-  const bool tma = (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) && tma_ok;
+  const bool tma = tma_family(ctx->path) && tma_ok;
+  // the resident kernel (TMEM pEdge) for frames up to ~10 Mpx, else the step kernel
+  // (AUTO takes it once it beats the step kernel: see DESIGN.md sec. 7)
+  const bool res = tma && ctx->path == SHARP_PATH_RES && sharp::res_supported(w, h, n);
+  if (ctx->path == SHARP_PATH_RES && !res)
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
+                   "SHARP_PATH_RES needs the step kernel's geometry and at most 2 x (resident grid) tiles of "
+                   "960 x 12 per frame");
   if (tma) {  // the whole batch in one persistent launch
     sharp::BatchLaunch a;
     a.in = din;
@@ -375,12 +387,15 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
     a.means = ctx->means + frame_base;
     a.luts = ctx->luts + frame_base * sharp::kLutSize;
     a.lut_done = ctx->lut_done + frame_base;
+    a.lut_next = ctx->lut_next + frame_base;
     a.task_counter = tc;
     a.in_pitch = str.in_pitch;
     a.in_fs = str.in_fs;
     a.out_pitch = str.out_pitch;
     a.out_fs = str.out_fs;
-    CK(timed(ctx, st, 3, (double)n * fb, [&] { return sharp::launch_batch_tma(a, w, h, prm, st); }));
+    CK(timed(ctx, st, 3, (double)n * fb, [&] {
+      return res ? sharp::launch_batch_res(a, w, h, prm, st) : sharp::launch_batch_tma(a, w, h, prm, st);
+    }));
     *launches += 1;
     return SHARP_OK;
   }
@@ -427,7 +442,7 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   // kernel (gather + scatter cost 4 B/px, far less than the two-pass path's
   // compute at these widths).  Synchronous calls only.
   if (!async && kin == kDevice && kout == kDevice && (w % 16) == 8 && w >= 24 && !(prm.flags & sharp::kReadPerPixel) &&
-      (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) && (size_t)w * h <= (1u << 29)) {
+      tma_family(ctx->path) && (size_t)w * h <= (1u << 29)) {
     const Layout L{(size_t)w, (size_t)w * h, 1};
     return run_general(ctx, in, L, n, 1, w, h, prm, out, L, kin, kout);
   }
@@ -437,7 +452,7 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   // host pipeline whose chunks run on the step kernel (staging buffers are
   // cudaMalloc'd, so only the geometry, the path and the switches decide)
   const bool step_chunks = staged && (w % 16) == 0 && (size_t)w * h <= (1u << 29) &&
-                           (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+                           tma_family(ctx->path) &&
                            !(prm.flags & sharp::kReadPerPixel);
   const size_t chunk = chunk_frames(ctx, fb, n, step_chunks ? kHostStepChunkBudget : kL2ChunkBudget);
   if ((rc = ensure_frames(ctx, (size_t)n))) return rc;
@@ -548,7 +563,7 @@ int run_general(sharp_ctx *ctx, const uint8_t *in, const Layout &Li, int n, int 
   // Units whose padded width is a multiple of 8 run on the step kernel from a
   // scratch with a 16-byte row pitch (the TMA stride rule); others dense on
   // the two-pass path.
-  const bool step = (W4 % 8) == 0 && W4 >= 16 && H4 >= 8 && (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+  const bool step = (W4 % 8) == 0 && W4 >= 16 && H4 >= 8 && tma_family(ctx->path) &&
                     !(prm.flags & sharp::kReadPerPixel) && (size_t)W4 * H4 <= (1u << 29);
   const int P = step ? (W4 + 15) & ~15 : W4;
   const size_t ub = (size_t)P * H4;
@@ -687,7 +702,7 @@ int run_ex_impl(sharp_ctx *ctx, const uint8_t *in, const sharp_layout *lin, int 
   // zero-copy: single-channel device frames with w % 8 == 0, h % 4 == 0 and
   // strides the TMA step kernel takes directly
   if (C == 1 && Li.es == 1 && Lo.es == 1 && !overlap && kin == kDevice && kout == kDevice && !(w & 7) && !(h & 3) &&
-      w >= 8 && h >= 8 && (ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) &&
+      w >= 8 && h >= 8 && tma_family(ctx->path) &&
       !(flags & sharp::kReadPerPixel) &&
       sharp::tma_supported_strided(in, Li.pitch, Li.fs, out, Lo.pitch, Lo.fs, w, h))
     return run_device_strided(ctx, in, Li, n, w, h, prm, out, Lo);
@@ -725,7 +740,7 @@ int band_impl(sharp_ctx *ctx, int mode, const uint8_t *band, int w, int h, int r
     const size_t na = (size_t)(in1 - in0) * w, nb = (size_t)(row1 - row0) * w;
     if (a < b + nb && b < a + na) return set_err(ctx, SHARP_EINVAL, "%s", "input and output overlap");
   }
-  if (!(ctx->path == SHARP_PATH_AUTO || ctx->path == SHARP_PATH_STEP) ||
+  if (!tma_family(ctx->path) ||
       !sharp::tma_supported(band, mode == sharp::kStepPass2 ? out : (uint8_t *)band, w, h))
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
                    "row bands need the TMA path (w % 16 == 0, 16-byte aligned band, 8-byte aligned out)");
@@ -831,7 +846,7 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
     }
     if (e != cudaSuccess) break;
     // load every kernel now (lazy module loading can deadlock spinning kernels, kernels.h)
-    if ((e = sharp::preload_step()) != cudaSuccess || (e = sharp::preload_two_pass()) != cudaSuccess ||
+    if ((e = sharp::preload_step()) != cudaSuccess || (e = sharp::preload_res()) != cudaSuccess || (e = sharp::preload_two_pass()) != cudaSuccess ||
         (e = sharp::preload_staged()) != cudaSuccess || (e = sharp::preload_p2p()) != cudaSuccess ||
         (e = sharp::preload_layout()) != cudaSuccess)
       break;
@@ -1162,7 +1177,7 @@ int sharp_ipc_close_handle(void *d_ptr) {
 }
 
 int sharp_set_path(sharp_ctx *ctx, int path) {
-  if (!ctx || path < SHARP_PATH_AUTO || path > SHARP_PATH_STAGED) return SHARP_EINVAL;
+  if (!ctx || path < SHARP_PATH_AUTO || path > SHARP_PATH_RES) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
   ctx->path = path;
   return SHARP_OK;

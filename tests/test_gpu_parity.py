@@ -27,11 +27,12 @@ PARAMS = [
 ]
 
 
-@pytest.fixture(scope="module", params=["auto", "generic", "staged"])
+@pytest.fixture(scope="module", params=["auto", "step", "generic", "staged"])
 def sh(request):
-    """A context on the automatic kernel path (TMA-staged persistent kernels
-    when W % 16 == 0), one forced onto the generic two-pass LDG kernels, and
-    one on the paper's staged base design (one kernel per stage)."""
+    """A context on the automatic kernel path (the TMEM-resident kernel, else
+    the step kernel, when W % 16 == 0), one forced onto the step kernel, one
+    forced onto the generic two-pass LDG kernels, and one on the paper's
+    staged base design (one kernel per stage)."""
     assert torch.cuda.is_available(), "GPU tests need a CUDA device"
     import os
     old = os.environ.get("SHARP_FORCE_GENERIC")
@@ -39,6 +40,9 @@ def sh(request):
     s = Sharpener()
     if request.param == "staged":
         s.set_path(SHARP_PATH_STAGED)
+    if request.param == "step":
+        s.set_path(SHARP_PATH_STEP)
+        s._force_step = True
     if old is None:
         del os.environ["SHARP_FORCE_GENERIC"]
     else:
@@ -57,6 +61,8 @@ def gpu_run(sh, img, prm=DEFAULT):
 
 
 def assert_parity(sh, img, prm=DEFAULT):
+    if getattr(sh, "_force_step", False) and (img.shape[-1] % 16 or img.shape[-1] < 16):
+        pytest.skip("SHARP_PATH_STEP needs W % 16 == 0 (the other fixtures cover this size)")
     out, S, mean = gpu_run(sh, img, prm)
     ref, S_ref, mean_ref = oracle.sharpen(img, *prm)
     bad = np.argwhere(out != ref)
