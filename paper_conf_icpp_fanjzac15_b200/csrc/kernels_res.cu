@@ -51,42 +51,63 @@ namespace sharp {
 namespace {
 using namespace dev;
 
-constexpr int kT = kTH;                // rows per tile (pass 1 and pass 2)
-constexpr int kRowsP1 = kT + 2;        // pass-1 boxes: rows R0-1 .. R0+kT
-constexpr int kResCtasPerSm = 3;
+constexpr int kT = kTH;                 // rows per warp tile (pass 1 and pass 2)
+constexpr int kWR = 3;                  // warp rows per CTA tile
+constexpr int kTileRows = kWR * kT;     // 36 rows per CTA tile
+constexpr int kCompute = kWarpsT * kWR;  // 12 compute warps (4 columns x 3 rows of warp tiles)
+constexpr int kThreadsR = 32 * (kCompute + 2);  // + producer warp + table warp: ONE CTA per SM
+constexpr int kRowsStage = kTileRows + 8;       // stage rows: image rows R0-4 .. R0+39
+constexpr int kRowsP1 = kTileRows + 2;          // pass-1 boxes: rows R0-1 .. R0+36 (stage rows 3 ..)
+constexpr int kSlotR = kPitch * kRowsStage;     // region A of one warp column
+constexpr int kRegBR = kWarpsT * kSlotR;        // region B (the last warp column's right halo)
 #ifndef SHARP_RES_STAGES
-#define SHARP_RES_STAGES 2
+#define SHARP_RES_STAGES 3
 #endif
-constexpr int kResStages = SHARP_RES_STAGES;  // smem ring depth (P1 / P2 stages)
-constexpr int kResStage = (kRegB + kPitchB * kRows2 + 127) / 128 * 128;
-#ifndef SHARP_RES_SLOTS
-#define SHARP_RES_SLOTS 3
-#endif
-#ifndef SHARP_RES_LUTBUFS
-#define SHARP_RES_LUTBUFS 1
-#endif
-// pEdge slots per CTA: tile k uses slot k % kSlots; slots 0 and 1 are in
-// TMEM, slot 2 (if any) in shared memory (4 warps x 12 rows x 32 lanes x 16 B).
-constexpr int kSlots = SHARP_RES_SLOTS;
-constexpr int kLutBufs = SHARP_RES_LUTBUFS;  // 1 suffices: consecutive pass-2 stages never overlap (2 stages)
-constexpr int kPeRowBytes = 32 * 16;          // one warp's pEdge row in the smem slot
-constexpr int kResLutOff = kResStages * kResStage;  // LUT buffer(s) after the stages
-constexpr int kResPeOff = kResLutOff + kLutBufs * kLutBytes;  // the smem pEdge slot
-constexpr int kResDummy = kResPeOff + (kSlots > 2 ? kWarpsT * kT * kPeRowBytes : 0);  // end stage's 16-B copy
+constexpr int kResStages = SHARP_RES_STAGES;    // smem ring depth (P1 / P2 stages)
+constexpr int kResStage = (kRegBR + kPitchB * kRowsStage + 127) / 128 * 128;
+constexpr int kLutBufs = 2;
+constexpr int kResLutOff = kResStages * kResStage;     // LUT buffers after the stages
+constexpr int kResDummy = kResLutOff + kLutBufs * kLutBytes;  // end stage's 16-B copy target
 constexpr int kResBarOff = kResDummy + 16;
 constexpr int kResSmem = kResBarOff + 16 * kResStages;
-// TMEM: 128 columns per CTA (3 CTAs -> 384 of the SM's 512); slot q of a
-// tile at column 48 q, pEdge row j of the tile at +4 j (4 words per lane).
-constexpr uint32_t kTmemCols = 128;
+// TMEM: all 512 columns (one CTA per SM); warp w uses lane quarter w % 4
+// (the hardware's mapping) and columns 160 (w / 4) ..: three slots of 48
+// columns, slot q of a tile at +48 q, pEdge row j of the warp tile at +4 j.
+constexpr uint32_t kTmemCols = 512;
+constexpr int kWarpCols = 160;
+constexpr int kSlots = 3;
 constexpr int kSlotCols = 4 * kT;
-static_assert(2 * kSlotCols <= (int)kTmemCols, "two tile slots fit the allocation");
-static_assert(kSlots == 2 || kSlots == 3, "2 TMEM slots (+ 1 in shared memory)");
+static_assert(kSlots * kSlotCols <= kWarpCols && kWR * kWarpCols <= (int)kTmemCols, "TMEM slots");
 constexpr int kChunk = 16;                  // table entries per chunk: lanes 0-15 adj, 16-31 osc
 constexpr int kChunks = kLut2 / kChunk;     // 48
 constexpr int kAccShift = 40;
-static_assert(kResStage % 128 == 0 && kResLutOff % 128 == 0, "TMA smem destinations");
+static_assert(kResStage % 128 == 0 && kResLutOff % 128 == 0 && (3 * kPitch) % 128 == 0, "TMA smem destinations");
+static_assert(kResSmem <= 227 * 1024, "one CTA per SM");
 
 using RRing = RingT<kResStages, kResStage>;
+
+// Lane words of a warp column in this kernel's stage layout (cf. lane_row of
+// tma_common.cuh: 44-row regions).  rb_shift: row offset of region B (the
+// pass-1 region-B box lands at row 0 of region B but holds image row R0-1,
+// stage row 3, so its base is moved 3 rows back).
+__device__ __forceinline__ LaneRow lane_row_r(uint32_t stage, int wc, int lane, int rb_shift) {
+  if (lane == 30) {
+    if (wc == kWarpsT - 1) return LaneRow{stage + (uint32_t)(kRegBR - rb_shift * kPitchB), (uint32_t)kPitchB};
+    return LaneRow{stage + (uint32_t)((wc + 1) * kSlotR + kCol0), (uint32_t)kPitch};
+  }
+  return LaneRow{stage + (uint32_t)(wc * kSlotR + kCol0 + 8 * (lane < 31 ? lane : -1)), (uint32_t)kPitch};
+}
+// The boxes of a CTA tile of nw warp columns into stage st: region A per
+// column at row a_row, region B (when all 4 columns exist) at row 0.
+__device__ __forceinline__ void tma_tiles_r(uint32_t st, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0,
+                                            int nw, int a_row, int r, int f, uint32_t bar, uint64_t policy) {
+  for (int w = 0; w < nw; ++w)
+    tma_box(st + w * kSlotR + a_row * kPitch, mapA, C0 + w * kTW - kCol0, r, f, bar, policy);
+  if (nw == kWarpsT) tma_box(st + kRegBR, mapB, C0 + kWarpsT * kTW, r, f, bar, policy);
+}
+__device__ __forceinline__ uint32_t tile_bytes_r(int nw, int rows) {
+  return (uint32_t)((nw * kPitch + (nw == kWarpsT ? kPitchB : 0)) * rows);
+}
 #ifndef SHARP_RES_CWAIT_NS
 #define SHARP_RES_CWAIT_NS 0  // consumer stage waits: 0 = try_wait, else test_wait + back-off up to this (ns)
 #endif
@@ -149,14 +170,6 @@ __device__ __forceinline__ void tmem_ld4(uint32_t taddr, uint32_t v[4]) {
                : "r"(taddr)
                : "memory");
 }
-__device__ __forceinline__ void sts_u128(uint32_t a, const uint32_t v[4]) {
-  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3])
-               : "memory");
-}
-__device__ __forceinline__ void lds_u128(uint32_t a, uint32_t v[4]) {
-  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(a)
-               : "memory");
-}
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
@@ -164,10 +177,11 @@ __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.
 // pEdge of rows R0 .. R0+kT-1 (smem row of image row r: r - R0 + 1) into
 // TMEM row j = r - R0 of the slot, and the warp's partial sum of the Sobel
 // body (rows 1..rmax1, columns 1..W-2; L160: the frame is 0).
-__device__ __forceinline__ float p1_tile(uint32_t stage, int warp, int W, int rmax1, int C0w, int R0, int lane,
-                                         uint32_t tslot, uint32_t spe) {
+// (aw: the warp column's lane words; sb: stage row of image row R0 - 1.)
+__device__ __forceinline__ float p1_tile(const LaneRow &aw0, int sb, int W, int rmax1, int C0w, int R0, int lane,
+                                         uint32_t tslot) {
   const int c0 = C0w + 8 * lane;
-  const LaneRow aw = lane_row(stage, warp, lane);
+  const LaneRow aw{aw0.base + (uint32_t)sb * aw0.pitch, aw0.pitch};  // row offsets below are compile-time
   RowD ra = derive_w<false>(row_words(aw, 0), lane);
   RowD rb = derive_w<false>(row_words(aw, 1), lane);
   float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};  // exact: < 12 rows * 1530
@@ -179,8 +193,7 @@ __device__ __forceinline__ float p1_tile(uint32_t stage, int warp, int W, int rm
       const RowD rc = derive_w<false>(row_words(aw, m + a + 2), lane);
       uint32_t pe[4];
       sobel(ra, rb, rc, pe);
-      if (spe) sts_u128(spe + (uint32_t)((m + a) * kPeRowBytes), pe);  // the shared-memory slot
-      else tmem_st4(tslot + (uint32_t)(4 * (m + a)), pe);
+      tmem_st4(tslot + (uint32_t)(4 * (m + a)), pe);
       const uint16_t on = ((unsigned)(r - 1) < (unsigned)rmax1) ? (uint16_t)0x3C00u : (uint16_t)0u;
 #pragma unroll
       for (int x = 0; x < 8; ++x)
@@ -198,7 +211,7 @@ __device__ __forceinline__ float p1_tile(uint32_t stage, int warp, int W, int rm
   if (c0 == 0) sum = __fsub_rn(sum, acc[0]);
   if (c0 == W - 8) sum = __fsub_rn(sum, acc[7]);
   if (lane >= 30 || c0 >= W) sum = 0.0f;
-  if (!spe) tmem_wait_st();  // the slot's rows are in TMEM before this warp's pass 2 reads them
+  tmem_wait_st();  // the slot's rows are in TMEM before this warp's pass 2 reads them
   return sum;
 }
 
@@ -279,14 +292,15 @@ __device__ __forceinline__ void p2_row_res(const RowM &ra, const RowM &rb, const
 
 // Pass 2 of one warp tile (rows R0 .. R0+kT-1; smem row of image row r:
 // r - R0 + 4), pEdge row j from TMEM column tslot + 4 j.
-__device__ __forceinline__ void p2_tile(uint32_t stage, uint32_t lut_q, uint32_t tslot, uint32_t spe,
-                                        uint8_t *__restrict__ out,
-                                        uint32_t out_pitch, int W, int H, int C0w, int R0, int warp, int lane) {
+// (aw: the warp column's lane words; sb: stage row of image row R0 - 4.)
+__device__ __forceinline__ void p2_tile(const LaneRow &aw0, int sb, uint32_t lut_q, uint32_t tslot,
+                                        uint8_t *__restrict__ out, uint32_t out_pitch, int W, int H, int C0w, int R0,
+                                        int lane) {
+  const LaneRow aw{aw0.base + (uint32_t)sb * aw0.pitch, aw0.pitch};
   const int c0 = C0w + 8 * lane;
   const bool active = lane < 30 && c0 < W;
   const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
-  const LaneRow aw = lane_row(stage, warp, lane);
   // Vertical interpolation (L146, R3): V(r+1) = V(r) + 2 (D_{i+1} - D_i) on
   // r = 4i+2 .. 4i+5, restarted at r = 4i+2 (exact integers, x 128).
   const float4 Dp = dblock(aw, 0, lane);  // D row R0/4 - 1
@@ -301,7 +315,7 @@ __device__ __forceinline__ void p2_tile(uint32_t stage, uint32_t lut_q, uint32_t
   const int rend_l = active ? rend : R0;
   // pEdge rows: the TMEM load of row j + 1 is issued while row j is computed
   uint32_t pe_next[4];
-  if (!spe) tmem_ld4(tslot, pe_next);
+  tmem_ld4(tslot, pe_next);
 #pragma unroll 1
   for (int r = R0; r < rend; r += 3) {
 #pragma unroll
@@ -309,14 +323,10 @@ __device__ __forceinline__ void p2_tile(uint32_t stage, uint32_t lut_q, uint32_t
       const int rr = r + u;
       const int sm = rr - R0 + 4;
       uint32_t pe[4];
-      if (spe) {
-        lds_u128(spe + (uint32_t)((rr - R0) * kPeRowBytes), pe);
-      } else {
-        tmem_wait_ld();
+      tmem_wait_ld();
 #pragma unroll
-        for (int i = 0; i < 4; ++i) pe[i] = pe_next[i];
-        tmem_ld4(tslot + (uint32_t)(4 * (rr - R0 + 1)), pe_next);  // (row kT: inside the allocation, unused)
-      }
+      for (int i = 0; i < 4; ++i) pe[i] = pe_next[i];
+      tmem_ld4(tslot + (uint32_t)(4 * (rr - R0 + 1)), pe_next);  // (row kT: inside the warp's columns, unused)
       if ((rr & 3) == 0) {  // next D block row
         D0 = D1;
         D1 = dblock(aw, sm + 4, lane);
@@ -332,7 +342,7 @@ __device__ __forceinline__ void p2_tile(uint32_t stage, uint32_t lut_q, uint32_t
       rb = rc;
     }
   }
-  if (!spe) tmem_wait_ld();  // the last prefetch lands before the slot is rewritten
+  tmem_wait_ld();  // the last prefetch lands before the slot is rewritten
 }
 
 // ------------------------------------------------- table build (producer)
@@ -360,7 +370,7 @@ __device__ __forceinline__ void build_chunk(const ResParams &sp, int f, int c, u
 // builds one chunk if the frame's pass 1 is complete and a chunk is left
 // (returns 0), else returns -1 (nothing to do now).  Warp-uniform.
 __device__ __forceinline__ int table_step(const ResParams &sp, int f, int lane) {
-  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kWarpsT) << kAccShift;
+  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kCompute) << kAccShift;
   unsigned done = 0;
   unsigned long long a = 0;
   if (lane == 0) {
@@ -397,7 +407,7 @@ __device__ __forceinline__ void ensure_table(const ResParams &sp, int f, int lan
 #ifdef SHARP_DIAG_NO_TABLE_WAIT  // timing experiment only: wrong output
   return;
 #endif
-  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kWarpsT) << kAccShift;
+  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kCompute) << kAccShift;
 #ifdef SHARP_DIAG_RES
   long long t_first_complete = 0, t_enter = clock64();
   int iters = 0;
@@ -445,7 +455,7 @@ __device__ __forceinline__ void ensure_table(const ResParams &sp, int f, int lan
 }
 
 // ============================================================== the kernel
-__global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
+__global__ void __launch_bounds__(kThreadsR, 1)
     res_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
                const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, ResParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
@@ -465,7 +475,7 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
   if (threadIdx.x == 0) {
     for (int i = 0; i < kResStages; ++i) {
       mbar_init(ring.full0 + 8 * i, 1);
-      mbar_init(ring.empty0 + 8 * i, kWarpsT);
+      mbar_init(ring.empty0 + 8 * i, kCompute);
     }
     fence_barrier_init();
   }
@@ -473,7 +483,28 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 
-  if (warp == kWarpsT) {
+  if (warp == kCompute + 1) {
+    // --------------------------------------------------------- table warp
+    // Builds chunks of every frame's table as soon as the frame's pass 1 is
+    // complete (all SMs' table warps in parallel: a frame's 48 chunks take
+    // about one f64 pow latency).  The tables are the dependency of every
+    // pass-2 tile, so their build must not wait for the producers that need
+    // them (measured: 5 us per frame when only the waiting producers built).
+    for (int f = 0; f < sp.n; ++f) {
+      for (;;) {
+        const int st = table_step(sp, f, lane);
+        if (st == 1) break;                                      // complete
+        if (st < 0) {
+          unsigned next = 0;
+          if (lane == 0) next = ld_relaxed_u32(&sp.lut_next[f]);
+          if (__shfl_sync(0xffffffffu, next, 0) >= (unsigned)kChunks) break;  // all chunks taken
+          __nanosleep(SHARP_RES_HELP_NS);
+        }
+      }
+    }
+    return;
+  }
+  if (warp == kCompute) {
     // ------------------------------------------------------------ producer
     const uint64_t pol_keep = policy_evict_last(), pol_drop = policy_evict_first();
     int s = 0;                                        // stages filled
@@ -507,7 +538,7 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
       f = t / sp.per_frame;
       const int i = t - f * sp.per_frame, ty = i / sp.tiles_x;
       C0 = (i - ty * sp.tiles_x) * kCtaCols;
-      R0 = ty * kT;
+      R0 = ty * kTileRows;
       nw = 0;
 #pragma unroll
       for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < sp.W);
@@ -520,8 +551,8 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
         const uint32_t full = ring.full0 + 8u * b, st = ring.stage(s);
         stage_task[b] = make_int4(kRP1, f, C0, R0);
         stage_aux[b] = make_int2(q, 0);
-        mbar_expect_tx(full, tile_bytes(nw, kRowsP1));
-        tma_tiles(st, &map1A, &map1B, C0, nw, R0 - 1, f, full, pol_keep);
+        mbar_expect_tx(full, tile_bytes_r(nw, kRowsP1));
+        tma_tiles_r(st, &map1A, &map1B, C0, nw, 3, R0 - 1, f, full, pol_keep);  // stage row 3 = image row R0-1
       }
       __syncwarp();
       ++s;
@@ -532,7 +563,7 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
       // LUT buffer: the one already holding frame f's table, else the one the
       // previous pass-2 tile did not use (free once the stage that last read
       // it is released)
-      const int lb = kLutBufs == 1 ? 0 : lut_frame0 == f ? 0 : lut_frame1 == f ? 1 : (lut_prev ^ 1);
+      const int lb = lut_frame0 == f ? 0 : lut_frame1 == f ? 1 : (lut_prev ^ 1);
       const bool copy = (lb ? lut_frame1 : lut_frame0) != f;
       // While the stage is still in use: help build frame f's table (its
       // builders are the producers that wait for it), and once it is complete
@@ -540,6 +571,9 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
       // tile loads go out at once (each global round trip here costs ~0.5 us
       // under load; measured).
       bool ready = !copy;
+#ifdef SHARP_DIAG_NO_TABLE_WAIT
+      ready = true;
+#endif
       if (s >= kResStages) {
         const uint32_t eb = ring.empty0 + 8u * RRing::buf(s), par = RRing::phase(s) ^ 1u;
         while (!ready && !mbar_test(eb, par)) {
@@ -561,13 +595,13 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
         stage_aux[b] = make_int2(q, lb);
         const int tl = lb ? lut_last1 : lut_last0;
         if (copy && tl > s - kResStages) mbar_wait(ring.empty0 + 8u * RRing::buf(tl), RRing::phase(tl));
-        mbar_expect_tx(full, tile_bytes(nw, kRows2) + (copy ? (uint32_t)kLutBytes : 0u));
+        mbar_expect_tx(full, tile_bytes_r(nw, kRowsStage) + (copy ? (uint32_t)kLutBytes : 0u));
 #ifdef SHARP_DIAG_RES
         rd_tma[b] = clock64();
         rd_lut[b] = rd_tma[b];
 #endif
         if (copy && ready) bulk_copy(lut_dst, lut_src, kLutBytes, full);
-        tma_tiles(st, &map2A, &map2B, C0, nw, R0 - 4, f, full, pol_drop);  // (loads need no table)
+        tma_tiles_r(st, &map2A, &map2B, C0, nw, 0, R0 - 4, f, full, pol_drop);  // (loads need no table)
       }
       if (copy && !ready) {
 #ifdef SHARP_DIAG_RES
@@ -596,22 +630,15 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
     if (t0 < sp.ntasks) issue_p1(t0, 0);
     int t1 = t0 < sp.ntasks ? next_tile() : sp.ntasks;
     if (t1 < sp.ntasks) issue_p1(t1, 1);
-    int t2 = sp.ntasks;
-    if (kSlots > 2) {
-      t2 = t1 < sp.ntasks ? next_tile() : sp.ntasks;
-      if (t2 < sp.ntasks) issue_p1(t2, 2);
-    }
-    for (int k = 0, q = 0; t0 < sp.ntasks; ++k, q = q + 1 == kSlots ? 0 : q + 1) {
+    int t2 = t1 < sp.ntasks ? next_tile() : sp.ntasks;
+    if (t2 < sp.ntasks) issue_p1(t2, 2);
+    for (int q = 0; t0 < sp.ntasks; q = q + 1 == kSlots ? 0 : q + 1) {
       issue_p2(t0, q);
-      const int tn = (kSlots > 2 ? t2 : t1) < sp.ntasks ? next_tile() : sp.ntasks;
+      const int tn = t2 < sp.ntasks ? next_tile() : sp.ntasks;
       if (tn < sp.ntasks) issue_p1(tn, q);
       t0 = t1;
-      if (kSlots > 2) {
-        t1 = t2;
-        t2 = tn;
-      } else {
-        t1 = tn;
-      }
+      t1 = t2;
+      t2 = tn;
     }
     // end stage: the descriptor is published through a (16-byte) bulk copy's
     // complete_tx like every data stage
@@ -626,15 +653,17 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
   }
 
   // -------------------------------------------------------------- consumers
-  const uint32_t tmem_lane = tmem_base + ((uint32_t)(32 * warp) << 16);  // this warp's 32 TMEM lanes
+  // warp (wc, wr): warp column wc (240 columns), warp row wr (12 rows) of the
+  // CTA tile; TMEM lane quarter wc, columns 160 wr + 48 slot ..
+  const int wc = warp % kWarpsT, wr = warp / kWarpsT;
+  const uint32_t tmem_w = tmem_base + ((uint32_t)(32 * wc) << 16) + (uint32_t)(wr * kWarpCols);
   const int W = sp.W, H = sp.H;
   for (int s = 0;; ++s) {
     const int b = RRing::buf(s);
 #ifdef SHARP_DIAG_RES
     const long long w0 = clock64();
 #endif
-    if (SHARP_RES_CWAIT_NS) mbar_wait_backoff(ring.full0 + 8u * b, RRing::phase(s), SHARP_RES_CWAIT_NS);
-    else ring.wait_full(s);
+    ring.wait_full(s);
     const int4 d = stage_task[b];
     const int2 aux = stage_aux[b];
 #ifdef SHARP_DIAG_RES
@@ -646,33 +675,34 @@ __global__ void __launch_bounds__(kThreadsT, kResCtasPerSm)
         RD_ADD(14, now - rd_tma[b]);
         RD_ADD(15, now - rd_lut[b]);
         RD_ADD(13, 1);
-
       }
     }
 #endif
     if (d.x == kREnd) break;
-    const int f = d.y, C0w = d.z + warp * kTW, R0 = d.w;
-    const uint32_t tslot = tmem_lane + (uint32_t)((aux.x & 1) * kSlotCols);
-    const uint32_t spe = aux.x == 2 ? sbase + kResPeOff + (uint32_t)(warp * kT * kPeRowBytes + 16 * lane) : 0u;
+    const int f = d.y, C0w = d.z + wc * kTW, R0w = d.w + wr * kT;
+    const uint32_t tslot = tmem_w + (uint32_t)(aux.x * kSlotCols);
     if (d.x == kRP1) {
-      const float acc = C0w < W ? p1_tile(ring.stage(s), warp, W, sp.rmax1, C0w, R0, lane, tslot, spe) : 0.0f;
+      const float acc = C0w < W ? p1_tile(lane_row_r(ring.stage(s), wc, lane, 3), wr * kT + 3, W, sp.rmax1, C0w, R0w,
+                                          lane, tslot)
+                                : 0.0f;
       // Reduction (sec. V-C): warp REDUX, one u64 atomic per warp adding the
       // arrival and the partial in one word (the table builders wait on it).
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
       if (lane == 0) atomicAdd(&sp.acc[f], (1ull << kAccShift) + (unsigned long long)ws);
-    } else if (C0w < W) {
+    } else if (C0w < W && R0w < H) {
       // LDS address of entry k = pEdge/2: f32 bits of (2^21 + pEdge) + lut_q
       // (warp-uniform by the vote: folded into LDS [R + UR]).
       const uint32_t lut_q =
           lutbase + (__any_sync(0xffffffffu, aux.y) ? (uint32_t)kLutBytes : 0u) - 0x4A000000u;
-      p2_tile(ring.stage(s), lut_q, tslot, spe, sp.out + (size_t)f * sp.out_fs + (size_t)R0 * sp.out_pitch,
-              (uint32_t)sp.out_pitch, W, H, C0w, R0, warp, lane);
+      p2_tile(lane_row_r(ring.stage(s), wc, lane, 0), wr * kT, lut_q, tslot,
+              sp.out + (size_t)f * sp.out_fs + (size_t)R0w * sp.out_pitch, (uint32_t)sp.out_pitch, W, H, C0w, R0w,
+              lane);
     }
     ring.release(s, lane);
   }
   // teardown: every consumer warp's TMEM accesses are complete
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-  asm volatile("bar.sync 1, %0;" ::"n"(kWarpsT * 32) : "memory");
+  asm volatile("bar.sync 1, %0;" ::"n"(kCompute * 32) : "memory");
   if (warp == 0) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(kTmemCols));
@@ -694,7 +724,7 @@ int res_grid() { return g_res_grid[cur_dev()].load(std::memory_order_relaxed); }
 
 bool res_supported(int W, int H, int n) {
   (void)n;
-  const long long per_frame = (long long)((W + kCtaCols - 1) / kCtaCols) * ((H + kT - 1) / kT);
+  const long long per_frame = (long long)((W + kCtaCols - 1) / kCtaCols) * ((H + kTileRows - 1) / kTileRows);
   const int grid = res_grid();
   return grid > 0 && per_frame <= 2ll * grid;
 }
@@ -706,15 +736,15 @@ cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p
   CUtensorMap m1A, m1B, m2A, m2B;
   if (!make_map(&m1A, a.in, a.n, W, H, ip, ifs, kPitch, kRowsP1) ||
       !make_map(&m1B, a.in, a.n, W, H, ip, ifs, kPitchB, kRowsP1) ||
-      !make_map(&m2A, a.in, a.n, W, H, ip, ifs, kPitch, kRows2) ||
-      !make_map(&m2B, a.in, a.n, W, H, ip, ifs, kPitchB, kRows2))
+      !make_map(&m2A, a.in, a.n, W, H, ip, ifs, kPitch, kRowsStage) ||
+      !make_map(&m2B, a.in, a.n, W, H, ip, ifs, kPitchB, kRowsStage))
     return cudaErrorInvalidValue;
   ResParams sp;
   sp.W = W;
   sp.H = H;
   sp.n = a.n;
   sp.tiles_x = (W + kCtaCols - 1) / kCtaCols;
-  sp.per_frame = sp.tiles_x * ((H + kT - 1) / kT);
+  sp.per_frame = sp.tiles_x * ((H + kTileRows - 1) / kTileRows);
   sp.ntasks = a.n * sp.per_frame;
   sp.rmax1 = H - 2;
   sp.prm = p;
@@ -731,9 +761,12 @@ cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p
   int grid = std::min(res_grid(), sp.ntasks);
   if (a.grid_cap > 0) grid = std::min(grid, a.grid_cap);
   if (sp.per_frame > 2 * grid) return cudaErrorNotSupported;  // the no-deadlock bound (header comment)
-  sp.pad = sp.per_frame <= grid ? 0 : 2 * grid;
+  // (dense order: with three pEdge slots a frame may span three positions of
+  // a CTA -- P2 of position k follows P1 of position k+2 -- so up to 2 x grid
+  // tiles need no padding)
+  sp.pad = 0;
   sp.npos = sp.pad ? a.n * sp.pad : sp.ntasks;
-  res_kernel<<<grid, kThreadsT, kResSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
+  res_kernel<<<grid, kThreadsR, kResSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
   return cudaGetLastError();
 }
 
@@ -747,9 +780,9 @@ extern "C" int sharp_debug_res_occ(int *out) {
   out[2] = fa.maxDynamicSharedSizeBytes;
   out[3] = kResSmem;
   int r = -1;
-  out[4] = (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, res_kernel, kThreadsT, kResSmem);
+  out[4] = (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, res_kernel, kThreadsR, kResSmem);
   out[5] = r;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, res_kernel, kThreadsT, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, res_kernel, kThreadsR, 0);
   out[6] = r;
   out[7] = fa.maxThreadsPerBlock;
   return 0;
@@ -779,15 +812,15 @@ cudaError_t preload_res() {
   cudaFuncAttributes fa;
   if ((e = cudaGetDeviceProperties(&pr, dev)) != cudaSuccess) return e;
   if ((e = cudaFuncGetAttributes(&fa, res_kernel)) != cudaSuccess) return e;
-  const int warps = kThreadsT / 32;
+  const int warps = kThreadsR / 32;
   const int regs_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
   const int by_regs = pr.regsPerMultiprocessor / (regs_warp * warps);
   const int by_smem =
       (int)(pr.sharedMemPerMultiprocessor / (kResSmem + fa.sharedSizeBytes + pr.reservedSharedMemPerBlock));
-  const int by_threads = pr.maxThreadsPerMultiProcessor / kThreadsT;
+  const int by_threads = pr.maxThreadsPerMultiProcessor / kThreadsR;
   int res = std::min(std::min(by_regs, by_smem), std::min(by_threads, pr.maxBlocksPerMultiProcessor));
   res = std::min(res, (int)(512 / kTmemCols));
-  res = std::min(res, kResCtasPerSm);
+  res = std::min(res, 1);  // one CTA per SM (it allocates all 512 TMEM columns)
   const int sms = pr.multiProcessorCount;
   g_res_grid[dev].store(std::max(1, res) * (sms > 0 ? sms : 148));
   return cudaSuccess;

@@ -22,6 +22,7 @@ buf = (ctypes.c_ulonglong * 16)()
 imgs = torch.from_numpy(synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 5)).cuda()
 out = torch.empty_like(imgs)
 sh = Sharpener()
+sh.set_path(4)  # SHARP_PATH_RES
 for _ in range(2):
     sh.enqueue_batch(imgs, out, (1.0, 0.5, 0.5, 2.0))
 torch.cuda.synchronize()
