@@ -51,37 +51,38 @@ namespace sharp {
 namespace {
 using namespace dev;
 
-constexpr int kT = kTH;                 // rows per warp tile (pass 1 and pass 2)
-constexpr int kWR = 3;                  // warp rows per CTA tile
-constexpr int kTileRows = kWR * kT;     // 36 rows per CTA tile
-constexpr int kCompute = kWarpsT * kWR;  // 12 compute warps (4 columns x 3 rows of warp tiles)
-constexpr int kThreadsR = 32 * (kCompute + 2);  // + producer warp + table warp: ONE CTA per SM
-constexpr int kRowsStage = kTileRows + 8;       // stage rows: image rows R0-4 .. R0+39
-constexpr int kRowsP1 = kTileRows + 2;          // pass-1 boxes: rows R0-1 .. R0+36 (stage rows 3 ..)
-constexpr int kSlotR = kPitch * kRowsStage;     // region A of one warp column
-constexpr int kRegBR = kWarpsT * kSlotR;        // region B (the last warp column's right halo)
+constexpr int kT = kTH;                 // rows per tile (pass 1 and pass 2)
+constexpr int kPipes = 3;               // independent pipelines per CTA (each: 4 compute warps + a producer)
+constexpr int kCompute = kWarpsT * kPipes;       // 12 compute warps
+constexpr int kThreadsR = 32 * (kCompute + kPipes + 1);  // + 3 producers + 1 table warp: ONE CTA per SM
+constexpr int kRowsStage = kT + 8;               // stage rows: image rows R0-4 .. R0+15
+constexpr int kRowsP1 = kT + 2;                  // pass-1 boxes: rows R0-1 .. R0+12 (at stage row 3)
+constexpr int kSlotR = kPitch * kRowsStage;      // region A of one warp column
+constexpr int kRegBR = kWarpsT * kSlotR;         // region B (the last warp column's right halo)
 #ifndef SHARP_RES_STAGES
 #define SHARP_RES_STAGES 3
 #endif
-constexpr int kResStages = SHARP_RES_STAGES;    // smem ring depth (P1 / P2 stages)
+constexpr int kResStages = SHARP_RES_STAGES;     // smem ring depth per pipeline
 constexpr int kResStage = (kRegBR + kPitchB * kRowsStage + 127) / 128 * 128;
 constexpr int kLutBufs = 2;
-constexpr int kResLutOff = kResStages * kResStage;     // LUT buffers after the stages
-constexpr int kResDummy = kResLutOff + kLutBufs * kLutBytes;  // end stage's 16-B copy target
-constexpr int kResBarOff = kResDummy + 16;
-constexpr int kResSmem = kResBarOff + 16 * kResStages;
-// TMEM: all 512 columns (one CTA per SM); warp w uses lane quarter w % 4
-// (the hardware's mapping) and columns 160 (w / 4) ..: three slots of 48
-// columns, slot q of a tile at +48 q, pEdge row j of the warp tile at +4 j.
+constexpr int kPipeLutOff = kResStages * kResStage;          // per pipeline: stages, LUT buffers, 16-B dummy
+constexpr int kPipeDummy = kPipeLutOff + kLutBufs * kLutBytes;
+constexpr int kPipeBytes = (kPipeDummy + 16 + 127) / 128 * 128;
+constexpr int kResBarOff = kPipes * kPipeBytes;               // then full + empty barriers of every pipeline
+constexpr int kResSmem = kResBarOff + kPipes * 16 * kResStages;
+// TMEM: all 512 columns (one CTA per SM); compute warp w (pipeline w / 4)
+// uses lane quarter w % 4 (the hardware's mapping) and columns 160 (w / 4)
+// ..: three slots of 48 columns, slot q of a tile at +48 q, pEdge row j of
+// the tile at +4 j.
 constexpr uint32_t kTmemCols = 512;
 constexpr int kWarpCols = 160;
 constexpr int kSlots = 3;
 constexpr int kSlotCols = 4 * kT;
-static_assert(kSlots * kSlotCols <= kWarpCols && kWR * kWarpCols <= (int)kTmemCols, "TMEM slots");
+static_assert(kSlots * kSlotCols <= kWarpCols && kPipes * kWarpCols <= (int)kTmemCols, "TMEM slots");
 constexpr int kChunk = 16;                  // table entries per chunk: lanes 0-15 adj, 16-31 osc
 constexpr int kChunks = kLut2 / kChunk;     // 48
 constexpr int kAccShift = 40;
-static_assert(kResStage % 128 == 0 && kResLutOff % 128 == 0 && (3 * kPitch) % 128 == 0, "TMA smem destinations");
+static_assert(kResStage % 128 == 0 && kPipeLutOff % 128 == 0 && (3 * kPitch) % 128 == 0, "TMA smem destinations");
 static_assert(kResSmem <= 227 * 1024, "one CTA per SM");
 
 using RRing = RingT<kResStages, kResStage>;
@@ -370,7 +371,7 @@ __device__ __forceinline__ void build_chunk(const ResParams &sp, int f, int c, u
 // builds one chunk if the frame's pass 1 is complete and a chunk is left
 // (returns 0), else returns -1 (nothing to do now).  Warp-uniform.
 __device__ __forceinline__ int table_step(const ResParams &sp, int f, int lane) {
-  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kCompute) << kAccShift;
+  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kWarpsT) << kAccShift;
   unsigned done = 0;
   unsigned long long a = 0;
   if (lane == 0) {
@@ -403,11 +404,18 @@ __device__ __forceinline__ void acquire_table(const ResParams &sp, int f, int la
 
 // Returns once frame f's table is complete; meanwhile builds chunks of it
 // (once its pass 1 is complete).  Warp-uniform (all 32 producer lanes).
+// A frame whose table never completes (a bug, or a broken no-deadlock
+// condition) must not hang the device: the dependency waits trap after 10 s.
+__device__ __forceinline__ void watchdog(unsigned long long t0) {
+  if (gtime_ns() - t0 > 10000000000ull) __trap();
+}
+
 __device__ __forceinline__ void ensure_table(const ResParams &sp, int f, int lane) {
+  const unsigned long long wd0 = gtime_ns();
 #ifdef SHARP_DIAG_NO_TABLE_WAIT  // timing experiment only: wrong output
   return;
 #endif
-  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kCompute) << kAccShift;
+  const unsigned long long arrivals = (unsigned long long)(sp.per_frame * kWarpsT) << kAccShift;
 #ifdef SHARP_DIAG_RES
   long long t_first_complete = 0, t_enter = clock64();
   int iters = 0;
@@ -439,6 +447,7 @@ __device__ __forceinline__ void ensure_table(const ResParams &sp, int f, int lan
       }
     }
     __nanosleep(SHARP_RES_HELP_NS);
+    watchdog(wd0);
   }
 #ifdef SHARP_DIAG_RES
   if (lane == 0) {
@@ -459,13 +468,17 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     res_kernel(const __grid_constant__ CUtensorMap map1A, const __grid_constant__ CUtensorMap map1B,
                const __grid_constant__ CUtensorMap map2A, const __grid_constant__ CUtensorMap map2B, ResParams sp) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ int4 stage_task[kResStages];  // {type, frame, C0, R0}
-  __shared__ int2 stage_aux[kResStages];   // {TMEM slot, LUT buffer}
+  __shared__ int4 stage_task[kPipes][kResStages];  // {type, frame, C0, R0}
+  __shared__ int2 stage_aux[kPipes][kResStages];   // {TMEM slot, LUT buffer}
   __shared__ uint32_t tmem_base;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t sbase = smem_u32(smem);
-  const RRing ring{sbase, sbase + kResBarOff, sbase + kResBarOff + 8 * kResStages};
-  const uint32_t lutbase = sbase + kResLutOff;
+  // pipeline of this warp: compute warps 4p..4p+3, producer warp kCompute + p
+  const int pipe = warp < kCompute ? warp / kWarpsT : (warp < kCompute + kPipes ? warp - kCompute : 0);
+  const uint32_t pbase = sbase + (uint32_t)(pipe * kPipeBytes);
+  const uint32_t bars = sbase + kResBarOff + (uint32_t)(pipe * 16 * kResStages);
+  const RRing ring{pbase, bars, bars + 8 * kResStages};
+  const uint32_t lutbase = pbase + kPipeLutOff;
 
   if (warp == 0) {  // TMEM for the pEdge slots (warp 0 allocates and frees)
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)),
@@ -473,9 +486,10 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kResStages; ++i) {
-      mbar_init(ring.full0 + 8 * i, 1);
-      mbar_init(ring.empty0 + 8 * i, kCompute);
+    for (int i = 0; i < kPipes * kResStages; ++i) {
+      const uint32_t b0 = sbase + kResBarOff + (uint32_t)((i / kResStages) * 16 * kResStages);
+      mbar_init(b0 + 8 * (i % kResStages), 1);
+      mbar_init(b0 + 8 * kResStages + 8 * (i % kResStages), kWarpsT);
     }
     fence_barrier_init();
   }
@@ -483,7 +497,7 @@ __global__ void __launch_bounds__(kThreadsR, 1)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 
-  if (warp == kCompute + 1) {
+  if (warp == kCompute + kPipes) {
     // --------------------------------------------------------- table warp
     // Builds chunks of every frame's table as soon as the frame's pass 1 is
     // complete (all SMs' table warps in parallel: a frame's 48 chunks take
@@ -491,7 +505,9 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     // pass-2 tile, so their build must not wait for the producers that need
     // them (measured: 5 us per frame when only the waiting producers built).
     for (int f = 0; f < sp.n; ++f) {
+      const unsigned long long wd0 = gtime_ns();
       for (;;) {
+        watchdog(wd0);
         const int st = table_step(sp, f, lane);
         if (st == 1) break;                                      // complete
         if (st < 0) {
@@ -504,19 +520,22 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     }
     return;
   }
-  if (warp == kCompute) {
+  if (warp >= kCompute) {
     // ------------------------------------------------------------ producer
+    // (one per pipeline: a "virtual CTA" v = kPipes * blockIdx.x + pipe of a
+    // grid of kPipes * gridDim.x, with its own stages and LUT buffers)
     const uint64_t pol_keep = policy_evict_last(), pol_drop = policy_evict_first();
     int s = 0;                                        // stages filled
     // per LUT buffer b (scalars, not arrays: no local memory): the last stage
     // that used it and the frame whose table it holds
     int lut_last0 = -kResStages, lut_last1 = -kResStages, lut_frame0 = -1, lut_frame1 = -1;
     int lut_prev = 1;                                 // buffer of the previous pass-2 tile
-    int pos = blockIdx.x;
-    auto next_tile = [&]() -> int {  // this CTA's next tile (static schedule), or ntasks
+    const int vgrid = kPipes * gridDim.x;
+    int pos = kPipes * blockIdx.x + pipe;
+    auto next_tile = [&]() -> int {  // this pipeline's next tile (static schedule), or ntasks
       while (pos < sp.npos) {
         const int p = pos;
-        pos += gridDim.x;
+        pos += vgrid;
         if (!sp.pad) return p;
         const int f = p / sp.pad, i = p - f * sp.pad;
         if (i < sp.per_frame) return f * sp.per_frame + i;
@@ -538,7 +557,7 @@ __global__ void __launch_bounds__(kThreadsR, 1)
       f = t / sp.per_frame;
       const int i = t - f * sp.per_frame, ty = i / sp.tiles_x;
       C0 = (i - ty * sp.tiles_x) * kCtaCols;
-      R0 = ty * kTileRows;
+      R0 = ty * kT;
       nw = 0;
 #pragma unroll
       for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < sp.W);
@@ -549,8 +568,8 @@ __global__ void __launch_bounds__(kThreadsR, 1)
       const int b = begin_stage();
       if (lane == 0) {
         const uint32_t full = ring.full0 + 8u * b, st = ring.stage(s);
-        stage_task[b] = make_int4(kRP1, f, C0, R0);
-        stage_aux[b] = make_int2(q, 0);
+        stage_task[pipe][b] = make_int4(kRP1, f, C0, R0);
+        stage_aux[pipe][b] = make_int2(q, 0);
         mbar_expect_tx(full, tile_bytes_r(nw, kRowsP1));
         tma_tiles_r(st, &map1A, &map1B, C0, nw, 3, R0 - 1, f, full, pol_keep);  // stage row 3 = image row R0-1
       }
@@ -576,7 +595,9 @@ __global__ void __launch_bounds__(kThreadsR, 1)
 #endif
       if (s >= kResStages) {
         const uint32_t eb = ring.empty0 + 8u * RRing::buf(s), par = RRing::phase(s) ^ 1u;
+        const unsigned long long wd0 = gtime_ns();
         while (!ready && !mbar_test(eb, par)) {
+          watchdog(wd0);
           const int st = table_step(sp, f, lane);
           if (st == 1) {
             acquire_table(sp, f, lane, 0);
@@ -591,8 +612,8 @@ __global__ void __launch_bounds__(kThreadsR, 1)
       const uint32_t lut_dst = lutbase + (uint32_t)(lb * kLutBytes);
       const float2 *lut_src = sp.luts + (size_t)f * kLutSize;
       if (lane == 0) {
-        stage_task[b] = make_int4(kRP2, f, C0, R0);
-        stage_aux[b] = make_int2(q, lb);
+        stage_task[pipe][b] = make_int4(kRP2, f, C0, R0);
+        stage_aux[pipe][b] = make_int2(q, lb);
         const int tl = lb ? lut_last1 : lut_last0;
         if (copy && tl > s - kResStages) mbar_wait(ring.empty0 + 8u * RRing::buf(tl), RRing::phase(tl));
         mbar_expect_tx(full, tile_bytes_r(nw, kRowsStage) + (copy ? (uint32_t)kLutBytes : 0u));
@@ -645,18 +666,18 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     const int b = begin_stage();
     if (lane == 0) {
       const uint32_t full = ring.full0 + 8u * b;
-      stage_task[b] = make_int4(kREnd, 0, 0, 0);
+      stage_task[pipe][b] = make_int4(kREnd, 0, 0, 0);
       mbar_expect_tx(full, 16u);
-      bulk_copy(sbase + kResDummy, sp.luts, 16u, full);
+      bulk_copy(pbase + kPipeDummy, sp.luts, 16u, full);
     }
     return;
   }
 
   // -------------------------------------------------------------- consumers
-  // warp (wc, wr): warp column wc (240 columns), warp row wr (12 rows) of the
-  // CTA tile; TMEM lane quarter wc, columns 160 wr + 48 slot ..
-  const int wc = warp % kWarpsT, wr = warp / kWarpsT;
-  const uint32_t tmem_w = tmem_base + ((uint32_t)(32 * wc) << 16) + (uint32_t)(wr * kWarpCols);
+  // warp wc (240 columns) of its pipeline's tiles; TMEM lane quarter wc,
+  // columns 160 pipe + 48 slot ..
+  const int wc = warp % kWarpsT;
+  const uint32_t tmem_w = tmem_base + ((uint32_t)(32 * wc) << 16) + (uint32_t)(pipe * kWarpCols);
   const int W = sp.W, H = sp.H;
   for (int s = 0;; ++s) {
     const int b = RRing::buf(s);
@@ -664,8 +685,8 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     const long long w0 = clock64();
 #endif
     ring.wait_full(s);
-    const int4 d = stage_task[b];
-    const int2 aux = stage_aux[b];
+    const int4 d = stage_task[pipe][b];
+    const int2 aux = stage_aux[pipe][b];
 #ifdef SHARP_DIAG_RES
     if (lane == 0) {
       const long long now = clock64();
@@ -679,12 +700,11 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     }
 #endif
     if (d.x == kREnd) break;
-    const int f = d.y, C0w = d.z + wc * kTW, R0w = d.w + wr * kT;
+    const int f = d.y, C0w = d.z + wc * kTW, R0w = d.w;
     const uint32_t tslot = tmem_w + (uint32_t)(aux.x * kSlotCols);
     if (d.x == kRP1) {
-      const float acc = C0w < W ? p1_tile(lane_row_r(ring.stage(s), wc, lane, 3), wr * kT + 3, W, sp.rmax1, C0w, R0w,
-                                          lane, tslot)
-                                : 0.0f;
+      const float acc =
+          C0w < W ? p1_tile(lane_row_r(ring.stage(s), wc, lane, 3), 3, W, sp.rmax1, C0w, R0w, lane, tslot) : 0.0f;
       // Reduction (sec. V-C): warp REDUX, one u64 atomic per warp adding the
       // arrival and the partial in one word (the table builders wait on it).
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
@@ -694,7 +714,7 @@ __global__ void __launch_bounds__(kThreadsR, 1)
       // (warp-uniform by the vote: folded into LDS [R + UR]).
       const uint32_t lut_q =
           lutbase + (__any_sync(0xffffffffu, aux.y) ? (uint32_t)kLutBytes : 0u) - 0x4A000000u;
-      p2_tile(lane_row_r(ring.stage(s), wc, lane, 0), wr * kT, lut_q, tslot,
+      p2_tile(lane_row_r(ring.stage(s), wc, lane, 0), 0, lut_q, tslot,
               sp.out + (size_t)f * sp.out_fs + (size_t)R0w * sp.out_pitch, (uint32_t)sp.out_pitch, W, H, C0w, R0w,
               lane);
     }
@@ -724,9 +744,9 @@ int res_grid() { return g_res_grid[cur_dev()].load(std::memory_order_relaxed); }
 
 bool res_supported(int W, int H, int n) {
   (void)n;
-  const long long per_frame = (long long)((W + kCtaCols - 1) / kCtaCols) * ((H + kTileRows - 1) / kTileRows);
+  const long long per_frame = (long long)((W + kCtaCols - 1) / kCtaCols) * ((H + kT - 1) / kT);
   const int grid = res_grid();
-  return grid > 0 && per_frame <= 2ll * grid;
+  return grid > 0 && per_frame <= 2ll * kPipes * grid;
 }
 
 cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p, cudaStream_t stream) {
@@ -744,7 +764,7 @@ cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p
   sp.H = H;
   sp.n = a.n;
   sp.tiles_x = (W + kCtaCols - 1) / kCtaCols;
-  sp.per_frame = sp.tiles_x * ((H + kTileRows - 1) / kTileRows);
+  sp.per_frame = sp.tiles_x * ((H + kT - 1) / kT);
   sp.ntasks = a.n * sp.per_frame;
   sp.rmax1 = H - 2;
   sp.prm = p;
@@ -758,9 +778,9 @@ cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p
   sp.out = a.out;
   sp.out_pitch = a.out_pitch ? a.out_pitch : (size_t)W;
   sp.out_fs = a.out_fs ? a.out_fs : sp.out_pitch * (size_t)H;
-  int grid = std::min(res_grid(), sp.ntasks);
+  int grid = std::min(res_grid(), (sp.ntasks + kPipes - 1) / kPipes);
   if (a.grid_cap > 0) grid = std::min(grid, a.grid_cap);
-  if (sp.per_frame > 2 * grid) return cudaErrorNotSupported;  // the no-deadlock bound (header comment)
+  if (sp.per_frame > 2 * kPipes * grid) return cudaErrorNotSupported;  // the no-deadlock bound (header comment)
   // (dense order: with three pEdge slots a frame may span three positions of
   // a CTA -- P2 of position k follows P1 of position k+2 -- so up to 2 x grid
   // tiles need no padding)
