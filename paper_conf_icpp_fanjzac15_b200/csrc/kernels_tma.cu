@@ -493,6 +493,24 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           const int tl = lut_last[j & 1];
           if (k == 0 && tl > s - kStages) mbar_wait(ring.empty0 + 8u * Ring::buf(tl), Ring::phase(tl));
           mbar_expect_tx(full, tile_bytes(nw, kRows2) + lut_bytes);
+#ifndef SHARP_OLD_LUT_FENCE
+          // The frame's LUT (its LUT tasks were grabbed rounds earlier) is
+          // normally complete: then the table copy goes out first.  Acquire
+          // LOADS, not fence.acq_rel: a fence after this thread's tile loads
+          // also waits for them (measured on the resident kernel: ~2 us).
+          const unsigned want = (unsigned)(kLutTasks * kWarpsT);
+          const bool lut_now = lut_bytes && ld_acquire(&sp.lut_done[d.y]) >= want;
+          if (lut_now) {
+            fence_proxy_async_global();
+            bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
+          }
+          tma_tiles(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
+          if (lut_bytes && !lut_now) {
+            while (ld_acquire(&sp.lut_done[d.y]) < want) __nanosleep(kPollNs);
+            fence_proxy_async_global();
+            bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
+          }
+#else
           tma_tiles(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
           if (lut_bytes) {
             // the frame's LUT tasks (grabbed earlier) have finished
@@ -502,6 +520,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           }
           if (lut_bytes)
             bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
+#endif
         } else {
           stage_task[b] = d;
           if (d.x == kLut) stage_sum[b] = S & ((1ull << kAccShift) - 1);
