@@ -65,7 +65,28 @@ typedef struct {
   int max_frames;
   int streams;            /* transfer pipeline depth for host buffers; 0 -> 3    */
   int chunk_frames;       /* frames per pass-1/pass-2 chunk; 0 -> automatic      */
+  /* Several devices in ONE context.  num_devices
+   * 0 or 1: the single device `device`.  num_devices G > 1: G devices
+   * (device_ids[0..G-1], NULL -> 0..G-1; an ordinal may repeat, e.g. {0, 0}
+   * to exercise the sharded paths on one GPU); the context keeps one
+   * single-device context per entry and shards the work:
+   *   SHARP_SHARD_FRAMES  sharp_run_batch splits the frames into G contiguous
+   *                       ranges, one per device, run concurrently (frames
+   *                       are independent: no data exchange);
+   *   SHARP_SHARD_ROWS    sharp_run splits the image into G row bands (the
+   *                       h/4 block rows split evenly, sharp_band_halo rows
+   *                       of halo), sums the G partial pEdge sums (the L174
+   *                       mean) and sharpens the bands -- bit-identical to
+   *                       the single-device result;
+   *   SHARP_SHARD_AUTO    frames for batches of >= 2 frames, rows for one image.
+   * Multi-device contexts take HOST buffers in sharp_run / sharp_run_batch
+   * (device-resident bands: sharp_run_bands); the other entry points return
+   * SHARP_EUNSUPPORTED on them.  Ignored when num_devices <= 1. */
+  int num_devices;
+  const int *device_ids;  /* copied at sharp_create */
+  int shard;              /* SHARP_SHARD_* */
 } sharp_config;
+enum { SHARP_SHARD_AUTO = 0, SHARP_SHARD_NONE = 1, SHARP_SHARD_ROWS = 2, SHARP_SHARD_FRAMES = 3 };
 
 typedef struct {
   uint64_t edge_sum;  /* S = sum of pEdge over the image (frame 0 of a batch)    */
@@ -214,6 +235,21 @@ int sharp_band_edge_sum(sharp_ctx *ctx, const uint8_t *band, int w, int h, int r
                         uint64_t *d_partial);
 int sharp_band_sharpen(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
                        const uint64_t *d_total, const sharp_params *params, uint8_t *out);
+
+/* ---- Device-resident row bands over the devices of a multi-device context
+ * (SURVEY.md sec. 8(b) / 8(e) 2).  bands[g] / outs[g]: DEVICE pointers on
+ * device_ids[g] holding rows [row0_g, row1_g) of the w x h image (dense, pitch
+ * w), the partition of sharp_band_rows (the h/4 block rows split as evenly as
+ * possible, the first (h/4) % G bands one block row longer).  The library
+ * copies each band with its 4-row halos (the neighbours' edge rows, peer
+ * copies) into its own scratch, sums the bands' partial pEdge sums (L174:
+ * one global mean) and writes outs[g] = rows [row0_g, row1_g) of the result,
+ * bit-identical to sharp_run on the whole image.  Synchronous.  A
+ * single-device context takes G = 1 (bands[0] = the whole image).
+ * Requirements as for sharp_band_edge_sum (w % 16 == 0, w * h < 2^29). */
+int sharp_band_rows(int h, int n_bands, int band, int *row0, int *row1);
+int sharp_run_bands(sharp_ctx *ctx, const uint8_t *const *bands, int w, int h, const sharp_params *params,
+                    uint8_t *const *outs);
 
 /* ---- Fused peer-memory band exchange (
  * DESIGN.md sec. 9): the same two couplings as above -- 4 halo rows per side

@@ -35,7 +35,15 @@ class SharpParams(ctypes.Structure):
 
 class SharpConfig(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("max_width", ctypes.c_int), ("max_height", ctypes.c_int),
-                ("max_frames", ctypes.c_int), ("streams", ctypes.c_int), ("chunk_frames", ctypes.c_int)]
+                ("max_frames", ctypes.c_int), ("streams", ctypes.c_int), ("chunk_frames", ctypes.c_int),
+                ("num_devices", ctypes.c_int), ("device_ids", ctypes.POINTER(ctypes.c_int)), ("shard", ctypes.c_int)]
+
+
+# multi-device sharding (sharp_config.shard, include/sharp.h)
+SHARP_SHARD_AUTO = 0
+SHARP_SHARD_NONE = 1
+SHARP_SHARD_ROWS = 2
+SHARP_SHARD_FRAMES = 3
 
 
 class SharpStats(ctypes.Structure):
@@ -102,6 +110,8 @@ _SIGS = {
                              ctypes.POINTER(SharpParams), _P, _I], _I),
     "sharp_run_ex": ([_P, _P, ctypes.POINTER(SharpLayout), _I, _I, _I, _I, ctypes.POINTER(SharpParams), _I, _P,
                       ctypes.POINTER(SharpLayout)], _I),
+    "sharp_band_rows": ([_I, _I, _I, ctypes.POINTER(_I), ctypes.POINTER(_I)], _I),
+    "sharp_run_bands": ([_P, ctypes.POINTER(_P), _I, _I, ctypes.POINTER(SharpParams), ctypes.POINTER(_P)], _I),
 }
 
 _lib = None
@@ -169,9 +179,16 @@ def _check(rc, ctx=None):
 # ---------------------------------------------------------------- C-ABI names
 def sharp_create(cfg=None):
     """-> opaque context handle (int).  cfg: SharpConfig or dict or None."""
+    keep = None
     if isinstance(cfg, dict):
         c = SharpConfig(device=-1)
         for k, v in cfg.items():
+            if k == "device_ids":
+                if v:
+                    keep = (ctypes.c_int * len(v))(*[int(x) for x in v])
+                    c.device_ids = keep
+                    c.num_devices = len(v)
+                continue
             setattr(c, k, int(v))
         cfg = c
     h = _P()
@@ -183,6 +200,22 @@ def sharp_create(cfg=None):
 
 def sharp_destroy(ctx):
     lib().sharp_destroy(ctx)
+
+
+def sharp_band_rows(h, n_bands, band):
+    """Rows [row0, row1) of band `band` of `n_bands` (the h/4 block rows split evenly)."""
+    a, b = _I(), _I()
+    rc = lib().sharp_band_rows(h, n_bands, band, ctypes.byref(a), ctypes.byref(b))
+    if rc != SHARP_OK:
+        raise SharpError(rc, f"sharp_band_rows: {sharp_strerror(rc)}")
+    return a.value, b.value
+
+
+def sharp_run_bands(ctx, bands, w, h, params, outs):
+    """bands / outs: per device of the context, device buffers of the band's rows."""
+    arr_in = (_P * len(bands))(*[_addr(b) for b in bands])
+    arr_out = (_P * len(outs))(*[_addr(o) for o in outs])
+    return _check(lib().sharp_run_bands(ctx, arr_in, w, h, _pp(params), arr_out), ctx)
 
 
 def sharp_default_params():
@@ -410,9 +443,14 @@ def sharp_band_sharpen(ctx, band, w, h, row0, row1, d_total, params, out):
 class Sharpener:
     """Owns one sharp_ctx.  Images: uint8 [H, W] (run) or [N, H, W] (run_batch)."""
 
-    def __init__(self, device=-1, streams=0, chunk_frames=0, max_width=0, max_height=0, max_frames=0):
+    def __init__(self, device=-1, streams=0, chunk_frames=0, max_width=0, max_height=0, max_frames=0,
+                 device_ids=None, shard=SHARP_SHARD_AUTO):
+        """device_ids: a list of >= 2 device ordinals makes a multi-device
+        context (sharp_config.num_devices / device_ids / shard)."""
         self.ctx = sharp_create(dict(device=device, streams=streams, chunk_frames=chunk_frames,
-                                     max_width=max_width, max_height=max_height, max_frames=max_frames))
+                                     max_width=max_width, max_height=max_height, max_frames=max_frames,
+                                     device_ids=device_ids if device_ids and len(device_ids) > 1 else None,
+                                     shard=shard))
 
     def close(self):
         if self.ctx:
@@ -460,6 +498,13 @@ class Sharpener:
             out = self._like(img)
         sharp_run(self.ctx, img, W, H, params, out)
         return out
+
+    def run_bands(self, bands, W, H, params=None, outs=None):
+        """Device-resident row bands (one per device of the context)."""
+        if outs is None:
+            outs = [self._like(b) for b in bands]
+        sharp_run_bands(self.ctx, bands, W, H, params, outs)
+        return outs
 
     def run_batch(self, imgs, params=None, out=None):
         N, H, W = self._shape(imgs)

@@ -101,6 +101,19 @@ struct sharp_ctx {
   std::vector<cudaEvent_t> ev_pool;
   bool poisoned = false;
   char err[256] = {0};
+  // Multi-device context (sharp_config.num_devices > 1): one single-device
+  // context per entry of device_ids; this one owns no device resources but
+  // the per-band scratch below (allocated on the sub-contexts' devices).
+  std::vector<sharp_ctx *> sub;
+  int shard = SHARP_SHARD_AUTO;
+  std::vector<std::pair<int, int>> last_split;  // frame ranges of the last sharded batch
+  struct BandBuf {
+    uint8_t *in = nullptr, *out = nullptr;
+    size_t in_cap = 0, out_cap = 0;
+    unsigned long long *part = nullptr, *total = nullptr;  // device u64
+    unsigned long long *h = nullptr;                       // pinned: [0] partial, [1] total
+  };
+  std::vector<BandBuf> bb;
 };
 
 namespace {
@@ -777,9 +790,221 @@ int band_impl(sharp_ctx *ctx, int mode, const uint8_t *band, int w, int h, int r
   return SHARP_OK;
 }
 
+// ---- Multi-device contexts (sharp_config.num_devices > 1).
+bool is_multi(const sharp_ctx *c) { return c && !c->sub.empty(); }
+
+int band_rows_of(int h, int G, int g, int *r0, int *r1) {
+  if (h < 8 || (h & 3) || G < 1 || g < 0 || g >= G || h / 4 < G) return SHARP_EINVAL;
+  const int blocks = h / 4, base = blocks / G, rem = blocks % G;
+  const int start = g * base + std::min(g, rem), count = base + (g < rem ? 1 : 0);
+  *r0 = 4 * start;
+  *r1 = 4 * (start + count);
+  return SHARP_OK;
+}
+
+// Copies a sub-context's failure into the multi context.
+int sub_fail(sharp_ctx *m, int g, int rc) {
+  if (rc != SHARP_OK) snprintf(m->err, sizeof(m->err), "device %d (entry %d): %s", m->sub[g]->device, g, m->sub[g]->err);
+  return rc;
+}
+
+int grow_dev(sharp_ctx *sc, uint8_t **buf, size_t *cap, size_t need) {
+  if (need <= *cap) return SHARP_OK;
+  cudaSetDevice(sc->device);
+  cudaStreamSynchronize(sc->stream);
+  cudaFree(*buf);
+  *buf = nullptr;
+  *cap = 0;
+  if (cudaMalloc(buf, need) != cudaSuccess) {
+    cudaGetLastError();
+    return SHARP_ENOMEM;
+  }
+  *cap = need;
+  return SHARP_OK;
+}
+
+// Frames split over the devices: contiguous ranges, one
+// thread per device (each sub-context is used by one thread), host buffers.
+int multi_frames(sharp_ctx *m, const uint8_t *in, int n, int w, int h, const sharp_params *pp, uint8_t *out) {
+  const int G = (int)m->sub.size();
+  const size_t fb = (size_t)w * h;
+  const auto t0 = std::chrono::steady_clock::now();
+  m->last_split.assign(G, {0, 0});
+  std::vector<int> rc(G, SHARP_OK);
+  std::vector<std::thread> th;
+  for (int g = 0; g < G; ++g) {
+    const int base = n / G, rem = n % G, f0 = g * base + std::min(g, rem), cnt = base + (g < rem ? 1 : 0);
+    m->last_split[g] = {f0, cnt};
+    if (cnt == 0) continue;
+    th.emplace_back([=, &rc] { rc[g] = run_impl(m->sub[g], in + (size_t)f0 * fb, cnt, w, h, pp, out + (size_t)f0 * fb, false); });
+  }
+  for (auto &t : th) t.join();
+  m->stats = sharp_stats{};
+  for (int g = 0; g < G; ++g) {
+    if (rc[g] != SHARP_OK) return sub_fail(m, g, rc[g]);
+    if (m->last_split[g].second == 0) continue;
+    const sharp_stats &st = m->sub[g]->stats;
+    if (m->last_split[g].first == 0) {
+      m->stats.edge_sum = st.edge_sum;
+      m->stats.edge_mean = st.edge_mean;
+    }
+    m->stats.device_ms = std::max(m->stats.device_ms, st.device_ms);
+    m->stats.kernels += st.kernels;
+  }
+  m->stats.frames = n;
+  m->last_frames = n;
+  m->stats.total_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return SHARP_OK;
+}
+
+// One image as G row bands, one per device: each band's rows
+// with their 4-row halos go to the band's device (from the host image, or
+// from the neighbouring device bands by peer copies), pass 1 sums pEdge over
+// the band's rows, the G partials are added (the L174 mean), pass 2 writes
+// the band.  `bands` == nullptr: `img`/`out` are host images; else device
+// bands / outputs per device (sharp_run_bands).
+int multi_rows(sharp_ctx *m, const uint8_t *img, const uint8_t *const *bands, int w, int h, const sharp_params *pp,
+               uint8_t *out, uint8_t *const *outs) {
+  const int G = (int)m->sub.size();
+  const auto t0 = std::chrono::steady_clock::now();
+  if (w < 16 || (w & 15) || h < 8 || (h & 3) || h / 4 < G)
+    return set_err(m, SHARP_EUNSUPPORTED, "%s", "row bands need w % 16 == 0, h % 4 == 0 and >= 4 rows per band");
+  if (pp && !params_ok(*pp)) return set_err(m, SHARP_EINVAL, "%s", "parameter out of range or not finite");
+  std::vector<int> r0(G), r1(G), i0(G), i1(G);
+  for (int g = 0; g < G; ++g) {
+    band_rows_of(h, G, g, &r0[g], &r1[g]);
+    band_halo(h, r0[g], r1[g], &i0[g], &i1[g]);
+  }
+  int rc;
+  for (int g = 0; g < G; ++g) {  // stage each band + halos on its device, pass 1
+    sharp_ctx *sc = m->sub[g];
+    sharp_ctx::BandBuf &b = m->bb[g];
+    const size_t in_bytes = (size_t)(i1[g] - i0[g]) * w, own = (size_t)(r1[g] - r0[g]) * w;
+    if ((rc = grow_dev(sc, &b.in, &b.in_cap, in_bytes)) || (!bands && (rc = grow_dev(sc, &b.out, &b.out_cap, own))))
+      return set_err(m, rc, "%s", "band scratch allocation failed");
+    if (cudaSetDevice(sc->device) != cudaSuccess) return set_err(m, SHARP_ECUDA, "%s", "cudaSetDevice");
+    cudaError_t e = cudaSuccess;
+    if (!bands) {
+      e = cudaMemcpyAsync(b.in, img + (size_t)i0[g] * w, in_bytes, cudaMemcpyHostToDevice, sc->stream);
+    } else {
+      uint8_t *dst = b.in + (size_t)(r0[g] - i0[g]) * w;
+      e = cudaMemcpyAsync(dst, bands[g], own, cudaMemcpyDeviceToDevice, sc->stream);  // own rows
+      if (e == cudaSuccess && g > 0)  // upper halo: the last r0 - i0 rows of band g-1
+        e = cudaMemcpyPeerAsync(b.in, sc->device, bands[g - 1] + (size_t)(i0[g] - r0[g - 1]) * w,
+                                m->sub[g - 1]->device, (size_t)(r0[g] - i0[g]) * w, sc->stream);
+      if (e == cudaSuccess && g + 1 < G)  // lower halo: the first i1 - r1 rows of band g+1
+        e = cudaMemcpyPeerAsync(b.in + (size_t)(r1[g] - i0[g]) * w, sc->device, bands[g + 1],
+                                m->sub[g + 1]->device, (size_t)(i1[g] - r1[g]) * w, sc->stream);
+    }
+    if (e != cudaSuccess) return set_err(m, SHARP_ECUDA, "band copy: %s", cudaGetErrorString(e));
+    if ((rc = band_impl(sc, sharp::kStepPass1, b.in, w, h, r0[g], r1[g], b.part, nullptr, nullptr, nullptr)))
+      return sub_fail(m, g, rc);
+    if ((e = cudaMemcpyAsync(&b.h[0], b.part, 8, cudaMemcpyDeviceToHost, sc->stream)) != cudaSuccess)
+      return set_err(m, SHARP_ECUDA, "partial D2H: %s", cudaGetErrorString(e));
+  }
+  unsigned long long S = 0;  // L174: the sum over the whole image
+  for (int g = 0; g < G; ++g) {
+    cudaSetDevice(m->sub[g]->device);
+    if (cudaStreamSynchronize(m->sub[g]->stream) != cudaSuccess) return set_err(m, SHARP_ECUDA, "%s", "band pass 1");
+    S += m->bb[g].h[0];
+  }
+  for (int g = 0; g < G; ++g) {  // pass 2 with the all-reduced S
+    sharp_ctx *sc = m->sub[g];
+    sharp_ctx::BandBuf &b = m->bb[g];
+    cudaSetDevice(sc->device);
+    b.h[1] = S;
+    cudaError_t e = cudaMemcpyAsync(b.total, &b.h[1], 8, cudaMemcpyHostToDevice, sc->stream);
+    if (e != cudaSuccess) return set_err(m, SHARP_ECUDA, "total H2D: %s", cudaGetErrorString(e));
+    uint8_t *dst = bands ? outs[g] : b.out;
+    if ((rc = band_impl(sc, sharp::kStepPass2, b.in, w, h, r0[g], r1[g], nullptr, b.total, pp, dst)))
+      return sub_fail(m, g, rc);
+    if (!bands && (e = cudaMemcpyAsync(out + (size_t)r0[g] * w, b.out, (size_t)(r1[g] - r0[g]) * w,
+                                       cudaMemcpyDeviceToHost, sc->stream)) != cudaSuccess)
+      return set_err(m, SHARP_ECUDA, "band D2H: %s", cudaGetErrorString(e));
+  }
+  for (int g = 0; g < G; ++g) {
+    cudaSetDevice(m->sub[g]->device);
+    if (cudaStreamSynchronize(m->sub[g]->stream) != cudaSuccess) return set_err(m, SHARP_ECUDA, "%s", "band pass 2");
+  }
+  m->stats = sharp_stats{};
+  m->stats.edge_sum = S;
+  m->stats.edge_mean = (double)S / ((double)w * (double)h);  // R8 (sharp_run: default readings)
+  m->stats.frames = 1;
+  m->stats.kernels = 4 * G;
+  m->last_frames = 1;
+  m->last_split.assign(1, {0, 1});
+  m->stats.total_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  m->stats.device_ms = m->stats.total_ms;
+  return SHARP_OK;
+}
+
+// Host buffers only (the sub-contexts classify the pointers themselves).
+int multi_host_check(sharp_ctx *m, const void *a, const void *b) {
+  cudaPointerAttributes at;
+  for (const void *p : {a, b}) {
+    if (cudaPointerGetAttributes(&at, p) == cudaSuccess &&
+        (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged))
+      return set_err(m, SHARP_EUNSUPPORTED, "%s",
+                     "multi-device contexts take host buffers (device-resident bands: sharp_run_bands)");
+    cudaGetLastError();
+  }
+  return SHARP_OK;
+}
+
+int multi_run(sharp_ctx *m, const uint8_t *in, int n, int w, int h, const sharp_params *pp, uint8_t *out) {
+  if (m->poisoned) return SHARP_ESTATE;
+  if (!in || !out || n < 1) return set_err(m, SHARP_EINVAL, "%s", "NULL image pointer or n < 1");
+  if (w < 8 || h < 8 || (w & 3) || (h & 3))
+    return set_err(m, SHARP_EINVAL, "%s", "width and height must be multiples of 4 and >= 8 (R1)");
+  const size_t bytes = (size_t)n * w * h;
+  if ((uintptr_t)in < (uintptr_t)out + bytes && (uintptr_t)out < (uintptr_t)in + bytes)
+    return set_err(m, SHARP_EINVAL, "%s", "input and output overlap");
+  int rc;
+  if ((rc = multi_host_check(m, in, out))) return rc;
+  const int shard = m->shard == SHARP_SHARD_AUTO ? (n >= 2 ? SHARP_SHARD_FRAMES : SHARP_SHARD_ROWS) : m->shard;
+  if (shard == SHARP_SHARD_NONE) {  // everything on the first device
+    rc = run_impl(m->sub[0], in, n, w, h, pp, out, false);
+    if (rc) return sub_fail(m, 0, rc);
+    m->stats = m->sub[0]->stats;
+    m->last_frames = n;
+    m->last_split.assign(m->sub.size(), {0, 0});
+    m->last_split[0] = {0, n};
+    return SHARP_OK;
+  }
+  if (shard == SHARP_SHARD_ROWS) {
+    if (n != 1) return set_err(m, SHARP_EUNSUPPORTED, "%s", "SHARP_SHARD_ROWS shards one image (n == 1)");
+    return multi_rows(m, in, nullptr, w, h, pp, out, nullptr);
+  }
+  return multi_frames(m, in, n, w, h, pp, out);
+}
+
+#define NOT_MULTI(ctx)                                                                                       \
+  do {                                                                                                       \
+    if (is_multi(ctx))                                                                                       \
+      return set_err(ctx, SHARP_EUNSUPPORTED, "%s",                                                          \
+                     "not available on a multi-device context (sharp_run / sharp_run_batch / sharp_run_bands)"); \
+  } while (0)
+
 }  // namespace
 
 extern "C" {
+
+int sharp_band_rows(int h, int n_bands, int band, int *row0, int *row1) {
+  if (!row0 || !row1) return SHARP_EINVAL;
+  return band_rows_of(h, n_bands, band, row0, row1);
+}
+
+int sharp_run_bands(sharp_ctx *ctx, const uint8_t *const *bands, int w, int h, const sharp_params *params,
+                    uint8_t *const *outs) {
+  if (!ctx) return SHARP_EINVAL;
+  if (ctx->poisoned) return SHARP_ESTATE;
+  if (!bands || !outs) return set_err(ctx, SHARP_EINVAL, "%s", "NULL band array");
+  const int G = is_multi(ctx) ? (int)ctx->sub.size() : 1;
+  for (int g = 0; g < G; ++g)
+    if (!bands[g] || !outs[g]) return set_err(ctx, SHARP_EINVAL, "%s", "NULL band pointer");
+  if (G == 1) return run_impl(ctx, bands[0], 1, w, h, params, outs[0], false);
+  return multi_rows(ctx, nullptr, bands, w, h, params, nullptr, outs);
+}
 
 int sharp_band_halo(int h, int row0, int row1, int *in0, int *in1) {
   if (!in0 || !in1) return SHARP_EINVAL;
@@ -788,12 +1013,14 @@ int sharp_band_halo(int h, int row0, int row1, int *in0, int *in1) {
 
 int sharp_band_edge_sum(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
                         uint64_t *d_partial) {
+  NOT_MULTI(ctx);
   return band_impl(ctx, sharp::kStepPass1, band, w, h, row0, row1, (unsigned long long *)d_partial, nullptr,
                    nullptr, nullptr);
 }
 
 int sharp_band_sharpen(sharp_ctx *ctx, const uint8_t *band, int w, int h, int row0, int row1,
                        const uint64_t *d_total, const sharp_params *params, uint8_t *out) {
+  NOT_MULTI(ctx);
   return band_impl(ctx, sharp::kStepPass2, band, w, h, row0, row1, nullptr,
                    (const unsigned long long *)d_total, params, out);
 }
@@ -813,6 +1040,58 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
   c.device = -1;
   if (cfg) c = *cfg;
   if (c.streams < 0 || c.streams > kMaxSlots || c.chunk_frames < 0 || c.max_frames < 0) return SHARP_EINVAL;
+  if (c.num_devices < 0 || c.num_devices > 64 || c.shard < SHARP_SHARD_AUTO || c.shard > SHARP_SHARD_FRAMES)
+    return SHARP_EINVAL;
+  if (c.num_devices > 1) {  // one single-device context per entry
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
+      cudaGetLastError();
+      return SHARP_ECUDA;
+    }
+    sharp_ctx *m = new (std::nothrow) sharp_ctx();
+    if (!m) return SHARP_ENOMEM;
+    m->shard = c.shard;
+    m->device = c.device_ids ? c.device_ids[0] : 0;
+    m->bb.resize(c.num_devices);
+    for (int g = 0; g < c.num_devices; ++g) {
+      const int dev = c.device_ids ? c.device_ids[g] : g;
+      sharp_config cs = c;
+      cs.num_devices = 0;
+      cs.device_ids = nullptr;
+      cs.device = dev;
+      sharp_ctx *sc = nullptr;
+      int rc = (dev < 0 || dev >= ndev) ? SHARP_EINVAL : sharp_create(&sc, &cs);
+      if (rc == SHARP_OK) {
+        m->sub.push_back(sc);
+        sharp_ctx::BandBuf &b = m->bb[g];
+        cudaSetDevice(dev);
+        if (cudaMalloc(&b.part, 16) != cudaSuccess || cudaHostAlloc(&b.h, 16, cudaHostAllocDefault) != cudaSuccess)
+          rc = SHARP_ENOMEM;
+        else
+          b.total = b.part + 1;
+      }
+      if (rc != SHARP_OK) {
+        cudaGetLastError();
+        sharp_destroy(m);
+        return rc;
+      }
+    }
+    // peer access between neighbouring devices (the band halo copies); the
+    // copies also work without it (staged by the driver)
+    for (int g = 0; g + 1 < c.num_devices; ++g) {
+      const int a = m->sub[g]->device, b = m->sub[g + 1]->device;
+      int ok = 0;
+      if (a != b && cudaDeviceCanAccessPeer(&ok, a, b) == cudaSuccess && ok) {
+        cudaSetDevice(a);
+        cudaDeviceEnablePeerAccess(b, 0);
+        cudaSetDevice(b);
+        cudaDeviceEnablePeerAccess(a, 0);
+      }
+      cudaGetLastError();  // (already enabled is fine)
+    }
+    *out = m;
+    return SHARP_OK;
+  }
   sharp_ctx *ctx = new (std::nothrow) sharp_ctx();
   if (!ctx) return SHARP_ENOMEM;
   int dev = c.device;
@@ -867,6 +1146,20 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
 
 void sharp_destroy(sharp_ctx *ctx) {
   if (!ctx) return;
+  if (!ctx->bb.empty()) {  // multi-device context
+    for (size_t g = 0; g < ctx->bb.size(); ++g) {
+      sharp_ctx::BandBuf &b = ctx->bb[g];
+      if (g < ctx->sub.size()) cudaSetDevice(ctx->sub[g]->device);
+      cudaFree(b.in);
+      cudaFree(b.out);
+      cudaFree(b.part);
+      if (b.h) cudaFreeHost(b.h);
+    }
+    for (sharp_ctx *sc : ctx->sub) sharp_destroy(sc);
+    cudaGetLastError();
+    delete ctx;
+    return;
+  }
   cudaSetDevice(ctx->device);
   if (ctx->stream) cudaStreamSynchronize(ctx->stream);
   for (int i = 0; i < kMaxSlots; ++i) {
@@ -898,6 +1191,7 @@ void sharp_destroy(sharp_ctx *ctx) {
 
 int sharp_set_stream(sharp_ctx *ctx, void *stream) {
   if (!ctx) return SHARP_EINVAL;
+  NOT_MULTI(ctx);
   if (ctx->poisoned) return SHARP_ESTATE;
   cudaStream_t next = stream ? (cudaStream_t)stream : ctx->own_stream;
   if (next != ctx->stream) {
@@ -915,21 +1209,25 @@ int sharp_set_stream(sharp_ctx *ctx, void *stream) {
 }
 
 int sharp_run(sharp_ctx *ctx, const uint8_t *img, int w, int h, const sharp_params *params, uint8_t *out) {
+  if (is_multi(ctx)) return multi_run(ctx, img, 1, w, h, params, out);
   return run_impl(ctx, img, 1, w, h, params, out, false);
 }
 
 int sharp_run_batch(sharp_ctx *ctx, const uint8_t *imgs, int n, int w, int h, const sharp_params *params,
                     uint8_t *outs) {
+  if (is_multi(ctx)) return multi_run(ctx, imgs, n, w, h, params, outs);
   return run_impl(ctx, imgs, n, w, h, params, outs, false);
 }
 
 int sharp_enqueue_batch(sharp_ctx *ctx, const uint8_t *d_imgs, int n, int w, int h, const sharp_params *params,
                         uint8_t *d_outs) {
+  NOT_MULTI(ctx);
   return run_impl(ctx, d_imgs, n, w, h, params, d_outs, true);
 }
 
 int sharp_run_ex(sharp_ctx *ctx, const uint8_t *imgs, const sharp_layout *in_layout, int n, int channels, int w,
                  int h, const sharp_params *params, int flags, uint8_t *outs, const sharp_layout *out_layout) {
+  NOT_MULTI(ctx);
   return run_ex_impl(ctx, imgs, in_layout, n, channels, w, h, params, flags, outs, out_layout);
 }
 
@@ -944,6 +1242,19 @@ int sharp_get_batch_sums(sharp_ctx *ctx, uint64_t *sums, int n) {
   if (ctx->poisoned) return SHARP_ESTATE;
   if (n > ctx->last_frames) return set_err(ctx, SHARP_EINVAL, "%s", "n exceeds the frames of the last call");
   if (n == 0) return SHARP_OK;
+  if (is_multi(ctx)) {  // gathered from the devices' frame ranges
+    if (ctx->last_split.size() == 1) {  // one row-sharded image
+      sums[0] = ctx->stats.edge_sum;
+      return SHARP_OK;
+    }
+    for (size_t g = 0; g < ctx->last_split.size(); ++g) {
+      const int f0 = ctx->last_split[g].first, cnt = std::min(ctx->last_split[g].second, n - f0);
+      if (cnt <= 0) continue;
+      const int rc = sharp_get_batch_sums(ctx->sub[g], sums + f0, cnt);
+      if (rc) return sub_fail(ctx, (int)g, rc);
+    }
+    return SHARP_OK;
+  }
   CK(cudaStreamSynchronize(ctx->stream));
   CK(cudaMemcpy(sums, ctx->sums, (size_t)n * sizeof(uint64_t), cudaMemcpyDeviceToHost));
   return SHARP_OK;
@@ -951,6 +1262,7 @@ int sharp_get_batch_sums(sharp_ctx *ctx, uint64_t *sums, int n) {
 
 int sharp_set_profiling(sharp_ctx *ctx, int enable) {
   if (!ctx) return SHARP_EINVAL;
+  NOT_MULTI(ctx);
   if (ctx->poisoned) return SHARP_ESTATE;
   CK(cudaStreamSynchronize(ctx->stream));
   for (auto &r : ctx->recs) {
@@ -964,6 +1276,7 @@ int sharp_set_profiling(sharp_ctx *ctx, int enable) {
 
 int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t) {
   if (!ctx || !t) return SHARP_EINVAL;
+  NOT_MULTI(ctx);
   if (ctx->poisoned) return SHARP_ESTATE;
   *t = sharp_kernel_times{};
   for (auto &r : ctx->recs) {
@@ -988,6 +1301,7 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t) {
 
 int sharp_get_stage_times(sharp_ctx *ctx, float *ms, int n) {
   if (!ctx || !ms || n < SHARP_NUM_STAGES) return SHARP_EINVAL;
+  NOT_MULTI(ctx);
   if (ctx->poisoned) return SHARP_ESTATE;
   for (int i = 0; i < SHARP_NUM_STAGES; ++i) ms[i] = 0.0f;
   for (auto &r : ctx->recs) {
@@ -1031,6 +1345,7 @@ void sharp_p2p_window_destroy(void *d_window) {
 
 int sharp_band_p2p_halo(sharp_ctx *ctx, uint8_t *self_window, int w, int rows_own, uint8_t *up_window,
                         int up_rows_own, uint8_t *down_window, uint64_t epoch) {
+  NOT_MULTI(ctx);
   if (!ctx) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
   if (!self_window || w < 16 || (w & 15) || rows_own < 4 || epoch == 0 || (up_window && up_rows_own < 4) ||
@@ -1046,12 +1361,14 @@ static int band_fused_impl(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks,
 
 int sharp_band_p2p_sharpen(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
                            int row1, uint64_t epoch, const sharp_params *params, uint8_t *out, int grid_cap) {
+  NOT_MULTI(ctx);
   return band_fused_impl(ctx, windows, n_ranks, rank, w, h, row0, row1, 0, false, epoch, params, out, grid_cap);
 }
 
 int sharp_band_p2p_step(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank, int w, int h, int row0,
                         int row1, int up_rows_own, uint64_t epoch, const sharp_params *params, uint8_t *out,
                         int grid_cap) {
+  NOT_MULTI(ctx);
   if (rank > 0 && up_rows_own < 4)
     return ctx ? set_err(ctx, SHARP_EINVAL, "%s", "up_rows_own < 4") : SHARP_EINVAL;
   return band_fused_impl(ctx, windows, n_ranks, rank, w, h, row0, row1, up_rows_own, true, epoch, params, out,
@@ -1131,6 +1448,7 @@ static int band_fused_impl(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks,
 
 int sharp_band_p2p_allreduce(sharp_ctx *ctx, uint8_t *const *windows, int n_ranks, int rank,
                              const uint64_t *d_partial, uint64_t epoch, uint64_t *d_total) {
+  NOT_MULTI(ctx);
   if (!ctx) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
   if (!windows || !d_partial || !d_total || n_ranks < 1 || n_ranks > 32 || rank < 0 || rank >= n_ranks ||
@@ -1180,6 +1498,7 @@ int sharp_set_path(sharp_ctx *ctx, int path) {
   if (!ctx || path < SHARP_PATH_AUTO || path > SHARP_PATH_RES) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
   ctx->path = path;
+  for (sharp_ctx *sc : ctx->sub) sc->path = path;  // multi-device: every device
   return SHARP_OK;
 }
 

@@ -124,6 +124,81 @@ int main(void) {
   }
 
   sharp_destroy(ctx);
+
+  /* 6. multi-device contexts (sharp_config.num_devices / device_ids / shard):
+   *    a 2-way frame split, one image as 2 row bands, and device-resident
+   *    bands.  On a one-GPU box both entries are device 0. */
+  {
+    int ndev = 0;
+    CHECK(cudaGetDeviceCount(&ndev) == cudaSuccess && ndev >= 1, "cudaGetDeviceCount");
+    int ids[2] = {0, 1 % ndev};
+    sharp_config cfg;
+    memset(&cfg, 0, sizeof(cfg));
+    cfg.device = -1;
+    cfg.num_devices = 2;
+    cfg.device_ids = ids;
+    cfg.shard = SHARP_SHARD_AUTO;
+    sharp_ctx *m = NULL;
+    CHECK(sharp_create(&m, &cfg) == SHARP_OK, "sharp_create (2 devices)");
+    /* frames: 6 x 640x360 from host memory, 3 per device */
+    {
+      const int W = 640, H = 360, N = 6;
+      const size_t fb = (size_t)W * H;
+      uint8_t *imgs = malloc(N * fb), *ref = malloc(N * fb), *got = malloc(N * fb);
+      synth_frames(imgs, N, W, H, 0, 0x5EED2015ull + 21, 0, 0);
+      uint64_t sums[6], gsums[6];
+      CHECK(oracle_sharpen_batch(imgs, N, W, H, p.amount, p.gamma, p.osc_gain, p.osc_scale, ref, sums, 0) == 0,
+            "oracle batch");
+      CHECK(sharp_run_batch(m, imgs, N, W, H, &p, got) == SHARP_OK, "multi-device batch: %s", sharp_last_error(m));
+      compare(got, ref, N * fb, "frames split over 2 devices");
+      CHECK(sharp_get_batch_sums(m, gsums, N) == SHARP_OK, "multi-device batch sums");
+      for (int f = 0; f < N; ++f) CHECK(gsums[f] == sums[f], "S of frame %d (2 devices)", f);
+      free(imgs);
+      free(ref);
+      free(got);
+    }
+    /* one 1920x1080 image: 2 row bands (AUTO for n == 1), host buffers */
+    {
+      const int W = 1920, H = 1080;
+      const size_t n = (size_t)W * H;
+      uint8_t *img = malloc(n), *ref = malloc(n), *got = malloc(n);
+      synth_frames(img, 1, W, H, 0, 0x5EED2015ull + 22, 0, 0);
+      uint64_t S_ref = 0;
+      double m_ref = 0.0;
+      CHECK(oracle_sharpen(img, W, H, p.amount, p.gamma, p.osc_gain, p.osc_scale, ref, &S_ref, &m_ref) == 0, "oracle");
+      CHECK(sharp_run(m, img, W, H, &p, got) == SHARP_OK, "2 row bands: %s", sharp_last_error(m));
+      compare(got, ref, n, "one image as 2 row bands");
+      sharp_stats st;
+      CHECK(sharp_get_stats(m, &st) == SHARP_OK && st.edge_sum == S_ref && st.edge_mean == m_ref, "2-band S / mean");
+      /* the same image as device-resident bands (sharp_run_bands) */
+      uint8_t *bands[2], *outs[2];
+      int r0[2], r1[2];
+      for (int g = 0; g < 2; ++g) {
+        CHECK(sharp_band_rows(H, 2, g, &r0[g], &r1[g]) == SHARP_OK, "sharp_band_rows");
+        const size_t bytes = (size_t)(r1[g] - r0[g]) * W;
+        CHECK(cudaSetDevice(ids[g]) == cudaSuccess, "cudaSetDevice");
+        CHECK(cudaMalloc((void **)&bands[g], bytes) == cudaSuccess && cudaMalloc((void **)&outs[g], bytes) == cudaSuccess,
+              "band cudaMalloc");
+        CHECK(cudaMemcpy(bands[g], img + (size_t)r0[g] * W, bytes, cudaMemcpyHostToDevice) == cudaSuccess, "band H2D");
+      }
+      CHECK(sharp_run_bands(m, (const uint8_t *const *)bands, W, H, &p, outs) == SHARP_OK, "sharp_run_bands: %s",
+            sharp_last_error(m));
+      memset(got, 0, n);
+      for (int g = 0; g < 2; ++g) {
+        CHECK(cudaSetDevice(ids[g]) == cudaSuccess, "cudaSetDevice");
+        CHECK(cudaMemcpy(got + (size_t)r0[g] * W, outs[g], (size_t)(r1[g] - r0[g]) * W, cudaMemcpyDeviceToHost) ==
+                  cudaSuccess,
+              "band D2H");
+        cudaFree(bands[g]);
+        cudaFree(outs[g]);
+      }
+      compare(got, ref, n, "device-resident bands (sharp_run_bands)");
+      free(img);
+      free(ref);
+      free(got);
+    }
+    sharp_destroy(m);
+  }
   printf("c_abi_check ok (%s)\n", sharp_version());
   return 0;
 }

@@ -100,3 +100,43 @@ def test_reading_switch_values_agree_across_header_binding_and_oracle():
         h = int(re.search(rf"SHARP_READ_{name}\s*=\s*(\d+)", hdr).group(1))
         o = int(re.search(rf"#define ORACLE_READ_{name}\s+(\d+)", orc).group(1))
         assert h == o == getattr(p, f"SHARP_READ_{name}") == getattr(oracle, f"READ_{name}"), name
+
+
+def test_config_struct_layout_matches_the_header(tmp_path):
+    """The binding's SharpConfig mirrors include/sharp.h's sharp_config (the
+    multi-device fields num_devices / device_ids / shard included)."""
+    import subprocess
+    import paper_conf_icpp_fanjzac15_b200 as p
+    src = tmp_path / "layout.c"
+    src.write_text('#include <stddef.h>\n#include <stdio.h>\n#include "sharp.h"\n'
+                   'int main(void){printf("%zu %zu %zu %zu\\n", sizeof(sharp_config), '
+                   'offsetof(sharp_config, num_devices), offsetof(sharp_config, device_ids), '
+                   'offsetof(sharp_config, shard)); return 0;}\n')
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), "-o", str(exe), str(src)], check=True)
+    size, o_n, o_ids, o_sh = map(int, subprocess.run([str(exe)], capture_output=True, text=True).stdout.split())
+    C = p.binding.SharpConfig
+    assert ctypes.sizeof(C) == size
+    assert (C.num_devices.offset, C.device_ids.offset, C.shard.offset) == (o_n, o_ids, o_sh)
+
+
+def test_band_rows_of_the_abi_match_the_python_partition():
+    """sharp_band_rows (the C ABI's row-band partition) equals
+    bands.band_rows, tiles [0, h) with multiples of 4, and rejects bad requests."""
+    import paper_conf_icpp_fanjzac15_b200 as p
+    from paper_conf_icpp_fanjzac15_b200.bands import band_rows
+    for h in (8, 12, 1080, 2160, 4320, 16384, 1084):
+        for G in range(1, 9):
+            if h // 4 < G:
+                with pytest.raises(p.SharpError):
+                    p.sharp_band_rows(h, G, 0)
+                continue
+            prev = 0
+            for g in range(G):
+                r = p.sharp_band_rows(h, G, g)
+                assert r == band_rows(h, G, g)
+                assert r[0] == prev and r[1] > r[0] and r[0] % 4 == 0 and r[1] % 4 == 0
+                prev = r[1]
+            assert prev == h
+    with pytest.raises(p.SharpError):
+        p.sharp_band_rows(1080, 2, 2)

@@ -18,6 +18,7 @@ names = ["start", "p1_first", "p1_last_end", "lut_first", "lut_last_end", "p2_fi
 buf = (ctypes.c_ulonglong * 8)()
 for W, H in [(512, 512), (1920, 1080), (3840, 2160), (7680, 4320)]:
     s = Sharpener()
+    s.set_path(1)  # the step kernel (the timeline probes live there)
     d = torch.from_numpy(synth.image(W, H, "natural", seed=1)).cuda()
     o = torch.empty_like(d)
     rows = []
