@@ -283,14 +283,19 @@ def run_bands_workload(args, world, rank, local):
         from paper_conf_icpp_fanjzac15_b200.bands import P2PBand
         p2p = P2PBand(sh, W, H)
         epoch = [0]
+        # ranks sharing one GPU (the SHARP_BENCH_SHARE_GPU test hook) bound
+        # their persistent grids so that every band's launch can run
+        cap = 0
+        if SHARE_GPU and world > torch.cuda.device_count():
+            cap = max(1, (2 * torch.cuda.get_device_properties(local).multi_processor_count) // world)
 
         def step(src, dst):
             p2p.own.copy_(src)  # this image's rows into the window (the NCCL path copies them too)
             epoch[0] += 1
             if args.exchange == "one":
-                p2p.step_one_launch(epoch[0], dst, PARAMS)
+                p2p.step_one_launch(epoch[0], dst, PARAMS, grid_cap=cap)
             elif args.exchange == "fused":
-                p2p.step_fused(epoch[0], dst, PARAMS)
+                p2p.step_fused(epoch[0], dst, PARAMS, grid_cap=cap)
             else:
                 p2p.step(epoch[0], dst, PARAMS)
     else:
