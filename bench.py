@@ -149,31 +149,63 @@ def init_group(torch, dist, local):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
 
-def traffic_per_launch(px_per_launch):
+KERNEL_SOURCES = {  # the sources a kernel's SASS depends on (profiles are keyed on their hash)
+    "step": ["kernels_tma.cu", "tma_common.cuh", "device_common.cuh", "kernels.h"],
+    "res": ["kernels_res.cu", "tma_common.cuh", "device_common.cuh", "kernels.h"],
+}
+
+
+def kernel_source_hash(kind):
+    import hashlib
+    h = hashlib.sha256()
+    for f in KERNEL_SOURCES[kind]:
+        h.update(open(os.path.join(ROOT, "paper_conf_icpp_fanjzac15_b200", "csrc", f), "rb").read())
+    return h.hexdigest()
+
+
+def committed_profile(kind="step"):
+    """The newest committed ncu capture summary of this kernel
+    (profiles/<round>/traffic*.json), if it was taken from the CURRENT kernel
+    sources (else None: a stale capture is not reported)."""
+    import glob
+    for f in sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "traffic*.json")), reverse=True):
+        try:
+            t = json.load(open(f))
+        except Exception:
+            continue
+        if t.get("kernel_kind", "step") != kind:
+            continue
+        if t.get("source_sha256") != kernel_source_hash(kind):
+            return None
+        t["_file"] = os.path.relpath(f, ROOT)
+        return t
+    return None
+
+
+def traffic_per_launch(px_per_launch, kind="step"):
     """DRAM bytes (read + write) per launch of the dominant kernel, from the
-    committed ncu --set full capture of this kernel (profiles/<round>/
-    traffic.json: dram bytes per output pixel), scaled to this launch; None
-    if no capture is committed."""
-    import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "traffic.json")))
-    if not files:
-        return None
-    try:
-        t = json.load(open(files[-1]))
-        return float(t["dram_bytes_per_px"]) * px_per_launch
-    except Exception:
-        return None
+    committed ncu --set full capture of this kernel (dram bytes per output
+    pixel), scaled to this launch; None without a capture of the current
+    kernel sources."""
+    t = committed_profile(kind)
+    return float(t["dram_bytes_per_px"]) * px_per_launch if t else None
 
 
-def issue_profile():
+def issue_profile(kind="step"):
     """Warp instructions per output pixel of the dominant kernel, from the
-    committed ncu capture (profiles/<round>/traffic.json), or None."""
-    import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "traffic.json")))
+    committed capture of the current kernel sources, or None."""
+    t = committed_profile(kind)
+    return float(t["warp_instr_per_px"]) if t else None
+
+
+def cpu_model():
     try:
-        return float(json.load(open(files[-1]))["warp_instr_per_px"]) if files else None
-    except Exception:
-        return None
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def issue_roofline(px_per_launch, k_avg_ms, sm_mhz, n_sms):
@@ -223,7 +255,7 @@ def run_reference(args, world, rank):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(np.median(times) * 1e3),
         "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
         "data": "synthetic", "config": workload_config(args, world),
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
                          "sample": f"{len(idx)} of {args.frames} frames per step (every "
                                    f"{max(1, args.frames // sample)}th), OpenMP over frames"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -638,6 +670,26 @@ def main():
             graph = {"reps_per_graph": reps, "ms_per_call": e0.elapsed_time(e1) / (5 * reps)}
         except Exception as ex:  # capture is an extra, never a failure of the run
             graph = {"unavailable": f"{type(ex).__name__}: {ex}"[:200]}
+    # ---- strong scaling beside the weak line (BASELINE configs[4]: ONE batch
+    # of --frames frames split over the ranks): same kernels, each rank's
+    # share of the batch, the slowest rank's time
+    strong = None
+    if world > 1 and args.scaling == "weak":
+        _, sn = shard.frame_range(args.frames, world, rank)
+        sh.enqueue_batch(d_in[:sn], d_out[:sn], prm)
+        barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            sh.enqueue_batch(d_in[:sn], d_out[:sn], prm)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ms_strong = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+        strong = {"scaling": "strong", "value": args.frames * fb / (ms_strong * 1e-3) / 1e6, "unit": UNIT,
+                  "ms_per_step": ms_strong, "frames_total": args.frames, "frames_per_gpu": sn,
+                  "workload": f"one batch of {args.frames} x {W}x{H} frames split over {world} GPU(s)"}
     total_px = args.frames * fb * (world if args.scaling == "weak" else 1)  # all ranks' frames
     value = total_px / (ms_step * 1e-3) / 1e6
 
@@ -687,7 +739,7 @@ def main():
         cores = len(os.sched_getaffinity(0))
         idx = list(range(0, n, max(1, n // args.cpu_sample)))[:args.cpu_sample]
         rate, dt = cpu_oracle_rate(h_in.numpy()[idx], cores)
-        cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
+        cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
                "sample": f"{len(idx)} of {n} frames (every {max(1, n // args.cpu_sample)}th), "
                          f"{dt:.1f} s wall on {cores} threads"}
         # The paper's headline is end-to-end GPU (with transfers) vs a
@@ -709,6 +761,8 @@ def main():
             "config": workload_config(args, world),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic_per_launch(px_per_launch),
+                         "traffic_source": ((committed_profile() or {}).get("_file") or
+                                            "none: no ncu capture of the current kernel sources is committed"),
                          "kernel": kname, "peak_source": pk_src,
                          "alg_bytes_per_px": ALG_BYTES_PER_PX, "px_per_launch": px_per_launch,
                          "kernel_avg_ms": k_avg_ms, "kernel_launches": k_launches,
@@ -721,6 +775,7 @@ def main():
             "issue_roofline": issue_roofline(px_per_launch, k_avg_ms, clk.summary().get("sm_mhz"),
                                              torch.cuda.get_device_properties(local).multi_processor_count),
             "gpu_launches": launches_per_step * args.steps,
+            "strong_scaling": strong,
             "clocks": clk.summary(),
             "cpu_baseline": cpu,
             "paper_context": paper_context,

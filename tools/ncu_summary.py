@@ -103,7 +103,17 @@ def main():
         lines += ["```", ""]
     open(os.path.join(out_dir, "ncu_summary.md"), "w").write("\n".join(lines))
     if summary:
-        json.dump(summary[0], open(os.path.join(out_dir, "traffic.json"), "w"), indent=1)
+        # keyed on the kernel's sources, so bench.py reports it only while they are unchanged
+        sys.path.insert(0, os.path.join(os.path.dirname(os.path.abspath(__file__)), ".."))
+        import importlib.util
+        spec = importlib.util.spec_from_file_location("bench", os.path.join(os.path.dirname(__file__), "..", "bench.py"))
+        bench = importlib.util.module_from_spec(spec)
+        spec.loader.exec_module(bench)
+        kind = "res" if "res_kernel" in summary[0]["kernel"] else "step"
+        summary[0]["kernel_kind"] = kind
+        summary[0]["source_sha256"] = bench.kernel_source_hash(kind)
+        name = "traffic.json" if kind == "step" else f"traffic_{kind}.json"
+        json.dump(summary[0], open(os.path.join(out_dir, name), "w"), indent=1)
     print("\n".join(lines))
 
 
