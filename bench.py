@@ -427,16 +427,19 @@ STAGED_BYTES_PER_PX = {"downscale": 1.25, "border": 0.0, "center": 4.25, "sobel"
 
 
 def run_ladder_workload(args, world, rank, local):
-    """The optimisation ladder (sec. V, Fig. 12 / Fig. 14) on
-    BASELINE configs[2] (4K frames, "kernel-fusion roofline study"): the
-    paper's staged base design (one kernel per stage, Fig. 13 breakdown), the
-    two-pass fused kernels and the one-launch step kernel, each timed on the
-    same device-resident batch (> L2), all bit-identical."""
+    """The optimisation ladder (sec. V, Fig. 12 / Fig. 14)
+    on BASELINE configs[2] (4K frames, "kernel-fusion roofline study"): the
+    paper's staged base design (one kernel per stage, the Fig. 13 per-stage
+    breakdown), then one optimisation per rung -- fusion, the strength table,
+    vectorisation / data reuse, the persistent TMA kernel, the TMEM-resident
+    pEdge -- each timed on the same device-resident batch (> L2), all
+    bit-identical; plus the optimised kernel's per-stage instruction shares
+    (the Fig. 13(c) analogue) from a committed capture."""
     import torch
 
     import synth
-    from paper_conf_icpp_fanjzac15_b200 import (SHARP_PATH_STAGED, SHARP_PATH_STEP, SHARP_PATH_TWO_PASS,
-                                                Sharpener)
+    from paper_conf_icpp_fanjzac15_b200 import (SHARP_PATH_FUSED, SHARP_PATH_FUSED_EXP, SHARP_PATH_RES,
+                                                SHARP_PATH_STAGED, SHARP_PATH_STEP, SHARP_PATH_TWO_PASS, Sharpener)
 
     if world > 1:
         if rank == 0:
@@ -450,10 +453,18 @@ def run_ladder_workload(args, world, rank, local):
     torch.cuda.set_stream(stream)
     pk, pk_src = peaks()
     peak = float(pk["hbm_gbs"])
+    ladder = [("staged (paper base: 7 kernels per frame, every stage in HBM, per-pixel f64 exponentiation)",
+               SHARP_PATH_STAGED, 34.5),
+              ("+ fusion (scalar: 1 px / thread, 4 kernels per frame, per-pixel f64 exponentiation)",
+               SHARP_PATH_FUSED_EXP, 3.25),
+              ("+ strength table (the exponentiations once per frame from the reduced mean)", SHARP_PATH_FUSED, 3.25),
+              ("+ vectorisation / data reuse (8 px / lane f16x2 SIMD, shuffled halos, 2 kernels per chunk)",
+               SHARP_PATH_TWO_PASS, 3.0),
+              ("+ persistent TMA kernel (whole batch in ONE launch, in-kernel reduction barrier and tables)",
+               SHARP_PATH_STEP, ALG_BYTES_PER_PX),
+              ("+ TMEM-resident pEdge (pass 2 reuses pass 1's Sobel; DRAM ~2 B/px)", SHARP_PATH_RES, ALG_BYTES_PER_PX)]
     rungs, outs = [], {}
-    for name, path in [("staged (paper base: 7 kernels, all stages in HBM)", SHARP_PATH_STAGED),
-                       ("two-pass fused (edge_sum + sharpen per chunk)", SHARP_PATH_TWO_PASS),
-                       ("step kernel (one persistent TMA launch)", SHARP_PATH_STEP)]:
+    for name, path, alg in ladder:
         sh = Sharpener(device=local)
         sh.set_stream(stream)
         sh.set_path(path)
@@ -470,7 +481,7 @@ def run_ladder_workload(args, world, rank, local):
         torch.cuda.synchronize()
         ms = ev0.elapsed_time(ev1) / args.steps
         rung = {"path": name, "ms_per_step": ms, "mpix_s": n * W * H / (ms * 1e-3) / 1e6,
-                "launches_per_step": sh.stats().kernels}
+                "launches_per_step": sh.stats().kernels, "alg_bytes_per_px": alg}
         if path == SHARP_PATH_STAGED:
             st = sh.stage_times()
             tot = sum(st.values()) or 1.0
@@ -479,33 +490,42 @@ def run_ladder_workload(args, world, rank, local):
                                   "achieved_gbs": (STAGED_BYTES_PER_PX[k] * W * H / (v / (args.steps * n) * 1e-3)
                                                    / 1e9) if v > 0 and STAGED_BYTES_PER_PX[k] else None}
                               for k, v in st.items()}
-            rung["alg_bytes_per_px"] = sum(STAGED_BYTES_PER_PX.values())
-        else:
+        elif path == SHARP_PATH_TWO_PASS:
             kt = sh.kernel_times()
-            if path == SHARP_PATH_TWO_PASS:
-                rung["pass1_share"] = kt.pass1_ms / max(1e-9, kt.pass1_ms + kt.pass2_ms)
-            rung["alg_bytes_per_px"] = 3.0 if path == SHARP_PATH_TWO_PASS else ALG_BYTES_PER_PX
+            rung["pass1_share"] = kt.pass1_ms / max(1e-9, kt.pass1_ms + kt.pass2_ms)
         rung["hbm_frac_alg2"] = ALG_BYTES_PER_PX * n * W * H / (ms * 1e-3) / 1e9 / peak
         sh.set_profiling(False)
         outs[path] = d_out
         rungs.append(rung)
         sh.close()
-    identical = bool(torch.equal(outs[SHARP_PATH_STAGED], outs[SHARP_PATH_STEP]) and
-                     torch.equal(outs[SHARP_PATH_TWO_PASS], outs[SHARP_PATH_STEP]))
+    identical = all(bool(torch.equal(o, outs[SHARP_PATH_STEP])) for o in outs.values())
     parity = None
     if not args.no_cpu:
         import oracle
         ref, _ = oracle.sharpen_batch(imgs[:1], *PARAMS)
         parity = {"frames_checked": 1, "mismatched_pixels": int((outs[SHARP_PATH_STEP][:1].cpu().numpy() != ref).sum())}
     base = rungs[0]["ms_per_step"]
-    for r in rungs:
+    for i, r in enumerate(rungs):
         r["speedup_vs_staged"] = base / r["ms_per_step"]
+        r["speedup_vs_previous"] = rungs[i - 1]["ms_per_step"] / r["ms_per_step"] if i else 1.0
+    # Fig. 13(c) analogue for the optimised kernel: its instruction share per
+    # stage (SASS attribution of a committed ncu capture of the current sources)
+    shares = None
+    try:
+        import glob
+        f = sorted(glob.glob(os.path.join(ROOT, "profiles", "*", "stage_shares.json")))[-1]
+        t = json.load(open(f))
+        if t.get("source_sha256") == kernel_source_hash("step"):
+            shares = {"source": os.path.relpath(f, ROOT), "thread_instr_per_px": t["thread_instr_per_px"],
+                      "shares": t["shares"]}
+    except (IndexError, OSError, ValueError, KeyError):
+        pass
     line = {"metric": METRIC, "workload": "ladder", "unit": UNIT, "n_gpus": 1, "steps": args.steps,
             "warmup": args.warmup, "dtype": "f32", "data": "synthetic",
             "config": {"workload": f"{n} x {W}x{H} u8 frames (BASELINE configs[2]: kernel-fusion roofline study)",
                        "l2": f"batch {2 * n * W * H / 1e6:.0f} MB in + out > 126 MB L2"},
             "hbm_peak_gbs": peak, "peak_source": pk_src, "ladder": rungs, "paths_identical": identical,
-            "parity": parity}
+            "step_kernel_stage_shares": shares, "parity": parity}
     print(json.dumps(line), flush=True)
 
 

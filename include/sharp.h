@@ -352,12 +352,25 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
  *                       4K included), else SHARP_EUNSUPPORTED
  *   SHARP_PATH_TWO_PASS two fused kernels per chunk of frames (kernels.cu): Sobel +
  *                       reduction + LUT, then everything else; any w % 4 == 0
+ *   SHARP_PATH_FUSED    scalar fused kernels (kernels_scalar.cu): one thread per pixel, no SIMD
+ *                       or data reuse, the stages fused into downscale / Sobel + reduction /
+ *                       table / everything else (4 launches per frame; sec. V-B "kernel fusion")
+ *   SHARP_PATH_FUSED_EXP the same with strength and oscStrength evaluated per pixel in f64 (the
+ *                       "many exponentiations" of L232) instead of the per-frame table
  *   SHARP_PATH_STAGED   the paper's BASE GPU design (sec. IV): one kernel per
  *                       stage, every intermediate matrix in HBM (kernels_staged.cu,
  *                       7 launches per frame); the per-stage breakdown of Fig. 13
  * Takes effect at the next call.  Row-band calls need AUTO or STEP.  Environment
  * SHARP_FORCE_GENERIC=1 at sharp_create selects SHARP_PATH_TWO_PASS. */
-enum { SHARP_PATH_AUTO = 0, SHARP_PATH_STEP = 1, SHARP_PATH_TWO_PASS = 2, SHARP_PATH_STAGED = 3, SHARP_PATH_RES = 4 };
+enum {
+  SHARP_PATH_AUTO = 0,
+  SHARP_PATH_STEP = 1,
+  SHARP_PATH_TWO_PASS = 2,
+  SHARP_PATH_STAGED = 3,
+  SHARP_PATH_RES = 4,
+  SHARP_PATH_FUSED = 5,
+  SHARP_PATH_FUSED_EXP = 6
+};
 int sharp_set_path(sharp_ctx *ctx, int path);
 int sharp_get_path(const sharp_ctx *ctx);
 

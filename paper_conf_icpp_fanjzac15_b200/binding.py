@@ -24,6 +24,8 @@ SHARP_PATH_STEP = 1
 SHARP_PATH_TWO_PASS = 2
 SHARP_PATH_STAGED = 3
 SHARP_PATH_RES = 4
+SHARP_PATH_FUSED = 5
+SHARP_PATH_FUSED_EXP = 6
 STAGE_NAMES = ("downscale", "border", "center", "sobel", "reduction", "strength", "sharpness")
 SHARP_NUM_STAGES = len(STAGE_NAMES)
 

@@ -77,37 +77,6 @@ __device__ __forceinline__ void load_block(Block &B, const uint8_t *__restrict__
   B.S[3] = (float)(blk4(B.r[0].nw, B.r[1].nw, B.r[2].nw, B.r[3].nw) & smask);
 }
 
-// ------------------------------------------------------- upscale border (R4, R5)
-// Final value of U at a pixel of the 2-pixel ring (last writer of steps
-// i..vii of L140-L142).  Sc = 16*D of the current D row block (row k) for
-// columns j0-1..j0+2, Sn = the next D row (k+1); j0 = c0/4; r = 4k + a'.
-// col_wins: the R5 alternative (column work after the row work: the top-left
-// 2x2 keeps the column line's values instead of D[0][0]).
-__device__ __forceinline__ float ring_u(int r, int c, int W, int H, int j0, const float (&Sc)[4], const float (&Sn)[4],
-                                        bool col_wins) {
-  const int w = W >> 2, h = H >> 2;
-  auto col = [&](int j) { return j - j0 + 1; };  // index into Sc/Sn (0..3)
-  // register selects instead of a dynamically indexed local array (no stack frame)
-  auto at = [](const float(&a)[4], int i) { return i <= 0 ? a[0] : i == 1 ? a[1] : i == 2 ? a[2] : a[3]; };
-  if (r >= H - 2 && c >= W - 2) {                 // (vii): third last of last column = D[h-1][w-1]
-    return __fmul_rn(at(Sc, col(w - 1)), 1.0f / 16.0f);
-  }
-  if ((c <= 1 || c >= W - 2) && r <= H - 3) {     // (vi)/(ii)/(iv): column lines
-    const int j = (c <= 1) ? 0 : w - 1;
-    if (c <= 1 && r <= 1 && !col_wins) return __fmul_rn(at(Sc, col(0)), 1.0f / 16.0f);  // (v) then (vi): D[0][0]
-    const int rr = (r == H - 3) ? H - 4 : r;   // third last <- fourth last
-    const int k = rr & 3;                      // rr>>2 == current D row (rr in the block of r)
-    return line_val(at(Sc, col(j)), at(Sn, col(j)), k);
-  }
-  // rows 0/1 (line of D row 0) or H-2/H-1 (line of D row h-1); Sc is that D row.
-  const int cc = (c == W - 3) ? W - 4 : c;
-  const int jj = cc >> 2, k = cc & 3;
-  const float x = at(Sc, col(jj));
-  const float y = (k == 0) ? x : at(Sc, col(jj + 1));
-  (void)h;
-  return line_val(x, y, k);
-}
-
 // =========================================================================
 // Pass 1: Sobel + reduction + last-block-done LUT construction.
 // =========================================================================

@@ -149,6 +149,16 @@ cudaError_t launch_staged(const uint8_t *in, int W, int H, const Params &p, void
                           const StageTimer &timer);
 constexpr int kStagedLaunches = 7;
 
+// Scalar fused kernels (kernels_scalar.cu): one thread per pixel, stages fused
+// (downscale, Sobel + reduction, table, everything else); table = false
+// evaluates strength / oscStrength per pixel in f64 (the paper's fused
+// kernel), true looks them up.  4 launches per frame.
+size_t scalar_scratch_bytes(int W, int H);
+cudaError_t launch_scalar(const uint8_t *in, int W, int H, const Params &p, void *scratch, unsigned long long *sum,
+                          double *mean, uint8_t *out, bool table, cudaStream_t st);
+cudaError_t preload_scalar();
+constexpr int kScalarLaunches = 4;
+
 // Fused peer-memory band exchange (bands_p2p.cu).
 constexpr int kP2PCtlBytes = 1024;
 constexpr int kP2PHalo = 4;

@@ -309,7 +309,7 @@ cudaError_t timed(sharp_ctx *ctx, cudaStream_t st, int kind, double px, F launch
 
 // Staged-path scratch of a slot for one w x h frame (grown on demand).
 int rc_staged(sharp_ctx *ctx, Slot &slot, cudaStream_t st, int w, int h) {
-  const size_t need = sharp::staged_scratch_bytes(w, h);
+  const size_t need = std::max(sharp::staged_scratch_bytes(w, h), sharp::scalar_scratch_bytes(w, h));
   if (need <= slot.staged_cap) return SHARP_OK;
   cudaStreamSynchronize(st);
   cudaStreamSynchronize(ctx->stream);
@@ -355,8 +355,23 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
                    uint8_t *dout, cudaStream_t st, Slot &slot, size_t chunk, size_t frame_base, int *launches,
                    unsigned int *tc, const Strides &str = Strides()) {
   const size_t fb = (size_t)w * h;
-  if (!str.dense() && ctx->path == SHARP_PATH_STAGED) return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "strided frames on the staged path");
+  if (!str.dense() && (ctx->path == SHARP_PATH_STAGED || ctx->path == SHARP_PATH_FUSED || ctx->path == SHARP_PATH_FUSED_EXP))
+    return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "strided frames on the staged / scalar fused paths");
   const size_t nchunks = ((size_t)n + chunk - 1) / chunk;
+  if (ctx->path == SHARP_PATH_FUSED || ctx->path == SHARP_PATH_FUSED_EXP) {  // scalar fused ladder rungs
+    if (prm.flags & sharp::kReadPerPixel)
+      return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "the scalar fused paths implement the default R2 / R5 / R14");
+    if ((rc_staged(ctx, slot, st, w, h))) return SHARP_ENOMEM;
+    for (int f = 0; f < n; ++f) {
+      CK(timed(ctx, st, 2, (double)fb, [&] {
+        return sharp::launch_scalar(din + (size_t)f * fb, w, h, prm, slot.staged, ctx->sums + frame_base + f,
+                                    ctx->means + frame_base + f, dout + (size_t)f * fb, ctx->path == SHARP_PATH_FUSED,
+                                    st);
+      }));
+      *launches += sharp::kScalarLaunches;
+    }
+    return SHARP_OK;
+  }
   if (ctx->path == SHARP_PATH_STAGED) {  // the paper's base design: K1..K7 per frame
     if ((rc_staged(ctx, slot, st, w, h))) return SHARP_ENOMEM;
     sharp::StageTimer tm;
@@ -1126,7 +1141,7 @@ int sharp_create(sharp_ctx **out, const sharp_config *cfg) {
     if (e != cudaSuccess) break;
     // load every kernel now (lazy module loading can deadlock spinning kernels, kernels.h)
     if ((e = sharp::preload_step()) != cudaSuccess || (e = sharp::preload_res()) != cudaSuccess || (e = sharp::preload_two_pass()) != cudaSuccess ||
-        (e = sharp::preload_staged()) != cudaSuccess || (e = sharp::preload_p2p()) != cudaSuccess ||
+        (e = sharp::preload_staged()) != cudaSuccess || (e = sharp::preload_scalar()) != cudaSuccess || (e = sharp::preload_p2p()) != cudaSuccess ||
         (e = sharp::preload_layout()) != cudaSuccess)
       break;
     if (c.max_frames > 0 && (rc = ensure_frames(ctx, (size_t)c.max_frames))) break;
@@ -1495,7 +1510,7 @@ int sharp_ipc_close_handle(void *d_ptr) {
 }
 
 int sharp_set_path(sharp_ctx *ctx, int path) {
-  if (!ctx || path < SHARP_PATH_AUTO || path > SHARP_PATH_RES) return SHARP_EINVAL;
+  if (!ctx || path < SHARP_PATH_AUTO || path > SHARP_PATH_FUSED_EXP) return SHARP_EINVAL;
   if (ctx->poisoned) return SHARP_ESTATE;
   ctx->path = path;
   for (sharp_ctx *sc : ctx->sub) sc->path = path;  // multi-device: every device

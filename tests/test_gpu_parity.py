@@ -10,7 +10,8 @@ import torch
 
 import oracle
 import synth
-from paper_conf_icpp_fanjzac15_b200 import (SHARP_EINVAL, SHARP_EUNSUPPORTED, SHARP_PATH_RES, SHARP_PATH_STAGED,
+from paper_conf_icpp_fanjzac15_b200 import (SHARP_EINVAL, SHARP_EUNSUPPORTED, SHARP_PATH_FUSED, SHARP_PATH_FUSED_EXP,
+                                            SHARP_PATH_RES, SHARP_PATH_STAGED,
                                             SHARP_PATH_STEP, SHARP_PATH_TWO_PASS, STAGE_NAMES, SharpError, Sharpener)
 
 pytestmark = pytest.mark.gpu
@@ -27,7 +28,7 @@ PARAMS = [
 ]
 
 
-@pytest.fixture(scope="module", params=["auto", "res", "step", "generic", "staged"])
+@pytest.fixture(scope="module", params=["auto", "res", "step", "generic", "fused", "fused_exp", "staged"])
 def sh(request):
     """A context on the automatic kernel path (the TMEM-resident kernel, else
     the step kernel, when W % 16 == 0), one forced onto the step kernel, one
@@ -46,6 +47,10 @@ def sh(request):
     if request.param == "res":
         s.set_path(SHARP_PATH_RES)
         s._force_step = True  # same geometry rules
+    if request.param == "fused":
+        s.set_path(SHARP_PATH_FUSED)
+    if request.param == "fused_exp":
+        s.set_path(SHARP_PATH_FUSED_EXP)
     if old is None:
         del os.environ["SHARP_FORCE_GENERIC"]
     else:
@@ -232,12 +237,15 @@ def test_invalid_params_and_overlap_rejected(sh):
 
 
 def test_ladder_paths_identical_and_stage_times():
-    """The optimisation ladder (staged base -> two-pass fused -> step kernel)
-    gives the same bytes; the staged path reports a time for every stage."""
+    """The optimisation ladder (staged base -> scalar fused with per-pixel
+    exponentiation -> + strength table -> vectorised two-pass -> step kernel
+    -> TMEM-resident kernel) gives the same bytes; the staged path reports a
+    time for every stage."""
     imgs = synth.frames(2, 3840, 2160, "natural", seed=synth.BASE_SEED + 2)
     ref, ref_sums = oracle.sharpen_batch(imgs, *DEFAULT)
     d = torch.from_numpy(imgs).cuda()
-    for path in [SHARP_PATH_STAGED, SHARP_PATH_TWO_PASS, SHARP_PATH_STEP]:
+    for path in [SHARP_PATH_STAGED, SHARP_PATH_FUSED_EXP, SHARP_PATH_FUSED, SHARP_PATH_TWO_PASS, SHARP_PATH_STEP,
+                 SHARP_PATH_RES]:
         with Sharpener() as s:
             s.set_path(path)
             s.set_profiling(True)
