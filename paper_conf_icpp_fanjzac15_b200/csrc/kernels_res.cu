@@ -489,7 +489,7 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     for (int i = 0; i < kPipes * kResStages; ++i) {
       const uint32_t b0 = sbase + kResBarOff + (uint32_t)((i / kResStages) * 16 * kResStages);
       mbar_init(b0 + 8 * (i % kResStages), 1);
-      mbar_init(b0 + 8 * kResStages + 8 * (i % kResStages), kWarpsT);
+      mbar_init(b0 + 8 * kResStages + 8 * (i % kResStages), 32 * kWarpsT);  // every consumer thread arrives
     }
     fence_barrier_init();
   }

@@ -101,6 +101,7 @@ enum TaskType { kEmpty = 0, kP1 = 1, kLut = 2, kP2 = 3, kHalo = 4, kEnd = -1 };
 struct StepParams {
   Geo g;
   int mode;       // kStepAll, or a row band's kStepPass1 / kStepPass2
+  int compact;    // kStepAll with < 4 frames: [all pass 1][all LUT][all pass 2], no lag rounds
   int n;          // frames
   int L1, L2;     // round lags of the LUT and pass-2 tasks
   int per_round;  // 2 * per_frame + kLutTasks
@@ -142,6 +143,12 @@ __device__ __forceinline__ int4 decode(const StepParams &sp, int t) {  // {type,
     const int pf1 = sp.g.per_frame1;
     if (t < pf1) return make_int4(kP1, 0, t, 0);
     return t < pf1 + kLutTasks ? make_int4(kLut, 0, t - pf1, 0) : make_int4(kP2, 0, t - pf1 - kLutTasks, 0);
+  }
+  if (sp.compact) {  // a few frames: no lag rounds (their empty tasks cost a single image ~15 us)
+    const int pf1 = sp.g.per_frame1, A = sp.n * pf1, B = A + sp.n * kLutTasks;
+    if (t < A) return make_int4(kP1, t / pf1, t % pf1, 0);
+    if (t < B) return make_int4(kLut, (t - A) / kLutTasks, (t - A) % kLutTasks, 0);
+    return make_int4(kP2, (t - B) / sp.g.per_frame, (t - B) % sp.g.per_frame, 0);
   }
   const int rho = t / sp.per_round, k = t - rho * sp.per_round;
   const int pf1 = sp.g.per_frame1;
@@ -379,7 +386,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
   if (threadIdx.x == 0) {
     for (int i = 0; i < kStages; ++i) {
       mbar_init(ring.full0 + 8 * i, 1);
-      mbar_init(ring.empty0 + 8 * i, kWarpsT);
+      mbar_init(ring.empty0 + 8 * i, 32 * kWarpsT);  // every consumer thread arrives (RingT::release)
     }
     fence_barrier_init();
   }
@@ -524,7 +531,8 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         } else {
           stage_task[b] = d;
           if (d.x == kLut) stage_sum[b] = S & ((1ull << kAccShift) - 1);
-          mbar_arrive(full);  // no data: LUT, empty or end task
+          // no data (LUT, empty or end task): a plain arrive publishes it
+          mbar_arrive(full);
         }
       }
       if (d.x == kP2) lut_last[j++ & 1] = s - 1;
@@ -729,6 +737,7 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     sp.g.th1 = sp.g.th1 == kTH1 ? 9 : sp.g.th1 - 3;
   sp.g.per_frame1 = sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1);
   sp.mode = mode;
+  sp.compact = 0;
   sp.n = sg.n;
   sp.per_round = sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
 #ifndef SHARP_GRID_CTAS
@@ -766,16 +775,15 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     const int L1u = sp.L1, L2u = sp.L2;
     sp.L1 *= 2;  // measured: 2x the minimal lags removes most dependency waits
     sp.L2 *= 2;
-    if (sg.n < sp.L2) {
-      if (sg.n >= 4) {
-        sp.L1 = L1u;
-        sp.L2 = L2u;
-      } else {
-        sp.L1 = 1;
-        sp.L2 = 2;
-      }
+    if (sg.n < sp.L2) {  // (1x lags from 4 frames on: a few empty rounds cost less than LUT waits)
+      sp.L1 = L1u;
+      sp.L2 = L2u;
     }
     sp.ntasks = (sg.n + sp.L2) * sp.per_round;
+    if (sg.n < 4) {  // [pass 1 of all][LUT of all][pass 2 of all]: every dependency precedes its task
+      sp.compact = 1;
+      sp.ntasks = sg.n * sp.per_round;
+    }
   }
   sp.prm = p;
   sp.acc = a.acc;
