@@ -1,5 +1,5 @@
-// TMEM-resident sm_100a kernel (the "res" path; the default for frame
-// batches and single images up to ~10 Mpx).  ONE persistent launch per batch.
+// TMEM-resident sm_100a kernel (SHARP_PATH_RES).  ONE
+// persistent launch per batch, frames of up to ~10 Mpx.
 //
 // The two passes of the method -- pass 1: Sobel pEdge (L158-L172) summed for
 // the global mean (L174); pass 2: everything else (downscale L130, upscale
@@ -8,33 +8,34 @@
 // the Sobel twice.  Here pass 1 leaves each tile's pEdge in TENSOR MEMORY
 // (tcgen05.st: 8 pixels = 4 f16x2 words per lane and row; 256 KB per SM that
 // no other part of this path uses) and pass 2 of the same tile, on the same
-// CTA, reads it back (tcgen05.ld) after the frame's mean is known: no second
+// warps, reads it back (tcgen05.ld) after the frame's mean is known: no second
 // Sobel, no pEdge traffic to L2 or HBM.  The frame's input is re-read by pass
-// 2 from L2 (the re-read follows its pass 1 closely).
+// 2 from L2 (the re-read follows its pass 1 closely): ~2 B/px of DRAM.
 //
-// Work unit = one CTA tile (4 warp tiles of 240 columns x kT = 12 rows) of one
-// frame.  Per CTA the consumer warps process, in order,
-//     P1(t0) P1(t1) P2(t0) P1(t2) P2(t1) P1(t3) P2(t2) ...
-// (two TMEM slots of 48 columns: tile k uses slot k & 1), so between a tile's
-// pass 1 and its pass 2 the CTA does one full tile of other work while the
-// rest of the GPU completes the frame's pass 1 and its tables.  With a third
-// slot (in shared memory: TMEM holds 128 columns per CTA at 3 CTAs per SM)
-// the order is P1(t0) P1(t1) P1(t2) P2(t0) P1(t3) P2(t1) ..., one more tile
-// of slack: measured, two slots leave pass 2 waiting on the frame's table
-// (its build is on the critical path of every frame that straddles two of a
-// CTA's tile positions).
+// ONE CTA per SM (all 512 TMEM columns) = three independent pipelines (each:
+// 4 compute warps + a producer warp, its own smem stages and LUT buffers)
+// + one table warp.  Tile = 960 columns (4 warp tiles of 240) x kT = 12 rows.
+// Per pipeline the consumers process, in order,
+//     P1(t0) P1(t1) P1(t2) P2(t0) P1(t3) P2(t1) P1(t4) P2(t2) ...
+// (three TMEM slots of 48 columns per warp, tile k in slot k % 3), so between
+// a tile's pass 1 and its pass 2 the pipeline does one full tile of other
+// work while the rest of the GPU completes the frame's pass 1 and its table.
+//
+// Schedule: static -- pipeline v (of 3 x gridDim) takes positions v, v + 3
+// gridDim, ... of the frame-major tile order.  A producer issues P1 of
+// position k+2 before it waits for the table of position k, and a frame of
+// <= 2 x (3 gridDim) tiles spans at most three positions of a pipeline, so by
+// induction every awaited table completes (no deadlock; larger frames take
+// the step kernel).
 //
 // Dependencies (the global barrier of L174): every pass-1 warp adds
-// (1 << 40) + its partial sum to the frame's acc word.  The producer warp
-// needs frame f's table before it can issue P2 of an f tile; while waiting it
-// HELPS BUILD it: once acc shows all arrivals, its 32 lanes grab 32-entry
-// chunks (atomic chunk counter) and evaluate A (p/m)^gamma and
-// clamp(G exp(-p/(K m)), 0, 1) in f64 (R9, R11), so a frame's 24 chunks are
-// built by the producers that are waiting for them.  The producer grabs a
-// new tile only after the table of its oldest unfinished tile is complete,
-// so every grabbed tile's pass 1 runs without waiting on anything: with at
-// most 2 tiles per CTA in flight, a frame of <= 2 x grid tiles always
-// completes (no deadlock; larger frames take the step kernel).
+// (1 << 40) + its partial sum to the frame's acc word.  The table warp of
+// every SM walks the frames in order and, once a frame's acc shows all
+// arrivals, builds 16-entry chunks of its table (lanes 0-15 A (p/m)^gamma,
+// lanes 16-31 clamp(G exp(-p/(K m)), 0, 1), f64 rounded once: R9, R11); a
+// producer needing a frame's table helps build the remaining chunks, then
+// acquires it (an acquire load on its lane 0 or 1) and bulk-copies it into
+// its LUT buffer as part of the pass-2 stage.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
@@ -118,7 +119,7 @@ __device__ __forceinline__ uint32_t tile_bytes_r(int nw, int rows) {
 
 #ifdef SHARP_DIAG_RES  // diagnostics build only: wait-cycle counters
 __device__ unsigned long long g_rd[16];
-__shared__ long long rd_tma[4], rd_lut[4], rd_a[4], rd_b[4];  // producer clocks per stage
+__shared__ long long rd_tma[4], rd_lut[4];  // producer clocks per stage
 #define RD_ADD(i, v) atomicAdd(&g_rd[i], (unsigned long long)(v))
 #else
 #define RD_ADD(i, v)
