@@ -338,7 +338,8 @@ int sharp_get_kernel_times(sharp_ctx *ctx, sharp_kernel_times *t);
 
 /* ---- Kernel paths: the optimisation ladder of PAPER.md sec. V (Fig. 12,
  * Fig. 14), every rung bit-identical to the oracle.
- *   SHARP_PATH_AUTO     the resident kernel where it applies, else the step kernel, else the
+ *   SHARP_PATH_AUTO     the TMA kernels where they apply -- the resident kernel for launches of
+ *                       1 to 100 Mpx, the step kernel otherwise (measured crossovers) -- else the
  *                       two-pass path (default)
  *   SHARP_PATH_STEP     one persistent TMA-staged launch per batch (kernels_tma.cu): pass 1,
  *                       per-frame LUT and pass 2 as dynamically scheduled tasks with

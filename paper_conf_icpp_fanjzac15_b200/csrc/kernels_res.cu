@@ -787,7 +787,23 @@ cudaError_t launch_batch_res(const BatchLaunch &a, int W, int H, const Params &p
   // tiles need no padding)
   sp.pad = 0;
   sp.npos = sp.pad ? a.n * sp.pad : sp.ntasks;
-  res_kernel<<<grid, kThreadsR, kResSmem, stream>>>(m1A, m1B, m2A, m2B, sp);
+  // A COOPERATIVE launch: the static schedule needs every CTA resident at
+  // once (a CTA waits for tables that other CTAs' pass-1 tiles complete), and
+  // a cooperative launch is scheduled only as a whole -- two of these kernels
+  // on concurrent streams, or beside a persistent step kernel, cannot each
+  // hold part of the SMs and wait on their missing halves.
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreadsR);
+  cfg.dynamicSmemBytes = kResSmem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, res_kernel, m1A, m1B, m2A, m2B, sp);
+  if (e != cudaSuccess) return e;
   return cudaGetLastError();
 }
 

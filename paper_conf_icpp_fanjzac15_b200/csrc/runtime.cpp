@@ -49,6 +49,10 @@ constexpr size_t kL2ChunkBudget = 24u << 20;  // input bytes per chunk kept L2-r
 // ceiling with both directions busy 43.3 ms; tools/e2e_sweep.py).
 constexpr size_t kHostStepChunkBudget = 48u << 20;
 constexpr int kMaxSlots = 8;
+// SHARP_PATH_AUTO's choice of the TMEM-resident kernel (launch pixels), from
+// tools/step_time.py sweeps on B200: it wins from ~1 Mpx (below, its one
+// 16-warp CTA per SM costs more than it saves) up to ~100 Mpx per launch.
+constexpr double kResAutoMinPx = 1.0e6, kResAutoMaxPx = 1.0e8;
 
 struct Slot {
   cudaStream_t stream = nullptr;
@@ -399,8 +403,12 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
                    "and no per-pixel reading switch (R2, R5, R14)");
   const bool tma = tma_family(ctx->path) && tma_ok;
   // the resident kernel (TMEM pEdge) for frames up to ~10 Mpx, else the step kernel
-  // (AUTO takes it once it beats the step kernel: see DESIGN.md sec. 7)
-  const bool res = tma && ctx->path == SHARP_PATH_RES && sharp::res_supported(w, h, n);
+  // AUTO takes the resident kernel where it measured faster than the step
+  // kernel: launches of 1 .. 100 Mpx (single images from 1080p, batches up
+  // to ~48 x 1080p / 12 x 4K), else the step kernel.
+  const double px = (double)n * fb;
+  const bool res_auto = ctx->path == SHARP_PATH_AUTO && px > kResAutoMinPx && px <= kResAutoMaxPx;
+  const bool res = tma && (ctx->path == SHARP_PATH_RES || res_auto) && sharp::res_supported(w, h, n);
   if (ctx->path == SHARP_PATH_RES && !res)
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
                    "SHARP_PATH_RES needs the step kernel's geometry and at most 2 x (resident grid) tiles of "
