@@ -357,7 +357,7 @@ struct Strides {
 
 int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, const sharp::Params &prm,
                    uint8_t *dout, cudaStream_t st, Slot &slot, size_t chunk, size_t frame_base, int *launches,
-                   unsigned int *tc, const Strides &str = Strides()) {
+                   unsigned int *tc, const Strides &str = Strides(), bool pipelined = false) {
   const size_t fb = (size_t)w * h;
   if (!str.dense() && (ctx->path == SHARP_PATH_STAGED || ctx->path == SHARP_PATH_FUSED || ctx->path == SHARP_PATH_FUSED_EXP))
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s", "strided frames on the staged / scalar fused paths");
@@ -407,7 +407,9 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   // kernel: launches of 1 .. 100 Mpx (single images from 1080p, batches up
   // to ~48 x 1080p / 12 x 4K), else the step kernel.
   const double px = (double)n * fb;
-  const bool res_auto = ctx->path == SHARP_PATH_AUTO && px > kResAutoMinPx && px <= kResAutoMaxPx;
+  // (not for the host pipeline's chunks: its slots' kernels overlap on
+  // several streams, which a cooperative launch would serialise)
+  const bool res_auto = ctx->path == SHARP_PATH_AUTO && !pipelined && px > kResAutoMinPx && px <= kResAutoMaxPx;
   const bool res = tma && (ctx->path == SHARP_PATH_RES || res_auto) && sharp::res_supported(w, h, n);
   if (ctx->path == SHARP_PATH_RES && !res)
     return set_err(ctx, SHARP_EUNSUPPORTED, "%s",
@@ -531,7 +533,7 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
       }
       uint8_t *ddst = (kout == kDevice) ? out + f0 * fb : sl.d_out;
       if ((rc = enqueue_device(ctx, dsrc, (int)cn, w, h, prm, ddst, sl.stream, sl, cn, f0, &launches,
-                               ctx->tcounters + 2 * c)))
+                               ctx->tcounters + 2 * c, Strides(), true)))
         return rc;
       if (kout != kDevice) {
         uint8_t *hdst = (kout == kPinned) ? out + f0 * fb : sl.h_out;
