@@ -12,7 +12,7 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smok
 timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
 for wh in 512x512 1920x1080 3840x2160 7680x4320; do
   w=${wh%x*}; h=${wh#*x}
-  timeout 300 python bench.py --frames 1 --width $w --height $h --steps 200 --warmup 10 --e2e-steps 20 --no-cpu \
+  timeout 300 python bench.py --frames 1 --width $w --height $h --steps 200 --warmup 10 --e2e-steps 20 \
     > gpurun_out/single_$wh.json 2>> gpurun_out/single.err
 done
 timeout 300 python bench.py --frames 32 --width 3840 --height 2160 --steps 20 --warmup 3 --e2e-steps 3 --no-cpu \
