@@ -1545,8 +1545,8 @@ const char *sharp_strerror(int code) {
 const char *sharp_last_error(const sharp_ctx *ctx) { return ctx ? ctx->err : "no context"; }
 
 const char *sharp_version(void) {
-  return "libsharp 0.2 (sm_100a; persistent TMA step kernel, two-pass and staged paths; general layouts; "
-         "reading switches; peer-memory row bands)";
+  return "libsharp 0.3 (sm_100a; persistent TMA step kernel, TMEM-resident kernel, two-pass, scalar fused and "
+         "staged paths; general layouts; reading switches; multi-device contexts; peer-memory row bands)";
 }
 
 }  // extern "C"

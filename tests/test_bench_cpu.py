@@ -6,6 +6,8 @@ import importlib.util
 import json
 import os
 import subprocess
+
+import pytest
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -76,3 +78,17 @@ def test_gpus_n_beyond_visible_fails_loudly():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--steps", "1"],
                        capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
     assert r.returncode != 0 and "visible" in r.stderr
+
+
+def test_committed_profile_is_keyed_on_the_kernel_sources(monkeypatch):
+    """bench.py reports ncu-derived traffic / instruction counts only from a
+    capture of the CURRENT kernel sources (profiles/*/traffic*.json carry the
+    sources' sha256); a stale capture yields None, never old numbers."""
+    b = load_bench()
+    cur = b.committed_profile("step")
+    if cur is not None:
+        assert cur["source_sha256"] == b.kernel_source_hash("step")
+        assert b.traffic_per_launch(1000.0) == pytest.approx(1000.0 * cur["dram_bytes_per_px"])
+    monkeypatch.setattr(b, "kernel_source_hash", lambda kind: "0" * 64)
+    assert b.committed_profile("step") is None
+    assert b.traffic_per_launch(1000.0) is None and b.issue_profile() is None
