@@ -69,17 +69,26 @@ def exchange_halos(own, h, row0, row1, group=None):
             raise ValueError("a single rank must own the whole image")
         return band
     ops = []
-    up_recv = band[:top] if top else None
-    dn_recv = band[top + rows:] if bot else None
+    # gloo moves host tensors only (a CUDA band under gloo -- the one-GPU
+    # test hook -- is staged through host copies); NCCL moves device memory
+    host = own.is_cuda and dist.get_backend(group) == "gloo"
+    stage = (lambda t: t.cpu()) if host else (lambda t: t)
+    up_recv = stage(band[:top]) if top else None
+    dn_recv = stage(band[top + rows:]) if bot else None
     peer = (lambda r: dist.get_global_rank(group, r)) if group is not None else (lambda r: r)
     if rank > 0:  # exchange with the band above: it needs our first rows, we need its last
-        ops.append(dist.P2POp(dist.isend, own[:HALO].contiguous(), peer(rank - 1), group))
+        ops.append(dist.P2POp(dist.isend, stage(own[:HALO].contiguous()), peer(rank - 1), group))
         ops.append(dist.P2POp(dist.irecv, up_recv, peer(rank - 1), group))
     if rank < world - 1:
-        ops.append(dist.P2POp(dist.isend, own[rows - HALO:].contiguous(), peer(rank + 1), group))
+        ops.append(dist.P2POp(dist.isend, stage(own[rows - HALO:].contiguous()), peer(rank + 1), group))
         ops.append(dist.P2POp(dist.irecv, dn_recv, peer(rank + 1), group))
     for req in dist.batch_isend_irecv(ops):
         req.wait()
+    if host:
+        if top:
+            band[:top].copy_(up_recv)
+        if bot:
+            band[top + rows:].copy_(dn_recv)
     return band
 
 
@@ -98,8 +107,13 @@ def sharpen_band(sharpener, band, w, h, row0, row1, params=None, out=None, group
     s = torch.zeros(1, dtype=torch.int64, device=band.device)  # u64 bits; S < 2^40
     sharpener.band_edge_sum(band, w, h, row0, row1, s)
     world, _ = _world(group)
-    if world > 1:
-        dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)  # the L174 reduction across bands
+    if world > 1:  # the L174 reduction across bands (host-staged under gloo)
+        if s.is_cuda and dist.get_backend(group) == "gloo":
+            t = s.cpu()
+            dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+            s.copy_(t)
+        else:
+            dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)
     sharpener.band_sharpen(band, w, h, row0, row1, s, out, params)
     return out, s
 
