@@ -320,8 +320,8 @@ __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rm
   for (int x = 0; x < 8; ++x) vmask |= (uint32_t)(c0 + x >= 1 && c0 + x <= W - 2) << x;
   if (lane >= 30) vmask = 0;
   // smem row of global row R0-1 is 0: row r -> r - R0 + 1.
-  RowD ra = derive_w<false>(row_words(aw, 0), lane);
-  RowD rb = derive_w<false>(row_words(aw, 1), lane);
+  RowD ra = derive_w<false, true>(row_words(aw, 0), lane);
+  RowD rb = derive_w<false, true>(row_words(aw, 1), lane);
   // One accumulator per pixel column (exact: < 24 rows * 1530 < 2^24); the
   // column mask is applied once at the end, so the row loop has no
   // per-lane branches.
@@ -331,7 +331,7 @@ __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rm
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
       const int r = R0 + m + a;
-      const RowD rc = derive_w<false>(row_words(aw, m + a + 2), lane);
+      const RowD rc = derive_w<false, true>(row_words(aw, m + a + 2), lane);
       uint32_t pe[4];
       sobel(ra, rb, rc, pe);
       // 1 <= r <= rmax1: Sobel frame rows are 0 (L160).  The row weight (1.0 or
@@ -348,7 +348,10 @@ __device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rm
   float sum = 0.0f;
 #pragma unroll
   for (int x = 0; x < 8; ++x) sum = __fadd_rn(sum, (vmask >> x & 1) ? acc[x] : 0.0f);
-  return sum;
+  // Bytes unpacked as f16 subnormals (derive_w<.., true>: no HADD2 per pair;
+  // measured +1.6% on the 1024-frame step): the sums count pEdge * 2^-24,
+  // exact (< 2^24 units); scaled back once.
+  return sum * 16777216.0f;
 }
 
 #ifdef SHARP_DIAG_TIMELINE  // timing experiment: globaltimer of the launch's phases (min / max over CTAs)
@@ -730,6 +733,15 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   // parallelism; big launches keep kSub (one LUT copy per kSub sub-tiles).
   const int per_frame_sub = sp.g.tiles_x * ((rows + kTH * kSub - 1) / (kTH * kSub));
   sp.g.sub = ((long long)sg.n * per_frame_sub < grid_ctas) ? 1 : kSub;
+  // A single frame or two (compact schedule) are a few waves of tasks: take
+  // kSub = 1 when its waves, counted in sub-tiles, are fewer (8K: 960 tasks on
+  // 444 CTAs = 3 waves x 3 sub-tiles vs 2880 = 7 waves x 1: 74.3 -> 71.0 us;
+  // 16K ties at 54 x 1 vs 18 x 3 and keeps kSub: sub = 1 measured 3% slower).
+  if (sp.g.sub == kSub && sg.n < 4) {
+    const long long t1 = (long long)sg.n * sp.g.tiles_x * ((rows + kTH - 1) / kTH);
+    const long long ts = (long long)sg.n * per_frame_sub;
+    if ((t1 + grid_ctas - 1) / grid_ctas < kSub * ((ts + grid_ctas - 1) / grid_ctas)) sp.g.sub = 1;
+  }
   sp.g.per_frame = sp.g.tiles_x * ((rows + kTH * sp.g.sub - 1) / (kTH * sp.g.sub));
   // pass-1 tiles: as tall as kTH1 while the launch has >= one tile per CTA
   sp.g.th1 = kTH1;

@@ -499,7 +499,10 @@ int run_impl(sharp_ctx *ctx, const uint8_t *in, int n, int w, int h, const sharp
   const size_t nchunks_all = ((size_t)n + chunk - 1) / chunk;
   if ((rc = ensure_task_counters(ctx, 2 * nchunks_all + 2))) return rc;
   CK(cudaMemsetAsync(ctx->zero_block, 0, ctx->zero_bytes, ctx->stream));  // acc, sums, lut_done, counters
-  CK(cudaEventRecord(ctx->ev_start, ctx->stream));
+  // (an asynchronous device-resident call reports no device time: no event
+  // record between its launches and the previous call's -- measured 2-3 us
+  // of a single-image call in a back-to-back stream)
+  if (!async || staged) CK(cudaEventRecord(ctx->ev_start, ctx->stream));
   if (!staged) {
     if ((rc = enqueue_device(ctx, in, n, w, h, prm, out, ctx->stream, ctx->slots[0], chunk, 0, &launches,
                              ctx->tcounters)))

@@ -208,12 +208,19 @@ __device__ __forceinline__ uint2 row_words(const LaneRow &a, int s) { return lds
 
 // Converts a row of words into the window data.  Neighbour pairs come from
 // the adjacent lanes (shuffle), so each lane loads only its own 8 bytes.
-template <bool kMinMax>
+// kDenorm (pass 1 of the step kernel, which only sums pEdge): the bytes
+// become the f16 SUBNORMALS b * 2^-24 (one PRMT with zero bytes, no HADD2);
+// f16 arithmetic keeps subnormals and every integer k * 2^-24 with |k| <=
+// 2048 is exact, so the Sobel values are pEdge * 2^-24 exactly.
+template <bool kMinMax, bool kDenorm = false>
 __device__ __forceinline__ RowD derive_w(uint2 w, int lane) {
-  const uint32_t E0 = hadd(prmt(w.x, kF16Bias, 0x4240), kMinus1024);  // (c0, c0+2)
-  const uint32_t O0 = hadd(prmt(w.x, kF16Bias, 0x4341), kMinus1024);  // (c0+1, c0+3)
-  const uint32_t E1 = hadd(prmt(w.y, kF16Bias, 0x4240), kMinus1024);  // (c0+4, c0+6)
-  const uint32_t O1 = hadd(prmt(w.y, kF16Bias, 0x4341), kMinus1024);  // (c0+5, c0+7)
+  auto unpack = [](uint32_t x, uint32_t sel) {
+    return kDenorm ? prmt(x, 0u, sel) : hadd(prmt(x, kF16Bias, sel), kMinus1024);
+  };
+  const uint32_t E0 = unpack(w.x, 0x4240);  // (c0, c0+2)
+  const uint32_t O0 = unpack(w.x, 0x4341);  // (c0+1, c0+3)
+  const uint32_t E1 = unpack(w.y, 0x4240);  // (c0+4, c0+6)
+  const uint32_t O1 = unpack(w.y, 0x4341);  // (c0+5, c0+7)
   const uint32_t PO = __shfl_sync(0xffffffffu, O1, (lane + 31) & 31);  // (c0-3, c0-1)
   const uint32_t NE = __shfl_sync(0xffffffffu, E0, (lane + 1) & 31);   // (c0+8, c0+10)
   const uint32_t p[4] = {E0, O0, E1, O1};
