@@ -19,9 +19,9 @@
 //
 // CTA = 4 compute warps + 1 producer warp.  A pass-1/2 task is a CTA tile of
 // 4 warp tiles side by side; a warp tile is 240 output columns x 12 rows
-// (pass 2) or 18 rows (pass 1).  The producer issues two TMA boxes per warp
-// tile (out-of-image pixels are zero-filled: no bounds checks in the pixel
-// loops) plus a bulk copy of the frame's LUT, into one of two smem stages
+// (pass 2) or 18 rows (pass 1).  The producer issues one 256-column TMA box
+// per warp tile (out-of-image pixels are zero-filled: no bounds checks in the
+// pixel loops) plus a bulk copy of the frame's LUT, into one of two smem stages
 // guarded by full/empty mbarriers -- no CTA-wide barrier in the steady state.
 // Each lane owns 8 adjacent columns and walks down the rows with a 3-row
 // window unrolled by 3 (no register moves); lanes 30 and 31 fetch the
@@ -68,7 +68,42 @@ constexpr int kSub = SHARP_P2_SUB;
 #define SHARP_STAGES 2  // measured: 3 stages +0.3%, 2 stages (this layout) +0.6% vs the old layout
 #endif
 constexpr int kStages = SHARP_STAGES;          // smem ring depth
-constexpr int kStage = (kRegB + kPitchB * kRows2 + 127) / 128 * 128;  // one stage
+// Uniform-pitch stage layout: slot w holds one 256-column box; warps 0..2
+// load columns C0w-16 .. C0w+239 (own columns at slot column kCol0), the last
+// warp loads C0w .. C0w+255 (own columns at slot column 0, its right halo
+// C0w+240.. in its own slot), so every lane -- halo lanes included -- reads
+// its rows at pitch kPitch: row addresses are one base register plus
+// immediates, and no 16-column region-B box is needed.
+constexpr int kStage = kWarpsT * kSlot;  // one stage
+__device__ __forceinline__ int own_col(int w) { return w == kWarpsT - 1 ? 0 : kCol0; }
+struct LaneRowC {
+  uint32_t base;
+};
+__device__ __forceinline__ LaneRowC lane_row_s(uint32_t stage, int warp, int lane) {
+  const uint32_t own = stage + (uint32_t)(warp * kSlot + own_col(warp));
+  if (lane < 30) return LaneRowC{own + 8u * (uint32_t)lane};
+  if (lane == 30)  // right halo C0w+240..247
+    return LaneRowC{warp == kWarpsT - 1 ? own + (uint32_t)kTW
+                                        : stage + (uint32_t)((warp + 1) * kSlot + own_col(warp + 1))};
+  // lane 31: left halo C0w-8..C0w-1 (the previous warp's slot for the last warp)
+  return LaneRowC{warp == kWarpsT - 1 ? stage + (uint32_t)((warp - 1) * kSlot + kCol0 + kTW - 8) : own - 8u};
+}
+__device__ __forceinline__ uint2 row_words(const LaneRowC &a, int s) { return lds_u64(a.base + (uint32_t)(s * kPitch)); }
+__device__ __forceinline__ float4 dblock(const LaneRowC &a, int s, int lane) {
+  const uint32_t o = a.base + (uint32_t)(s * kPitch);
+  const uint2 r0 = lds_u64(o), r1 = lds_u64(o + kPitch), r2 = lds_u64(o + 2 * kPitch), r3 = lds_u64(o + 3 * kPitch);
+  const float d0 = (float)blk4(r0.x, r1.x, r2.x, r3.x);
+  const float d1 = (float)blk4(r0.y, r1.y, r2.y, r3.y);
+  const float dm1 = __shfl_sync(0xffffffffu, d1, (lane + 31) & 31);
+  const float d2 = __shfl_sync(0xffffffffu, d0, (lane + 1) & 31);
+  return make_float4(dm1, d0, d1, d2);
+}
+__device__ __forceinline__ uint32_t tile_bytes_s(int nw, int rows) { return (uint32_t)(nw * kPitch * rows); }
+__device__ __forceinline__ void tma_tiles_s(uint32_t st, const CUtensorMap *mapA, const CUtensorMap *, int C0, int nw,
+                                            int r, int f, uint32_t bar, uint64_t policy) {
+  for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, mapA, C0 + w * kTW - own_col(w), r, f, bar, policy);
+}
+using LR = LaneRowC;
 constexpr int kLutOff = kStages * kStage;      // two LUT buffers after the stages
 constexpr int kBarOff = kLutOff + 2 * kLutBytes;
 constexpr int kSmem = kBarOff + 16 * kStages;  // full + empty barrier per stage
@@ -176,8 +211,7 @@ template <bool kRingRows>
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
                                        const float4 &D0, const float4 &D1, uint32_t lut_q,
                                        uint8_t *orow, uint64_t pol_out, bool store, int r, int c0, int W, int H,
-                                       bool edge_warp,
-                                       int edge) {
+                                       bool edge_warp, int edge) {
   uint32_t pe[4], MX[4], MN[4];
   sobel(ra, rb, rc, pe);
 #pragma unroll
@@ -246,7 +280,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   // W-2,W-1 in the lane with c0 == W-8.
   const int edge = !active ? 0 : (c0 == 0 ? 1 : (c0 == W - 8 ? 2 : 0));
   const bool edge_warp = (C0w == 0) || (C0w <= W - 8 && W - 8 < C0w + kTW);
-  LaneRow aw = lane_row(ring.stage(s), warp, lane);
+  LR aw = lane_row_s(ring.stage(s), warp, lane);
   const uint64_t pol_out = policy_evict_first();  // output: written once, never re-read
   // LDS address of entry k = pEdge/2: the f32 bits of (2^21 + pEdge) plus
   // lut_q.  The vote makes the LUT-buffer choice -- and so lut_q -- provably
@@ -274,7 +308,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
     const int R0k = R0 + k * kTH;
     if (k) {  // next sub-tile: same rows layout in the next stage; state carried
       ring.wait_full(s + k);
-      aw = lane_row(ring.stage(s + k), warp, lane);
+      aw = lane_row_s(ring.stage(s + k), warp, lane);
     }
     const int rend = min(R0k + kTH, row_hi);
     const int rend_l = active ? rend : R0k;  // this lane stores rows < rend_l
@@ -310,48 +344,58 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 // without pairwise f16 row sums, is no faster -- pass 1 waits on its TMA
 // loads more than on issue -- and the 6-row variant's extra code is 5%
 // slower.)
-__device__ __forceinline__ float p1_warp(uint32_t stage, int warp, int W, int rmax1, int th1, int C0w, int R0,
-                                        int lane) {
+// Bytes are unpacked as f16 SUBNORMALS (derive_w<.., true>): every Sobel value
+// is k * 2^-24 with |k| < 2048 exactly, and for such values the f16 BIT
+// PATTERN is the integer k (subnormals, and the first normal binade whose
+// spacing is still 2^-24).  pEdge <= 1530, so each f16x2 word of pe holds two
+// pEdge values as u16 integers: the row sums are plain 32-bit integer adds of
+// the words (each half stays < 2^16: <= 42 rows x 1530), two pixels per add,
+// three rows per IADD3 pair; no conversions.
+__device__ __forceinline__ uint32_t p1_warp(uint32_t stage, int warp, int W, int rmax1, int th1, int C0w, int R0,
+                                           int lane) {
   const int c0 = C0w + 8 * lane;
-  const LaneRow aw = lane_row(stage, warp, lane);
-  // Sobel-body pixels of this lane (not frame columns, not beyond the image).
-  uint32_t vmask = 0;
-#pragma unroll
-  for (int x = 0; x < 8; ++x) vmask |= (uint32_t)(c0 + x >= 1 && c0 + x <= W - 2) << x;
-  if (lane >= 30) vmask = 0;
+  const LR aw = lane_row_s(stage, warp, lane);
   // smem row of global row R0-1 is 0: row r -> r - R0 + 1.
   RowD ra = derive_w<false, true>(row_words(aw, 0), lane);
   RowD rb = derive_w<false, true>(row_words(aw, 1), lane);
-  // One accumulator per pixel column (exact: < 24 rows * 1530 < 2^24); the
-  // column mask is applied once at the end, so the row loop has no
-  // per-lane branches.
-  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  uint32_t acc[4] = {0u, 0u, 0u, 0u};  // acc[i] = (sum of pEdge of pair i's low pixel, ... high pixel)
 #pragma unroll 1
   for (int m = 0; m < th1; m += 3) {
+    uint32_t pe[3][4];
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
-      const int r = R0 + m + a;
       const RowD rc = derive_w<false, true>(row_words(aw, m + a + 2), lane);
-      uint32_t pe[4];
-      sobel(ra, rb, rc, pe);
-      // 1 <= r <= rmax1: Sobel frame rows are 0 (L160).  The row weight (1.0 or
-      // 0.0 as f16) goes into a mixed-precision FMA -- no predicated updates
-      // (they cost a move per accumulator and row).
-      const uint16_t on = ((unsigned)(r - 1) < (unsigned)rmax1) ? (uint16_t)0x3C00u : (uint16_t)0u;
-#pragma unroll
-      for (int x = 0; x < 8; ++x)
-        acc[x] = fma_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), on, acc[x]);
+      sobel(ra, rb, rc, pe[a]);
       ra = rb;
       rb = rc;
     }
-  }
-  float sum = 0.0f;
+    // Rows 1 <= r <= rmax1 only (L160: the frame rows' pEdge is 0).  The
+    // test is warp-uniform (a vote): all three rows valid is the common case.
+    const int r = R0 + m;
+    if (__all_sync(0xffffffffu, r >= 1 && r + 2 <= rmax1)) {
 #pragma unroll
-  for (int x = 0; x < 8; ++x) sum = __fadd_rn(sum, (vmask >> x & 1) ? acc[x] : 0.0f);
-  // Bytes unpacked as f16 subnormals (derive_w<.., true>: no HADD2 per pair;
-  // measured +1.6% on the 1024-frame step): the sums count pEdge * 2^-24,
-  // exact (< 2^24 units); scaled back once.
-  return sum * 16777216.0f;
+      for (int i = 0; i < 4; ++i) acc[i] = acc[i] + pe[0][i] + pe[1][i] + pe[2][i];
+    } else {
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+        if ((unsigned)(r + a - 1) < (unsigned)rmax1) {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) acc[i] += pe[a][i];
+        }
+    }
+  }
+  // Sobel-body columns of this lane only (not the frame columns 0 / W-1, not
+  // beyond the image, not the halo lanes): x = 4 (i >> 1) + (i & 1) + 2 half.
+  uint32_t sum = 0;
+  if (lane < 30) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int x = 4 * (i >> 1) + (i & 1);
+      if (c0 + x >= 1 && c0 + x <= W - 2) sum += acc[i] & 0xffffu;
+      if (c0 + x + 2 >= 1 && c0 + x + 2 <= W - 2) sum += acc[i] >> 16;
+    }
+  }
+  return sum;
 }
 
 #ifdef SHARP_DIAG_TIMELINE  // timing experiment: globaltimer of the launch's phases (min / max over CTAs)
@@ -478,8 +522,8 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
             if (waited) fence_proxy_async_global();  // peer-written rows before the TMA reads them
           }
           stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
-          mbar_expect_tx(full, tile_bytes(nw, kRows1));
-          tma_tiles(st, &map1A, &map1B, C0, nw, R0 - 1 - g.y0, d.y, full, pol_keep);
+          mbar_expect_tx(full, tile_bytes_s(nw, kRows1));
+          tma_tiles_s(st, &map1A, &map1B, C0, nw, R0 - 1 - g.y0, d.y, full, pol_keep);
         } else if (d.x == kP2) {
           const int R0k = R0 + k * kTH;
           if (kFused && sp.halo_on) {  // (tile loads go out before the LUT wait: check the halo flags here too)
@@ -502,7 +546,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           // later one only after single-stage pass-2 tasks.
           const int tl = lut_last[j & 1];
           if (k == 0 && tl > s - kStages) mbar_wait(ring.empty0 + 8u * Ring::buf(tl), Ring::phase(tl));
-          mbar_expect_tx(full, tile_bytes(nw, kRows2) + lut_bytes);
+          mbar_expect_tx(full, tile_bytes_s(nw, kRows2) + lut_bytes);
 #ifndef SHARP_OLD_LUT_FENCE
           // The frame's LUT (its LUT tasks were grabbed rounds earlier) is
           // normally complete: then the table copy goes out first.  Acquire
@@ -514,14 +558,14 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
             fence_proxy_async_global();
             bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
           }
-          tma_tiles(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
+          tma_tiles_s(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
           if (lut_bytes && !lut_now) {
             while (ld_acquire(&sp.lut_done[d.y]) < want) __nanosleep(kPollNs);
             fence_proxy_async_global();
             bulk_copy(lutbase + (uint32_t)((j & 1) * kLutBytes), sp.luts + (size_t)d.y * kLutSize, kLutBytes, full);
           }
 #else
-          tma_tiles(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
+          tma_tiles_s(st, &map2A, &map2B, C0, nw, R0k - 4 - g.y0, d.y, full, pol_drop);
           if (lut_bytes) {
             // the frame's LUT tasks (grabbed earlier) have finished
             while (ld_relaxed_u32(&sp.lut_done[d.y]) < (unsigned)(kLutTasks * kWarpsT)) __nanosleep(kPollNs);
@@ -606,7 +650,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
-      const float acc = (C0w < g.W) ? p1_warp(ring.stage(s), warp, g.W, g.rmax1, g.th1, C0w, R0, lane) : 0.0f;
+      const auto acc = (C0w < g.W) ? p1_warp(ring.stage(s), warp, g.W, g.rmax1, g.th1, C0w, R0, lane) : 0;
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
       // atomic per warp adding (1 << 40) + partial: the frame's arrival count
       // and sum in one word, so its LUT tasks can tell when S is complete

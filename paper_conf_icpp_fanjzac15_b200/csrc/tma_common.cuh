@@ -30,18 +30,18 @@ constexpr unsigned kPollNs = 100;  // dependency polling interval of the produce
 // A warp tile needs columns C0w-8 .. C0w+247.  TMA box starts must be
 // 16-byte aligned in the innermost dimension and a box dimension is at most
 // 256, so a warp tile is fetched as one 256-column box of the [n][H][W]
-// frames, region A = columns C0w-16 .. C0w+239 (smem pitch 256).  Its right
-// halo C0w+240.. is the first own column of the next warp's region A (offset
-// kCol0 there); only the CTA tile's last warp needs one more box, region B =
-// 16 columns C0w+240 .. C0w+255 (smem pitch 16) after the four slots.  (When
-// the next warp has no columns, the halo lies beyond the image and only feeds
-// pixels that are either not stored or on the overridden frame column W-1.)
+// frames (region A, smem pitch 256).  The step kernel (kernels_tma.cu) loads
+// C0w-16 .. C0w+239 for warps 0..2 and C0w .. C0w+255 for the last warp, so
+// every halo lies in some warp's region A; the resident kernel
+// (kernels_res.cu) keeps a 16-column region B (pitch 16) for the last warp's
+// right halo.  (When the next warp has no columns, the halo lies beyond the
+// image and only feeds pixels that are either not stored or on the
+// overridden frame column W-1.)
 constexpr int kPitch = 256;           // region A pitch
 constexpr int kPitchB = 16;           // region B pitch
 constexpr int kCol0 = 16;             // region-A column of C0w
 constexpr int kRows2 = kTH + 8;       // pass-2 box rows: R0-4 .. R0+kTH+3
 constexpr int kSlot = kPitch * kRows2;  // per-warp smem slot: region A (128-B aligned)
-constexpr int kRegB = kWarpsT * kSlot;  // region B of the last warp
 static_assert(kSlot % 128 == 0, "TMA smem destinations must be 128-B aligned");
 static_assert(kTH % 3 == 0 && kTH % 4 == 0, "row loop is unrolled by 3, D blocks are 4 rows");
 static_assert(kLut2 <= kLutSize && 2 * (kLut2 - 1) >= 1530, "even-pEdge tables");
@@ -107,16 +107,6 @@ __device__ __forceinline__ void tma_box(uint32_t dst, const CUtensorMap *map, in
       "{%2, %3, %4}], [%5], %6;" ::"r"(dst),
       "l"(map), "r"(x), "r"(r), "r"(f), "r"(bar), "l"(policy)
       : "memory");
-}
-// The boxes of a CTA tile of nw warp tiles into stage st: region A per warp,
-// and region B (the last warp's right halo) when all kWarpsT warps have columns.
-__device__ __forceinline__ uint32_t tile_bytes(int nw, int rows) {
-  return (uint32_t)((nw * kPitch + (nw == kWarpsT ? kPitchB : 0)) * rows);
-}
-__device__ __forceinline__ void tma_tiles(uint32_t st, const CUtensorMap *mapA, const CUtensorMap *mapB, int C0, int nw,
-                                          int r, int f, uint32_t bar, uint64_t policy) {
-  for (int w = 0; w < nw; ++w) tma_box(st + w * kSlot, mapA, C0 + w * kTW - kCol0, r, f, bar, policy);
-  if (nw == kWarpsT) tma_box(st + kRegB, mapB, C0 + kWarpsT * kTW, r, f, bar, policy);
 }
 // Output store.  (Measured: an L2::cache_hint store costs ~5% of the step
 // through extra issue; plain STG.64 it is.)
@@ -191,19 +181,10 @@ __device__ __forceinline__ unsigned long long gtime_ns() {
 }
 
 // ------------------------------------------------------------- row window
-// Lane words of smem row s: lanes 0..29 own columns C0w+8l..+7 (region A);
-// lane 31 the left halo C0w-8..C0w-1 (region A); lane 30 the right halo
-// C0w+240..247 (the next warp's region A, or region B for the last warp).
+// A lane's row window in a stage: its 8 bytes of smem row s at base + s * pitch.
 struct LaneRow {
   uint32_t base, pitch;
 };
-__device__ __forceinline__ LaneRow lane_row(uint32_t stage, int warp, int lane) {
-  if (lane == 30) {
-    if (warp == kWarpsT - 1) return LaneRow{stage + (uint32_t)kRegB, (uint32_t)kPitchB};
-    return LaneRow{stage + (uint32_t)((warp + 1) * kSlot + kCol0), (uint32_t)kPitch};
-  }
-  return LaneRow{stage + (uint32_t)(warp * kSlot + kCol0 + 8 * (lane < 31 ? lane : -1)), (uint32_t)kPitch};
-}
 __device__ __forceinline__ uint2 row_words(const LaneRow &a, int s) { return lds_u64(a.base + (uint32_t)s * a.pitch); }
 
 // Converts a row of words into the window data.  Neighbour pairs come from
