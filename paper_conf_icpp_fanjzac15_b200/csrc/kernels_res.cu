@@ -186,40 +186,55 @@ __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.
 // TMEM row j = r - R0 of the slot, and the warp's partial sum of the Sobel
 // body (rows 1..rmax1, columns 1..W-2; L160: the frame is 0).
 // (aw: the warp column's lane words; sb: stage row of image row R0 - 1.)
-__device__ __forceinline__ float p1_tile(const LaneRow &aw0, int sb, int W, int rmax1, int C0w, int R0, int lane,
-                                         uint32_t tslot) {
+// The sums: with the bytes unpacked as f16 subnormals, the f16 bit pattern of
+// every pEdge value (<= 1530 < 2048 units of 2^-24) is the integer pEdge, so
+// each f16x2 word is a u16x2 pair of pEdge values and the row sums are plain
+// 32-bit integer adds, two pixels per add (halves stay < 2^16).
+static_assert(kDenorm, "p1_tile sums the subnormal bit patterns");
+__device__ __forceinline__ uint32_t p1_tile(const LaneRow &aw0, int sb, int W, int rmax1, int C0w, int R0, int lane,
+                                            uint32_t tslot) {
   const int c0 = C0w + 8 * lane;
   const LaneRow aw{aw0.base + (uint32_t)sb * aw0.pitch, aw0.pitch};  // row offsets below are compile-time
   RowD ra = derive_w<false, kDenorm>(row_words(aw, 0), lane);
   RowD rb = derive_w<false, kDenorm>(row_words(aw, 1), lane);
-  float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};  // exact: < 12 rows * 1530
+  uint32_t acc[4] = {0u, 0u, 0u, 0u};  // per pair: (sum of the low pixel, of the high pixel)
 #pragma unroll 1
   for (int m = 0; m < kT; m += 3) {
+    uint32_t pe[3][4];
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
-      const int r = R0 + m + a;
       const RowD rc = derive_w<false, kDenorm>(row_words(aw, m + a + 2), lane);
-      uint32_t pe[4];
-      sobel(ra, rb, rc, pe);
-      tmem_st4(tslot + (uint32_t)(4 * (m + a)), pe);
-      const uint16_t on = ((unsigned)(r - 1) < (unsigned)rmax1) ? (uint16_t)0x3C00u : (uint16_t)0u;
-#pragma unroll
-      for (int x = 0; x < 8; ++x)
-        acc[x] = fma_f32_f16(half_of(x) ? hi16(pe[pair_of(x)]) : lo16(pe[pair_of(x)]), on, acc[x]);
+      sobel(ra, rb, rc, pe[a]);
+      tmem_st4(tslot + (uint32_t)(4 * (m + a)), pe[a]);
       ra = rb;
       rb = rc;
     }
+    // rows 1 <= r <= rmax1 only (L160); warp-uniform (a vote)
+    const int r = R0 + m;
+    if (__all_sync(0xffffffffu, r >= 1 && r + 2 <= rmax1)) {
+#pragma unroll
+      for (int i = 0; i < 4; ++i) acc[i] = acc[i] + pe[0][i] + pe[1][i] + pe[2][i];
+    } else {
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+        if ((unsigned)(r + a - 1) < (unsigned)rmax1) {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) acc[i] += pe[a][i];
+        }
+    }
   }
-  // Sobel body columns only (L160: columns 0 and W-1 are frame; W % 8 == 0,
-  // so they are x = 0 of the lane at c0 = 0 and x = 7 of the lane at
-  // c0 = W-8); halo lanes and lanes beyond the image add nothing.  Exact
-  // (integers < 2^24), so the order of the additions does not matter.
-  float sum = __fadd_rn(__fadd_rn(__fadd_rn(acc[0], acc[1]), __fadd_rn(acc[2], acc[3])),
-                        __fadd_rn(__fadd_rn(acc[4], acc[5]), __fadd_rn(acc[6], acc[7])));
-  if (c0 == 0) sum = __fsub_rn(sum, acc[0]);
-  if (c0 == W - 8) sum = __fsub_rn(sum, acc[7]);
-  if (lane >= 30 || c0 >= W) sum = 0.0f;
-  if (kDenorm) sum *= 16777216.0f;  // subnormal units pEdge * 2^-24 (exact: < 2^24 units)
+  // Sobel body columns only (L160: columns 0 and W-1 are frame); halo lanes
+  // and lanes beyond the image add nothing.  Pair i holds x = 4 (i >> 1) +
+  // (i & 1) (low half) and x + 2 (high half).
+  uint32_t sum = 0;
+  if (lane < 30) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int x = 4 * (i >> 1) + (i & 1);
+      if (c0 + x >= 1 && c0 + x <= W - 2) sum += acc[i] & 0xffffu;
+      if (c0 + x + 2 >= 1 && c0 + x + 2 <= W - 2) sum += acc[i] >> 16;
+    }
+  }
   tmem_wait_st();  // the slot's rows are in TMEM before this warp's pass 2 reads them
   return sum;
 }
@@ -712,11 +727,11 @@ __global__ void __launch_bounds__(kThreadsR, 1)
     const int f = d.y, C0w = d.z + wc * kTW, R0w = d.w;
     const uint32_t tslot = tmem_w + (uint32_t)(aux.x * kSlotCols);
     if (d.x == kRP1) {
-      const float acc =
-          C0w < W ? p1_tile(lane_row_r(ring.stage(s), wc, lane, 3), 3, W, sp.rmax1, C0w, R0w, lane, tslot) : 0.0f;
+      const uint32_t acc =
+          C0w < W ? p1_tile(lane_row_r(ring.stage(s), wc, lane, 3), 3, W, sp.rmax1, C0w, R0w, lane, tslot) : 0u;
       // Reduction (sec. V-C): warp REDUX, one u64 atomic per warp adding the
       // arrival and the partial in one word (the table builders wait on it).
-      const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
+      const uint32_t ws = __reduce_add_sync(0xffffffffu, acc);
       if (lane == 0) atomicAdd(&sp.acc[f], (1ull << kAccShift) + (unsigned long long)ws);
     } else if (C0w < W && R0w < H) {
       // LDS address of entry k = pEdge/2: f32 bits of (2^21 + pEdge) + lut_q

@@ -55,13 +55,22 @@ constexpr int kLutPerTask = 32 * kWarpsT;      // LUT entries per LUT task (one 
 constexpr int kLutTasks = kLut2 / kLutPerTask;
 constexpr int kTH1 = 18;              // pass-1 output rows per warp tile (fits the same slot)
 constexpr int kRows1 = kTH1 + 2;      // pass-1 box rows: R0-1 .. R0+kTH1
+// A pass-1 task is kSub1 vertically adjacent sub-tiles (one stage each); the
+// warps carry their row window and sums from one to the next (no re-derived
+// warm-up rows, one reduction per task).  Sums stay < 2^16 per u16 half:
+// kSub1 * kTH1 * 1530 < 65536.
+#ifndef SHARP_P1_SUB
+#define SHARP_P1_SUB 2
+#endif
+constexpr int kSub1 = SHARP_P1_SUB;
+static_assert(kSub1 * kTH1 * 1530 < 65536, "pass-1 u16 sums");
 static_assert(kRows1 <= kRows2 && kSlot % 128 == 0, "pass-1 tiles fit the slots");
 // A pass-2 task is kSub vertically adjacent CTA tiles ("sub-tiles") of one
 // frame: each sub-tile fills one stage, the frame's LUT is copied once per
 // task into one of two LUT buffers (task parity), and the warps carry their
 // row window, D rows and interpolation state from one sub-tile to the next.
 #ifndef SHARP_P2_SUB
-#define SHARP_P2_SUB 3
+#define SHARP_P2_SUB 4
 #endif
 constexpr int kSub = SHARP_P2_SUB;
 #ifndef SHARP_STAGES
@@ -119,7 +128,8 @@ struct Geo {
   int per_frame;   // pass-2 tasks per frame (sub sub-tiles of kTH rows each)
   int sub;         // sub-tiles per pass-2 task (kSub; 1 when a launch has too few tasks to fill the GPU)
   int per_frame1;  // pass-1 CTA tiles per frame (th1 rows)
-  int th1;         // pass-1 rows per tile: kTH1, or 9 / 6 / 3 when a launch has too few tiles
+  int th1;         // pass-1 rows per sub-tile: kTH1, or 9 / 6 / 3 when a launch has too few tiles
+  int sub1;        // pass-1 sub-tiles per task (kSub1, or 1 with short sub-tiles)
   // Rows processed: [row_lo, row_hi) of the image (the whole image, or one
   // row band, sec. 8(e)); the tensor map's row 0 is image row y0 (a band's
   // buffer starts with its upper halo); rmax1 = min(H-2, row_hi-1) is the
@@ -351,39 +361,51 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
 // pEdge values as u16 integers: the row sums are plain 32-bit integer adds of
 // the words (each half stays < 2^16: <= 42 rows x 1530), two pixels per add,
 // three rows per IADD3 pair; no conversions.
-__device__ __forceinline__ uint32_t p1_warp(uint32_t stage, int warp, int W, int rmax1, int th1, int C0w, int R0,
-                                           int lane) {
+// One warp over a pass-1 task of nsub sub-tiles (stages s .. s+nsub-1, the
+// first already waited for); releases every stage it consumed.
+__device__ __forceinline__ uint32_t p1_warp(const Ring &ring, int s, int nsub, int warp, int W, int rmax1, int th1,
+                                           int C0w, int R0, int lane) {
   const int c0 = C0w + 8 * lane;
-  const LR aw = lane_row_s(stage, warp, lane);
+  LR aw = lane_row_s(ring.stage(s), warp, lane);
   // smem row of global row R0-1 is 0: row r -> r - R0 + 1.
   RowD ra = derive_w<false, true>(row_words(aw, 0), lane);
   RowD rb = derive_w<false, true>(row_words(aw, 1), lane);
   uint32_t acc[4] = {0u, 0u, 0u, 0u};  // acc[i] = (sum of pEdge of pair i's low pixel, ... high pixel)
 #pragma unroll 1
-  for (int m = 0; m < th1; m += 3) {
-    uint32_t pe[3][4];
-#pragma unroll
-    for (int a = 0; a < 3; ++a) {
-      const RowD rc = derive_w<false, true>(row_words(aw, m + a + 2), lane);
-      sobel(ra, rb, rc, pe[a]);
-      ra = rb;
-      rb = rc;
+  for (int k = 0; k < nsub; ++k) {
+    if (k) {  // next sub-tile: rows R0 + k th1 - 1 .. at smem row 0; the window (rows 0, 1) is carried
+      ring.release(s + k - 1, lane);
+      ring.wait_full(s + k);
+      aw = lane_row_s(ring.stage(s + k), warp, lane);
+      R0 += th1;
     }
-    // Rows 1 <= r <= rmax1 only (L160: the frame rows' pEdge is 0).  The
-    // test is warp-uniform (a vote): all three rows valid is the common case.
-    const int r = R0 + m;
-    if (__all_sync(0xffffffffu, r >= 1 && r + 2 <= rmax1)) {
+#pragma unroll 1
+    for (int m = 0; m < th1; m += 3) {
+      uint32_t pe[3][4];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) acc[i] = acc[i] + pe[0][i] + pe[1][i] + pe[2][i];
-    } else {
+      for (int a = 0; a < 3; ++a) {
+        const RowD rc = derive_w<false, true>(row_words(aw, m + a + 2), lane);
+        sobel(ra, rb, rc, pe[a]);
+        ra = rb;
+        rb = rc;
+      }
+      // Rows 1 <= r <= rmax1 only (L160: the frame rows' pEdge is 0).  The
+      // test is warp-uniform (a vote): all three rows valid is the common case.
+      const int r = R0 + m;
+      if (__all_sync(0xffffffffu, r >= 1 && r + 2 <= rmax1)) {
 #pragma unroll
-      for (int a = 0; a < 3; ++a)
-        if ((unsigned)(r + a - 1) < (unsigned)rmax1) {
+        for (int i = 0; i < 4; ++i) acc[i] = acc[i] + pe[0][i] + pe[1][i] + pe[2][i];
+      } else {
 #pragma unroll
-          for (int i = 0; i < 4; ++i) acc[i] += pe[a][i];
-        }
+        for (int a = 0; a < 3; ++a)
+          if ((unsigned)(r + a - 1) < (unsigned)rmax1) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) acc[i] += pe[a][i];
+          }
+      }
     }
   }
+  ring.release(s + nsub - 1, lane);
   // Sobel-body columns of this lane only (not the frame columns 0 / W-1, not
   // beyond the image, not the halo lanes): x = 4 (i >> 1) + (i & 1) + 2 half.
   uint32_t sum = 0;
@@ -496,8 +518,9 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       // its first stage's tile loads are issued: the loads do not need it.)
       int C0 = 0, R0 = 0, nsub = 1, nw = 0;
       if (d.x == kP1 || d.x == kP2) {
-        tile_xy(g, d.z, d.x == kP1 ? g.th1 : kTH * g.sub, C0, R0);
+        tile_xy(g, d.z, d.x == kP1 ? g.th1 * g.sub1 : kTH * g.sub, C0, R0);
         if (d.x == kP2) nsub = min(g.sub, (g.row_hi - R0 + kTH - 1) / kTH);
+        if (d.x == kP1) nsub = min(g.sub1, (g.row_hi - R0 + g.th1 - 1) / g.th1);
 #pragma unroll
         for (int w = 0; w < kWarpsT; ++w) nw += (C0 + w * kTW < g.W);
       }
@@ -506,24 +529,29 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
         if (s >= kStages) mbar_wait(ring.empty0 + 8u * b, Ring::phase(s) ^ 1u);
         // Grab the following task now: the atomic's latency overlaps this
         // task's loads and the next empty-wait.
-        if (k == 0 && d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
+#ifndef SHARP_GRAB_LATE
+#define SHARP_GRAB_LATE 1
+#endif
+        if (k == (SHARP_GRAB_LATE ? nsub - 1 : 0) && d.x != kEnd) t_next = (int)atomicAdd(sp.task_counter, 1u);
         const uint32_t full = ring.full0 + 8u * b, st = ring.stage(s);
         if (d.x == kP1) {
+          const int R0k = R0 + k * g.th1;
           if (kFused && sp.halo_on) {  // tiles at the band's edges read the neighbours' rows
             bool waited = false;
-            if (sp.up_ctl && R0 == g.row_lo) {
+            if (sp.up_ctl && R0k == g.row_lo) {
               wait_sys(sp.self_ctl + kCtlDataUp, sp.epoch);
               waited = true;
             }
-            if (sp.down_ctl && R0 + g.th1 >= g.row_hi) {
+            if (sp.down_ctl && R0k + g.th1 >= g.row_hi) {
               wait_sys(sp.self_ctl + kCtlDataDown, sp.epoch);
               waited = true;
             }
             if (waited) fence_proxy_async_global();  // peer-written rows before the TMA reads them
           }
-          stage_task[b] = make_int4(d.x, d.y, C0, R0);  // consumers get the tile origin (no division there)
+          stage_task[b] = make_int4(d.x, d.y, C0, R0k);  // consumers get the tile origin (no division there)
+          stage_aux[b] = make_int2(nsub, 0);
           mbar_expect_tx(full, tile_bytes_s(nw, kRows1));
-          tma_tiles_s(st, &map1A, &map1B, C0, nw, R0 - 1 - g.y0, d.y, full, pol_keep);
+          tma_tiles_s(st, &map1A, &map1B, C0, nw, R0k - 1 - g.y0, d.y, full, pol_keep);
         } else if (d.x == kP2) {
           const int R0k = R0 + k * kTH;
           if (kFused && sp.halo_on) {  // (tile loads go out before the LUT wait: check the halo flags here too)
@@ -650,7 +678,16 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     } else if (d.x == kP1) {
       const int C0 = d.z, R0 = d.w;
       const int C0w = C0 + warp * kTW;
-      const auto acc = (C0w < g.W) ? p1_warp(ring.stage(s), warp, g.W, g.rmax1, g.th1, C0w, R0, lane) : 0;
+      const int nsub = stage_aux[b].x;
+      uint32_t acc = 0;
+      if (C0w < g.W) {
+        acc = p1_warp(ring, s, nsub, warp, g.W, g.rmax1, g.th1, C0w, R0, lane);
+      } else {  // no columns for this warp: follow the stages
+        for (int k = 0; k < nsub; ++k) {
+          if (k) ring.wait_full(s + k);
+          ring.release(s + k, lane);
+        }
+      }
       // Reduction (sec. V-C, Fig. 9): warp-shuffle reduction, then one u64
       // atomic per warp adding (1 << 40) + partial: the frame's arrival count
       // and sum in one word, so its LUT tasks can tell when S is complete
@@ -658,6 +695,8 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
       const uint32_t ws = __reduce_add_sync(0xffffffffu, (uint32_t)acc);
       if (lane == 0) atomicAdd(&sp.acc[d.y], (1ull << kAccShift) + (unsigned long long)ws);
       if (lane == 0) TL_MAX(2);
+      s += nsub;  // (p1_warp / the loop above released the task's stages)
+      continue;
     }
     ring.release(s, lane);  // stage s may be refilled
     ++s;
@@ -791,7 +830,12 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
   sp.g.th1 = kTH1;
   while (sp.g.th1 > 3 && (long long)sg.n * sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1) < grid_ctas)
     sp.g.th1 = sp.g.th1 == kTH1 ? 9 : sp.g.th1 - 3;
-  sp.g.per_frame1 = sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1);
+  // sub-tiles per pass-1 task: kSub1 while the launch keeps >= one task per CTA
+  sp.g.sub1 = (sp.g.th1 == kTH1 &&
+               (long long)sg.n * sp.g.tiles_x * ((rows + kSub1 * kTH1 - 1) / (kSub1 * kTH1)) >= grid_ctas)
+                  ? kSub1
+                  : 1;
+  sp.g.per_frame1 = sp.g.tiles_x * ((rows + sp.g.th1 * sp.g.sub1 - 1) / (sp.g.th1 * sp.g.sub1));
   sp.mode = mode;
   sp.compact = 0;
   sp.n = sg.n;
@@ -812,31 +856,32 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     sp.L1 = sp.L2 = 0;
     sp.ntasks = (a.halo_on ? 1 : 0) + sp.g.per_frame1 + kLutTasks + sp.g.per_frame;
   } else {
-    // Lags: more tasks than can be in flight (2 stages per CTA + the CTAs'
-    // current ones) separate a frame's pass-1 tasks from its LUT tasks, and
-    // LUT tasks (a few microseconds of f64 pow/exp) are followed by >= ~2
-    // grids' worth of grabs before the frame's pass-2 tasks.
+    // Lags (in rounds): a frame's LUT tasks come L1 rounds after its pass-1
+    // tasks, its pass-2 tasks L2 rounds after them, so that dependencies are
+    // normally complete when a producer checks them.  Reference distances:
+    // the tasks the grid can hold (a current task and two stages per CTA)
+    // before the LUT, and two grids' worth of grabs more before the pass 2.
+    // A producer grabs its next task while it issues the current task's LAST
+    // stage, so a grabbed task starts about one task after the grab, and half
+    // of those distances suffice (measured, 1024 x 1080p: 0.5x 3.100 ms with
+    // 2.23 B/px of DRAM traffic -- the frames stay in L2 for their pass 2 --
+    // vs 1x 3.096 ms / 2.50 B/px; grabbing at the first stage needed 2x:
+    // 3.15 ms / 3.50 B/px).  The lag rounds past the last frame hold only
+    // empty tasks.  A dependency wait stalls one producer; it cannot
+    // deadlock -- every dependency was grabbed, and issued, earlier.
+#ifndef SHARP_LAG_X4
+#define SHARP_LAG_X4 2  // lag multiplier x 4
+#endif
     const int in_flight = 3 * grid;
-    sp.L1 = (in_flight + sp.per_round - 1) / sp.per_round + 1;
-    sp.L2 = sp.L1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
-    // The lag rounds past the last frame hold only empty tasks, so short
-    // batches use shorter lags: 2x the in-flight distance when the batch is at
-    // least that long, 1x from 4 frames on (a few empty rounds cost less than
-    // pass-2 producers stalling on their LUTs), else the minimal lags (one to
-    // three images: the empty rounds' latency would dominate).  Measured on
-    // 1080p (tools/small_batch_sweep.py): 8 frames 84 -> 61 us, 24 frames
-    // 227 -> 118 us, 1-2 frames and >= 32 frames unchanged.  A dependency
-    // wait stalls one producer; it cannot deadlock -- every dependency was
-    // grabbed, and issued, earlier.
-    const int L1u = sp.L1, L2u = sp.L2;
-    sp.L1 *= 2;  // measured: 2x the minimal lags removes most dependency waits
-    sp.L2 *= 2;
-    if (sg.n < sp.L2) {  // (1x lags from 4 frames on: a few empty rounds cost less than LUT waits)
-      sp.L1 = L1u;
-      sp.L2 = L2u;
-    }
+    const int l1 = (in_flight + sp.per_round - 1) / sp.per_round + 1;
+    const int l2 = l1 + std::max(1, (2 * grid + sp.per_round - 1) / sp.per_round);
+    sp.L1 = std::max(1, l1 * SHARP_LAG_X4 / 4);
+    sp.L2 = std::max(sp.L1 + 1, l2 * SHARP_LAG_X4 / 4);
     sp.ntasks = (sg.n + sp.L2) * sp.per_round;
-    if (sg.n < 4) {  // [pass 1 of all][LUT of all][pass 2 of all]: every dependency precedes its task
+#ifndef SHARP_COMPACT_N
+#define SHARP_COMPACT_N 32
+#endif
+    if (sg.n < SHARP_COMPACT_N) {  // [pass 1 of all][LUT of all][pass 2 of all]: every dependency precedes its task
       sp.compact = 1;
       sp.ntasks = sg.n * sp.per_round;
     }

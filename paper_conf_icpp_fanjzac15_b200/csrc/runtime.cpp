@@ -50,9 +50,14 @@ constexpr size_t kL2ChunkBudget = 24u << 20;  // input bytes per chunk kept L2-r
 constexpr size_t kHostStepChunkBudget = 48u << 20;
 constexpr int kMaxSlots = 8;
 // SHARP_PATH_AUTO's choice of the TMEM-resident kernel (launch pixels), from
-// tools/step_time.py sweeps on B200: it wins from ~1 Mpx (below, its one
-// 16-warp CTA per SM costs more than it saves) up to ~100 Mpx per launch.
-constexpr double kResAutoMinPx = 1.0e6, kResAutoMaxPx = 1.0e8;
+// tools/step_time.py sweeps on B200 (device-resident, back-to-back calls):
+// it wins from ~1 Mpx (below, its one 16-warp CTA per SM costs more than it
+// saves; 512^2: 18.5 vs 17.5 us) up to ~16 Mpx per launch (1080p x1 18.8 vs
+// 20.9 us, x2 20.5 vs 21.9, 4K x1 28.7 vs 29.7, 720p x16 49.5 vs 57.0); from
+// there the step kernel with compact / lagged schedules is as fast or faster
+// (1080p x8 41.2 vs 43.1 us, 4K x2 41.1 vs 44.2, x4 64.0 vs 75.8, x8 111 vs
+// 128; 1080p x16..48 within 1%).
+constexpr double kResAutoMinPx = 1.0e6, kResAutoMaxPx = 1.6e7;
 
 struct Slot {
   cudaStream_t stream = nullptr;
@@ -404,8 +409,8 @@ int enqueue_device(sharp_ctx *ctx, const uint8_t *din, int n, int w, int h, cons
   const bool tma = tma_family(ctx->path) && tma_ok;
   // the resident kernel (TMEM pEdge) for frames up to ~10 Mpx, else the step kernel
   // AUTO takes the resident kernel where it measured faster than the step
-  // kernel: launches of 1 .. 100 Mpx (single images from 1080p, batches up
-  // to ~48 x 1080p / 12 x 4K), else the step kernel.
+  // kernel: launches of 1 .. 16 Mpx (single images from 1080p to 4K,
+  // batches up to ~7 x 1080p), else the step kernel.
   const double px = (double)n * fb;
   // (not for the host pipeline's chunks: its slots' kernels overlap on
   // several streams, which a cooperative launch would serialise)

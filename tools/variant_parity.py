@@ -18,14 +18,14 @@ CASES = [(3, 1920, 1080), (1, 3840, 2160), (2, 1008, 36), (1, 16, 8), (1, 32, 12
          (40, 1920, 1080), (1, 1936, 1084), (2, 2000, 24)]
 
 CHILD = r'''
-import sys, numpy as np, torch
+import os, sys, numpy as np, torch
 sys.path.insert(0, ".")
 import oracle, synth
 from paper_conf_icpp_fanjzac15_b200 import Sharpener
 prm = (1.0, 0.5, 0.5, 2.0)
 bad = 0
 with Sharpener(device=0) as sh:
-    sh.set_path(1)
+    sh.set_path(int(os.environ.get("VP_PATH", "1")))
     for (n, W, H) in CASES:
         imgs = synth.frames(n, W, H, "natural", seed=synth.BASE_SEED + 7 + W + H)
         d = torch.from_numpy(imgs).cuda()
