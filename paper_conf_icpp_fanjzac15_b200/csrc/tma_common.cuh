@@ -212,7 +212,19 @@ __device__ __forceinline__ RowD derive_w(uint2 w, int lane) {
   for (int i = 0; i < 4; ++i) {
     d.c[i] = p[i];
     d.h[i] = hsub(r[i], l[i]);
-    d.s[i] = hadd(hfma(kTwo, p[i], l[i]), r[i]);
+    if (kDenorm) {
+      // s = l + 2c + r <= 1020 units: non-negative and < 2048, so its f16
+      // bit pattern is the integer itself -- two u16 lanes of plain integer
+      // adds (no carry between the halves: bytes < 2^8) instead of f16
+      // FMA-pipe ops (measured +1.4% on the 1024-frame step: pass 1 was
+      // throttled on the FMA pipe).
+      uint32_t t;
+      asm("add.u32 %0, %1, %2;" : "=r"(t) : "r"(l[i]), "r"(p[i]));
+      asm("add.u32 %0, %1, %2;" : "=r"(t) : "r"(t), "r"(p[i]));
+      asm("add.u32 %0, %1, %2;" : "=r"(d.s[i]) : "r"(t), "r"(r[i]));
+    } else {
+      d.s[i] = hadd(hfma(kTwo, p[i], l[i]), r[i]);
+    }
     if (kMinMax) {
       d.mx[i] = __vimax3_u16x2(l[i], p[i], r[i]);
       d.mn[i] = __vimin3_u16x2(l[i], p[i], r[i]);
