@@ -27,8 +27,9 @@ CSRC = os.path.join(ROOT, "paper_conf_icpp_fanjzac15_b200", "csrc")
 RULES = [
     ("table build (strength / oscStrength, L178 L184)", ["lut_entry", "lut_adj", "lut_osc", "frame_mean", "pow(", "exp("]),
     ("pass-1 accumulation + reduction (L174)", ["fma_f32_f16", "__reduce_add_sync", "atomicAdd(&sp.acc", "sum = __fadd_rn",
-                                                "vmask", "acc[x]"]),
-    ("Sobel (L158-L172)", ["hsub(", "hfma(kTwo", "habsadd", "sobel(", "gx =", "gy ="]),
+                                                "vmask", "acc[x]", "acc[i]", "sum += acc",
+                                                "r >= 1 && r + 2 <= rmax1"]),
+    ("Sobel (L158-L172)", ["hsub(", "hfma(kTwo", "habsadd", "sobel(", "gx =", "gy =", "add.u32", "d.s[i]"]),
     ("3x3 max / min (L182)", ["__vimax3", "__vimin3"]),
     ("unpack + neighbour exchange", ["kMinus1024", "kF16Bias", "__shfl_sync(0xffffffffu, O1", "__shfl_sync(0xffffffffu, E0",
                                     "prmt(PO", "prmt(O0", "prmt(E0", "prmt(E1", "row_words", "lds_u64"]),
