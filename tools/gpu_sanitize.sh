@@ -8,7 +8,7 @@ mkdir -p gpurun_out
 rm -f gpurun_out/sanitizer.txt
 for tool in memcheck racecheck synccheck initcheck; do
   echo "=== $tool" >> gpurun_out/sanitizer.txt
-  SANITIZE_TOOL=$tool timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_workload.py \
+  SANITIZE_TOOL=$tool timeout 1500 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_workload.py \
     >> gpurun_out/sanitizer.txt 2>&1
   echo "rc=$?" >> gpurun_out/sanitizer.txt
 done

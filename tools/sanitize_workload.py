@@ -30,6 +30,15 @@ for path in (SHARP_PATH_STEP, SHARP_PATH_RES, SHARP_PATH_TWO_PASS, SHARP_PATH_FU
     torch.cuda.synchronize()
     assert np.array_equal(o.cpu().numpy(), ref), path
     s.close()
+# a batch big enough for the step kernel's lagged schedule with multi-stage
+# pass-1 and pass-2 tasks (>= one 2-sub-tile / 4-sub-tile task per CTA)
+big = synth.frames(80, 480, 256, "natural", seed=synth.BASE_SEED + 4)
+s = Sharpener()
+s.set_path(SHARP_PATH_STEP)
+o = s.run_batch(torch.from_numpy(big).cuda())
+torch.cuda.synchronize()
+assert np.array_equal(o.cpu().numpy(), oracle.sharpen_batch(big)[0]), "step lagged batch"
+s.close()
 s = Sharpener()
 o = s.run(d[0])
 torch.cuda.synchronize()
