@@ -73,6 +73,11 @@ static_assert(kRows1 <= kRows2 && kSlot % 128 == 0, "pass-1 tiles fit the slots"
 #define SHARP_P2_SUB 4
 #endif
 constexpr int kSub = SHARP_P2_SUB;
+// Launches of fewer frames take the compact task order (no lag rounds).
+#ifndef SHARP_COMPACT_N
+#define SHARP_COMPACT_N 32
+#endif
+constexpr int kCompactN = SHARP_COMPACT_N;
 #ifndef SHARP_STAGES
 #define SHARP_STAGES 2  // measured: 3 stages +0.3%, 2 stages (this layout) +0.6% vs the old layout
 #endif
@@ -467,9 +472,9 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
     const unsigned long long arrivals = (unsigned long long)(g.per_frame1 * kWarpsT) << kAccShift;
     const uint64_t pol_keep = policy_evict_last(), pol_drop = policy_evict_first();
     int t_next = (int)atomicAdd(sp.task_counter, 1u);
-    // s: stages filled; j: pass-2 tasks (LUT buffer j & 1); lut_last[b]: the
+    // s: stages filled; j: pass-2 tasks (LUT buffer j & 1); lut_last0/1: the
     // last stage of the pass-2 task that used LUT buffer b.
-    int lut_last[2] = {-kStages, -kStages};
+    int lut_last0 = -kStages, lut_last1 = -kStages;  // (two scalars: no local-memory array)
     for (int s = 0, j = 0;;) {
       const int4 d = decode<kFused>(sp, t_next);
       // Resolve the task's dependency first (before waiting for a stage).
@@ -572,7 +577,7 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           // LUT buffer j & 1 is free once the stages of pass-2 task j-2 are
           // released: stages <= s - kStages are (the empty wait above); a
           // later one only after single-stage pass-2 tasks.
-          const int tl = lut_last[j & 1];
+          const int tl = (j & 1) ? lut_last1 : lut_last0;
           if (k == 0 && tl > s - kStages) mbar_wait(ring.empty0 + 8u * Ring::buf(tl), Ring::phase(tl));
           mbar_expect_tx(full, tile_bytes_s(nw, kRows2) + lut_bytes);
           // The frame's LUT (its LUT tasks were grabbed rounds earlier) is
@@ -598,7 +603,13 @@ __global__ void __launch_bounds__(kThreadsT, SHARP_LB_CTAS)
           mbar_arrive(full);
         }
       }
-      if (d.x == kP2) lut_last[j++ & 1] = s - 1;
+      if (d.x == kP2) {
+        if (j & 1)
+          lut_last1 = s - 1;
+        else
+          lut_last0 = s - 1;
+        ++j;
+      }
       if (d.x == kEnd) break;
     }
     return;
@@ -866,10 +877,7 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     sp.L1 = std::max(1, l1 * SHARP_LAG_X4 / 4);
     sp.L2 = std::max(sp.L1 + 1, l2 * SHARP_LAG_X4 / 4);
     sp.ntasks = (sg.n + sp.L2) * sp.per_round;
-#ifndef SHARP_COMPACT_N
-#define SHARP_COMPACT_N 32
-#endif
-    if (sg.n < SHARP_COMPACT_N) {  // [pass 1 of all][LUT of all][pass 2 of all]: every dependency precedes its task
+    if (sg.n < kCompactN) {  // [pass 1 of all][LUT of all][pass 2 of all]: every dependency precedes its task
       sp.compact = 1;
       sp.ntasks = sg.n * sp.per_round;
     }
