@@ -226,7 +226,7 @@ template <bool kRingRows>
 __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const RowD &rc, const float4 &V,
                                        const float4 &D0, const float4 &D1, uint32_t lut_q,
                                        uint8_t *orow, uint64_t pol_out, bool store, int r, int c0, int W, int H,
-                                       bool edge_warp, int edge) {
+                                       bool edge_warp, int edge, float cv, float dcv) {
   uint32_t pe[4], MX[4], MN[4];
   sobel(ra, rb, rc, pe);
 #pragma unroll
@@ -245,7 +245,9 @@ __device__ __forceinline__ void p2_row(const RowD &ra, const RowD &rb, const Row
   if (kRingRows && (r < 2 || r >= H - 2)) {  // warp-uniform
     ring_rows(NU, pe, MX, MN, D0, D1, r, c0, W, H, edge);
   } else if (edge_warp) {     // warp-uniform; only the edge lane changes
-    ring_cols(NU, pe, MX, MN, D0, D1, r, H, edge);
+    // the column line's -U of this row (the third-last row takes the
+    // fourth-last's, R4: one row step back; exact, multiples of 1/64)
+    ring_cols_v(NU, pe, MX, MN, r == H - 3 ? __fsub_rn(cv, dcv) : cv, edge);
   }
   float P[8], T8[8], osc[8];
 #pragma unroll
@@ -318,6 +320,7 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
   RowD ra = derive_w<true>(row_words(aw, 3), lane);
   RowD rb = derive_w<true>(row_words(aw, 4), lane);
   uint8_t *orow = out + (size_t)(R0 - row_lo) * out_pitch + c0;
+  float cv = 0.0f, dcv = 0.0f;  // ring-column line: -U of the current row, and its row step (restarted at rr % 4 == 0)
 #pragma unroll 1
   for (int k = 0; k < nsub; ++k) {
     const int R0k = R0 + k * kTH;
@@ -338,13 +341,21 @@ __device__ __forceinline__ void p2_warp(const Ring &ring, int s, int nsub, uint3
         if ((rr & 3) == 0) {  // next D block row
           D0 = D1;
           D1 = dblock(aw, sm + 4, lane);
+          // Ring columns (L140-L142 steps ii/iv/vi): the column line of D
+          // column 0 / w-1 between D rows rr/4 and rr/4 + 1 is linear in the
+          // row: -U = -x0/16 - k (x1 - x0)/64 at row 4i + k, kept as cv += dcv
+          // (exact: multiples of 1/64 below 256).
+          const float x0 = edge == 1 ? D0.y : D0.z, x1 = edge == 1 ? D1.y : D1.z;
+          cv = -div16(x0);
+          dcv = __fmul_rn(__fsub_rn(x0, x1), 1.0f / 64.0f);
         } else if ((rr & 3) == 2) {  // next interpolation interval: D rows (k, k+1)
           V = f4fma(7.0f, D0, D1);
           slope = f4twice_diff(D1, D0);
         }
         const RowD rc = derive_w<true>(row_words(aw, sm + 1), lane);
-        p2_row<true>(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge);
+        p2_row<true>(ra, rb, rc, V, D0, D1, lut_q, orow, pol_out, rr < rend_l, rr, c0, W, H, edge_warp, edge, cv, dcv);
         V = f4add(V, slope);
+        cv = __fadd_rn(cv, dcv);
         orow += out_pitch;
         ra = rb;
         rb = rc;

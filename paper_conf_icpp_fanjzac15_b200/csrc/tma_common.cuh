@@ -290,6 +290,20 @@ __device__ __forceinline__ void ring_rows(float NU[8], uint32_t pe[4], uint32_t 
     }
   }
 }
+// The same with the column line's value given: v = -U of this row (the step
+// kernel keeps it incrementally, sec. 7.1 of DESIGN.md).
+__device__ __forceinline__ void ring_cols_v(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4], float v,
+                                            int edge) {
+  if (edge == 1) {
+    NU[0] = v;
+    NU[1] = v;
+    set_frame_px(pe, MX, MN, 0);
+  } else if (edge == 2) {
+    NU[6] = v;
+    NU[7] = v;
+    set_frame_px(pe, MX, MN, 7);
+  }
+}
 // Columns 0,1 / W-2,W-1 on rows 2..H-3 (lines of D columns 0 / w-1).
 __device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4],
                                           const float4 &D0, const float4 &D1, int r, int H, int edge) {
@@ -308,7 +322,17 @@ __device__ __forceinline__ void ring_cols(float NU[8], uint32_t pe[4], uint32_t 
   }
 }
 
+#ifndef SHARP_F4_PACKED
+#define SHARP_F4_PACKED 1
+#endif
 __device__ __forceinline__ float4 f4fma(float a, const float4 &x, const float4 &y) {  // a*x + y, exact here
+  if (SHARP_F4_PACKED) {  // two packed f32x2 FMAs (single rounding per lane, as the scalar form)
+    unsigned long long lo, hi;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(lo) : "l"(f2pack(a, a)), "l"(f2pack(x.x, x.y)), "l"(f2pack(y.x, y.y)));
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(hi) : "l"(f2pack(a, a)), "l"(f2pack(x.z, x.w)), "l"(f2pack(y.z, y.w)));
+    const float2 l = f2unpack(lo), h = f2unpack(hi);
+    return make_float4(l.x, l.y, h.x, h.y);
+  }
   return make_float4(__fmaf_rn(a, x.x, y.x), __fmaf_rn(a, x.y, y.y), __fmaf_rn(a, x.z, y.z), __fmaf_rn(a, x.w, y.w));
 }
 __device__ __forceinline__ float4 f4add(const float4 &x, const float4 &y) {  // two packed f32x2 adds
@@ -319,6 +343,15 @@ __device__ __forceinline__ float4 f4add(const float4 &x, const float4 &y) {  // 
   return make_float4(a.x, a.y, b.x, b.y);
 }
 __device__ __forceinline__ float4 f4twice_diff(const float4 &x, const float4 &y) {  // 2 (x - y), exact here
+  if (SHARP_F4_PACKED) {  // packed sub then packed mul (exact: integers < 2^13)
+    unsigned long long lo, hi;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(lo) : "l"(f2pack(x.x, x.y)), "l"(f2pack(y.x, y.y)));
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(hi) : "l"(f2pack(x.z, x.w)), "l"(f2pack(y.z, y.w)));
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(lo) : "l"(lo), "l"(f2pack(2.0f, 2.0f)));
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(hi) : "l"(hi), "l"(f2pack(2.0f, 2.0f)));
+    const float2 l = f2unpack(lo), h = f2unpack(hi);
+    return make_float4(l.x, l.y, h.x, h.y);
+  }
   return make_float4(__fmul_rn(2.0f, __fsub_rn(x.x, y.x)), __fmul_rn(2.0f, __fsub_rn(x.y, y.y)),
                      __fmul_rn(2.0f, __fsub_rn(x.z, y.z)), __fmul_rn(2.0f, __fsub_rn(x.w, y.w)));
 }
