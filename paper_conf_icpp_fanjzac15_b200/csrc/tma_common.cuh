@@ -261,6 +261,30 @@ __device__ __forceinline__ void set_frame_px(uint32_t pe[4], uint32_t MX[4], uin
   set_px(MX, x, kF16_255);   // overshoot frame: the clamped preliminary value,
   set_px(MN, x, 0u);         // i.e. window [0, 255]
 }
+// The frame columns 0 / W-1 of the edge lanes (L160, L208): pEdge 0, window
+// [0, 255]; column 0 is the low half of pair 0, W-1 the high half of pair 3.
+// Selects, not branches: no lane-divergent control flow in the row loop.
+__device__ __forceinline__ void frame_cols(uint32_t pe[4], uint32_t MX[4], uint32_t MN[4], int edge) {
+  const bool e1 = edge == 1, e2 = edge == 2;
+  const uint32_t k0 = e1 ? 0xffff0000u : 0xffffffffu, k3 = e2 ? 0x0000ffffu : 0xffffffffu;
+  pe[0] &= k0;
+  MN[0] &= k0;
+  MX[0] = (MX[0] & k0) | (e1 ? kF16_255 : 0u);
+  pe[3] &= k3;
+  MN[3] &= k3;
+  MX[3] = (MX[3] & k3) | (e2 ? (kF16_255 << 16) : 0u);
+}
+// Columns 0,1 / W-2,W-1 on rows 2..H-3 with the column line's value given:
+// v = -U of this row (the step kernel keeps it incrementally).
+__device__ __forceinline__ void ring_cols_v(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4], float v,
+                                            int edge) {
+  const bool e1 = edge == 1, e2 = edge == 2;
+  NU[0] = e1 ? v : NU[0];
+  NU[1] = e1 ? v : NU[1];
+  NU[6] = e2 ? v : NU[6];
+  NU[7] = e2 ? v : NU[7];
+  frame_cols(pe, MX, MN, edge);
+}
 // Rows 0,1 (line of D row 0) and H-2,H-1 (line of D row h-1): here D0 is
 // that D row; the corners follow the step order (v)-(vii).
 __device__ __forceinline__ void ring_rows(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4],
@@ -269,18 +293,17 @@ __device__ __forceinline__ void ring_rows(float NU[8], uint32_t pe[4], uint32_t 
   const float q0 = D0.y, q1 = D0.z, q2 = D0.w;
   float u[8] = {div16(q0),         line_val(q0, q1, 1), line_val(q0, q1, 2), line_val(q0, q1, 3),
                 div16(q1),         line_val(q1, q2, 1), line_val(q1, q2, 2), line_val(q1, q2, 3)};
-  if (c0 + 5 == W - 3) u[5] = div16(q1);  // third last <- fourth last
+  // (lane-dependent choices as selects: no divergent control flow in the row loop)
+  u[5] = (c0 + 5 == W - 3) ? div16(q1) : u[5];  // third last <- fourth last
   const bool top = r < 2;
-  if (edge == 1 && top) u[1] = div16(q0);  // (v)+(vi): top-left 2x2 = D[0][0]
-  if (edge == 2) {                         // columns W-2, W-1 (D column w-1 = j0+1)
-    const float v = (top && r == 1) ? line_val(D0.z, D1.z, 1) : div16(D0.z);
-    u[6] = v;
-    u[7] = v;
-  }
+  u[1] = (edge == 1 && top) ? div16(q0) : u[1];  // (v)+(vi): top-left 2x2 = D[0][0]
+  // columns W-2, W-1 (D column w-1 = j0+1)
+  const float v = (top && r == 1) ? line_val(D0.z, D1.z, 1) : div16(D0.z);
+  u[6] = edge == 2 ? v : u[6];
+  u[7] = edge == 2 ? v : u[7];
 #pragma unroll
   for (int x = 0; x < 8; ++x) NU[x] = -u[x];
-  if (edge == 1) set_frame_px(pe, MX, MN, 0);  // column 0 (rows 1, H-2)
-  if (edge == 2) set_frame_px(pe, MX, MN, 7);  // column W-1
+  frame_cols(pe, MX, MN, edge);  // column 0 / W-1 (rows 1, H-2)
   if (r == 0 || r == H - 1) {
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
@@ -288,20 +311,6 @@ __device__ __forceinline__ void ring_rows(float NU[8], uint32_t pe[4], uint32_t 
       MX[i] = kF16_255 | (kF16_255 << 16);
       MN[i] = 0u;
     }
-  }
-}
-// The same with the column line's value given: v = -U of this row (the step
-// kernel keeps it incrementally, sec. 7.1 of DESIGN.md).
-__device__ __forceinline__ void ring_cols_v(float NU[8], uint32_t pe[4], uint32_t MX[4], uint32_t MN[4], float v,
-                                            int edge) {
-  if (edge == 1) {
-    NU[0] = v;
-    NU[1] = v;
-    set_frame_px(pe, MX, MN, 0);
-  } else if (edge == 2) {
-    NU[6] = v;
-    NU[7] = v;
-    set_frame_px(pe, MX, MN, 7);
   }
 }
 // Columns 0,1 / W-2,W-1 on rows 2..H-3 (lines of D columns 0 / w-1).
