@@ -137,10 +137,14 @@ def test_batch_frames_independent_and_equal_to_oracle(sh):
     assert sums == [int(s) for s in ref_sums]
 
 
-@pytest.mark.parametrize("n,W,H", [(1, 16, 8), (3, 16, 16), (40, 256, 40), (9, 976, 44), (2, 3840, 2160)])
+@pytest.mark.parametrize("n,W,H", [(1, 16, 8), (3, 16, 16), (40, 256, 40), (9, 976, 44), (2, 3840, 2160),
+                                   (20, 976, 100), (80, 480, 260)])
 def test_batch_single_launch_dependencies(n, W, H):
     """TMA batch kernel: pass 1 -> LUT -> pass 2 dependencies resolved inside
-    one launch (rounds with lags; empty tasks at the ends)."""
+    one launch (rounds with lags; empty tasks at the ends).  (20, 976, 100):
+    the compact order of a mid-size batch; (80, 480, 260): the lagged order
+    with 2-sub-tile pass-1 and 4-sub-tile pass-2 tasks and ragged last tasks
+    (260 = 7 x 36 + 8 = 5 x 48 + 20 rows)."""
     imgs = synth.frames(n, W, H, "natural", seed=n * 7 + W)
     with Sharpener() as s:
         d = torch.from_numpy(imgs).cuda()
