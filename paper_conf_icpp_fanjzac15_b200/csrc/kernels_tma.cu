@@ -17,9 +17,13 @@
 // fills a stage) normally complete long before they are needed; a frame's
 // input is re-read by pass 2 from L2 (pass-1 loads carry evict_last).
 //
-// CTA = 4 compute warps + 1 producer warp.  A pass-1/2 task is a CTA tile of
-// 4 warp tiles side by side; a warp tile is 240 output columns x 12 rows
-// (pass 2) or 18 rows (pass 1).  The producer issues one 256-column TMA box
+// CTA = 4 compute warps + 1 producer warp.  A pass-1/2 task is a column of
+// CTA tiles ("sub-tiles", one smem stage each: 4 warp tiles side by side of
+// 240 output columns x 12 rows for pass 2, x 18 rows for pass 1): 4 pass-2 /
+// 2 pass-1 sub-tiles per task in big launches, the warps carrying their row
+// window and sums from one sub-tile to the next.  The producer grabs its next
+// task while issuing the current task's last stage, so the dependency lags
+// stay short and a frame is still in L2 when its pass 2 re-reads it.  The producer issues one 256-column TMA box
 // per warp tile (out-of-image pixels are zero-filled: no bounds checks in the
 // pixel loops) plus a bulk copy of the frame's LUT, into one of two smem stages
 // guarded by full/empty mbarriers -- no CTA-wide barrier in the steady state.
