@@ -137,7 +137,7 @@ struct Geo {
   int per_frame;   // pass-2 tasks per frame (sub sub-tiles of kTH rows each)
   int sub;         // sub-tiles per pass-2 task (kSub; 1 when a launch has too few tasks to fill the GPU)
   int per_frame1;  // pass-1 CTA tiles per frame (th1 rows)
-  int th1;         // pass-1 rows per sub-tile: kTH1, or 9 / 6 / 3 when a launch has too few tiles
+  int th1;         // pass-1 rows per sub-tile: kTH1, or 9 when a launch has too few tiles
   int sub1;        // pass-1 sub-tiles per task (kSub1, or 1 with short sub-tiles)
   // Rows processed: [row_lo, row_hi) of the image (the whole image, or one
   // row band, sec. 8(e)); the tensor map's row 0 is image row y0 (a band's
@@ -840,9 +840,14 @@ cudaError_t launch_step(const BatchLaunch &a, const StepGeometry &sg, int mode, 
     if ((t1 + grid_ctas - 1) / grid_ctas < kSub * ((ts + grid_ctas - 1) / grid_ctas)) sp.g.sub = 1;
   }
   sp.g.per_frame = sp.g.tiles_x * ((rows + kTH * sp.g.sub - 1) / (kTH * sp.g.sub));
-  // pass-1 tiles: as tall as kTH1 while the launch has >= one tile per CTA
+  // pass-1 tiles: as tall as kTH1 while the launch has >= one tile per CTA,
+  // but not below 9 rows (3- and 6-row tiles are mostly warm-up rows and task
+  // overhead: 512^2 17.6 -> 17.0 us, one 1080p 20.7 -> 19.0 us with 9)
   sp.g.th1 = kTH1;
-  while (sp.g.th1 > 3 && (long long)sg.n * sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1) < grid_ctas)
+#ifndef SHARP_MIN_TH1
+#define SHARP_MIN_TH1 9
+#endif
+  while (sp.g.th1 > SHARP_MIN_TH1 && (long long)sg.n * sp.g.tiles_x * ((rows + sp.g.th1 - 1) / sp.g.th1) < grid_ctas)
     sp.g.th1 = sp.g.th1 == kTH1 ? 9 : sp.g.th1 - 3;
   // sub-tiles per pass-1 task: kSub1 while the launch keeps >= one task per CTA
   sp.g.sub1 = (sp.g.th1 == kTH1 &&
