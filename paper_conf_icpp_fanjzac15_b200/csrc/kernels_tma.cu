@@ -399,6 +399,10 @@ __device__ __forceinline__ uint32_t p1_warp(const Ring &ring, int s, int nsub, i
       aw = lane_row_s(ring.stage(s + k), warp, lane);
       R0 += th1;
     }
+    // rows 1 <= r <= rmax1 only (L160: the frame rows' pEdge is 0): decided
+    // once per sub-tile (a vote: warp-uniform) -- every row valid is the
+    // common case; only sub-tiles at the image's top / bottom test per row
+    const bool all_rows = __all_sync(0xffffffffu, R0 >= 1 && R0 + th1 - 1 <= rmax1);
 #pragma unroll 1
     for (int m = 0; m < th1; m += 3) {
       uint32_t pe[3][4];
@@ -409,10 +413,8 @@ __device__ __forceinline__ uint32_t p1_warp(const Ring &ring, int s, int nsub, i
         ra = rb;
         rb = rc;
       }
-      // Rows 1 <= r <= rmax1 only (L160: the frame rows' pEdge is 0).  The
-      // test is warp-uniform (a vote): all three rows valid is the common case.
       const int r = R0 + m;
-      if (__all_sync(0xffffffffu, r >= 1 && r + 2 <= rmax1)) {
+      if (all_rows) {
 #pragma unroll
         for (int i = 0; i < 4; ++i) acc[i] = acc[i] + pe[0][i] + pe[1][i] + pe[2][i];
       } else {
